@@ -1,0 +1,332 @@
+#!/usr/bin/env python
+"""Benchmark: SPN inference samples/s on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2]
+                    [--marginal] [--impl ours|reference]
+
+A step is one pass of the whole hot path (spn_infer_* over one batch of the
+config's N samples, inputs resident in HBM).  Default workload: config C2 (a
+speaker-ID-shaped Gaussian SPN over 26 features, 1M samples, joint), the
+configuration the metric is quoted on that fits one GPU.  At N GPUs each rank
+processes its own N-sample batch (weak scaling, no data-path collective).
+L2 is flushed (256 MiB write) between timed steps.  Prints ONE JSON line on
+rank 0.  ``--impl reference`` times the fp64 CPU oracle (the reference arm of
+this tier) on bounded samples of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SPN inference samples/sec (joint & marginal) at 1/2/4/8 B200; % of HBM/MUFU roofline"
+UNIT = "samples/s"
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def make_workload(cfg: str, rank: int, marginal: bool):
+    """Seeded graph + this rank's input batch (host numpy)."""
+    from spn_inputs import (CONFIGS, config_graph, ancestral_sample, add_outliers, nan_mask,
+                            toy_data, uniform_chunked)
+    c = CONFIGS[cfg]
+    g = config_graph(cfg)
+    n = c["n_samples"]
+    if cfg == "C1":
+        x = toy_data(n, seed=1001 + rank)
+        if marginal:
+            x = nan_mask(x, 0.2, 1002 + rank)
+    elif cfg == "C2":
+        x, _ = ancestral_sample(g, n, c["data_seed"] + 1000 * rank)
+        x = add_outliers(x, 0.01, c["data_seed"] + 1 + 1000 * rank)
+        if marginal:
+            x = nan_mask(x, 0.2, c["data_seed"] + 2 + 1000 * rank)
+    elif cfg == "C3":
+        x, _ = ancestral_sample(g, n, c["data_seed"] + 1000 * rank)
+        x = nan_mask(x, c["nan_p"], c["nan_seed"] + 1000 * rank)
+    else:
+        x = uniform_chunked(n, g.n_features, c["data_seed"], start=rank * n)
+    return g, x, n
+
+
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks / throttle reasons during a region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.path = os.path.join("/tmp", f"spnb_clocks_{os.getpid()}.csv")
+
+    def start(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "50"], stdout=self.f,
+                stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.12)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.close()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def cpu_baseline(g, x, marginal, target_s=12.0):
+    """The oracle as it stands, timed on this host's cores on a bounded
+    sample (~target_s seconds)."""
+    from oracle import oracle_eval, num_threads
+    n0 = min(len(x), 2000)
+    t = time.perf_counter()
+    oracle_eval(g, x[:n0], marginal=marginal)
+    dt = time.perf_counter() - t
+    n = int(min(len(x), max(n0, n0 * target_s / max(dt, 1e-6))))
+    t = time.perf_counter()
+    oracle_eval(g, x[:n], marginal=marginal)
+    dt = time.perf_counter() - t
+    return {"value": n / dt, "unit": UNIT, "cores": num_threads(), "kind": "oracle",
+            "sample": f"first {n} of the {len(x)} samples of this workload, "
+                      f"fp64 recursive oracle, {dt:.1f} s"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import oracle_eval, num_threads, build_oracle
+    build_oracle()
+    g, x, n = make_workload(args.config, 0, args.marginal)
+    # per step: a bounded sample sized so the whole run takes a few minutes
+    n0 = min(n, 1000)
+    t = time.perf_counter()
+    oracle_eval(g, x[:n0], marginal=args.marginal)
+    per = (time.perf_counter() - t) / n0
+    budget = 150.0 / max(1, args.steps + args.warmup)
+    m = int(max(100, min(n, budget / max(per, 1e-9))))
+    for i in range(args.warmup):
+        oracle_eval(g, x[:m], marginal=args.marginal)
+    ts = []
+    for i in range(args.steps):
+        off = (i * m) % max(1, n - m + 1)
+        t = time.perf_counter()
+        oracle_eval(g, x[off:off + m], marginal=args.marginal)
+        ts.append(time.perf_counter() - t)
+    tot = sum(ts)
+    val = m * args.steps / tot
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT,
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": _config_dict(args, g, n),
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": num_threads(),
+                             "kind": "oracle",
+                             "sample": f"{m} samples per step of the {args.config} workload"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def _config_dict(args, g, n):
+    from spn_inputs import CONFIGS
+    c = g.counts()
+    return {"workload": f"{args.config}: {CONFIGS[args.config]['desc']}",
+            "query": "marginal" if args.marginal else "joint",
+            "samples_per_gpu": n, "n_features": g.n_features, "n_roots": g.n_roots,
+            "graph_nodes": c["nodes"], "sum_edges": c["sum_edges"],
+            "l2": "flushed between timed steps (256 MiB write)",
+            "parallelism": f"dp{args.gpus} (sample sharding)"}
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+
+    from paper_conf_cgo_sommera022_b200.build import build
+    if rank == 0:
+        build()
+    if world > 1:
+        dist.barrier()
+    import paper_conf_cgo_sommera022_b200 as spnb
+
+    g, x, n = make_workload(args.config, rank, args.marginal)
+    G = spnb.Graph(g)
+    t0 = time.perf_counter()
+    P = spnb.Plan(G, device=local, samples_per_thread=args.K, block_threads=args.block)
+    prep_s = time.perf_counter() - t0
+    info = P.info()
+    xd = torch.from_numpy(x).to(dev)
+    R = g.n_roots
+    want_am = R > 1
+    out = torch.empty((n, R), dtype=torch.float32, device=dev)
+    am = torch.empty((n,), dtype=torch.int32, device=dev) if want_am else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    st = torch.cuda.current_stream(dev)
+
+    def step():
+        P.infer(xd, marginal=args.marginal, out=out, argmax=am, want_argmax=want_am, stream=st)
+
+    for _ in range(max(3, args.warmup)):
+        flush.fill_(1)
+        step()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    clocks.start()
+    # keep the GPU busy ~0.5 s before the timed region so clocks settle
+    t_end = time.perf_counter() + 0.5
+    while time.perf_counter() < t_end:
+        step()
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    for i in range(args.steps):
+        flush.fill_(i & 0xff)
+        evs[i][0].record(st)
+        step()
+        evs[i][1].record(st)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    times = [a.elapsed_time(b) for a, b in evs]          # ms, kernel-only per step
+    tot_ms = sum(times)
+    t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    tot_ms = float(t.item())
+    value = n * world * args.steps / (tot_ms / 1e3)
+
+    # ---- end to end through the public host-buffer API (H2D + D2H inside) ----
+    xh = torch.from_numpy(x).pin_memory()
+    oh = torch.empty((n, R), dtype=torch.float32).pin_memory()
+    amh = torch.empty((n,), dtype=torch.int32).pin_memory() if want_am else None
+    P.infer_host(xh, marginal=args.marginal, out=oh, argmax=amh, want_argmax=want_am)
+    e2e_steps = max(1, min(args.steps, 10))
+    if world > 1:
+        dist.barrier()
+    t_e = time.perf_counter()
+    for _ in range(e2e_steps):
+        P.infer_host(xh, marginal=args.marginal, out=oh, argmax=amh, want_argmax=want_am)
+    e2e_s = (time.perf_counter() - t_e) / e2e_steps
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_val = n * world / float(te.item())
+
+    if rank == 0:
+        peaks, src = _peaks()
+        ms = tot_ms / args.steps
+        clock_mhz = peaks.get("sm_max_mhz", 1965.0)
+        mufu_peak = 16 * 148 * clock_mhz * 1e6          # MUFU ops/s (16/clk/SM)
+        mufu = info["mufu_per_sample"] * n / (ms / 1e3)
+        hbm = info["bytes_per_sample"] * n / (ms / 1e3) / 1e9
+        prof = os.path.join(ROOT, "profiles", f"ncu_{args.config}.json")
+        traffic = None
+        if os.path.exists(prof):
+            with open(prof) as f:
+                traffic = json.load(f).get("dram_bytes_per_launch")
+        roof = {"bound": "alu", "pipe": "MUFU ex2/lg2 (16 op/clk/SM)",
+                "achieved": mufu / 1e9, "peak": mufu_peak / 1e9, "unit": "Gop/s",
+                "frac": mufu / mufu_peak, "traffic": traffic,
+                "peak_source": f"16 MUFU/clk/SM x 148 SMs x {clock_mhz:.0f} MHz "
+                               f"(sm_max_mhz, {src})",
+                "hbm": {"achieved": hbm, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                        "frac": hbm / peaks["hbm_gbs"]}}
+        cpu = cpu_baseline(g, x, args.marginal) if world == 1 or True else None
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f32", "data": "synthetic (seeded ancestral samples)",
+                "config": _config_dict(args, g, n) | {
+                    "plan": {k: info[k] for k in ("n_nodes", "n_tasks", "n_records",
+                                                  "block_threads", "samples_per_thread",
+                                                  "grid", "smem_bytes", "mufu_per_sample",
+                                                  "max_stack")},
+                    "prepare_s": prep_s},
+                "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
+                "e2e": {"value": e2e_val, "unit": UNIT,
+                        "h2d_bytes_per_step": int(x.nbytes),
+                        "d2h_bytes_per_step": int(n * R * 4 + (n * 4 if want_am else 0)),
+                        "timing": "wall clock around the synchronous host-buffer call"},
+                "gpu_launches": args.steps,
+                "step_ms": {"min": min(times), "median": statistics.median(times),
+                            "max": max(times)}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--marginal", action="store_true")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--K", type=int, default=0, help="samples per thread (0 = auto)")
+    ap.add_argument("--block", type=int, default=0, help="threads per CTA (0 = auto)")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,557 @@
+// api.cpp -- the C ABI of libspnb (include/spnb.h): handles, validation,
+// plan preparation (launch-configuration choice + device upload), inference
+// launches and the host-buffer end-to-end pipeline.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "prepare.h"
+#include "program.h"
+#include "spnb.h"
+
+namespace spnb {
+cudaError_t dag_eval_launch_k1(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
+cudaError_t dag_eval_launch_k2(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
+cudaError_t dag_eval_launch_k4(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
+int dag_eval_occupancy_k1(bool, bool, int, size_t);
+int dag_eval_occupancy_k2(bool, bool, int, size_t);
+int dag_eval_occupancy_k4(bool, bool, int, size_t);
+}  // namespace spnb
+
+using namespace spnb;
+
+namespace {
+
+thread_local std::string t_err;
+
+int set_err(int code, const std::string &m) {
+    t_err = m;
+    return code;
+}
+int cuda_err(cudaError_t e, const char *where) {
+    return set_err(SPN_E_CUDA, std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+enum { H_GRAPH = 0x47524150, H_PLAN = 0x504c414e };
+
+struct DevicePlan {
+    int device = 0;
+    int K = 4;
+    bool xs = true;
+    int tpw = 132;
+    int block = 384;
+    int grid_max = 0;        // persistent grid upper bound (SMs x CTAs/SM)
+    int sms = 0;
+    size_t smem = 0;
+    int prog_cap = 0;
+    int32_t F = 0, R = 0;
+    int32_t n_tasks = 1;
+    int32_t first_task_len = 0;
+    int64_t n_sslots = 0, n_gslots = 0;
+    Rec *d_prog = nullptr;
+    int64_t *d_task_off = nullptr;
+    float *d_tables = nullptr;
+    Edge *d_edges = nullptr;
+    float *d_gslots = nullptr;
+    // host pipeline buffers (lazily allocated)
+    std::mutex host_mu;
+    cudaStream_t hs[2] = {nullptr, nullptr};
+    float *hx[2] = {nullptr, nullptr};
+    float *hout[2] = {nullptr, nullptr};
+    int32_t *ham[2] = {nullptr, nullptr};
+    int64_t host_chunk = 0;
+    spn_plan_stats stats;
+};
+
+}  // namespace
+
+struct spn_handle {
+    uint32_t magic;
+    GraphData *graph = nullptr;
+    DevicePlan *plan = nullptr;
+};
+
+namespace {
+
+int launch_kernel(const KParams &p, int K, bool marg, bool xs, int grid, int block, size_t smem,
+                  cudaStream_t st) {
+    cudaError_t e;
+    switch (K) {
+        case 4: e = dag_eval_launch_k4(p, marg, xs, grid, block, smem, st); break;
+        case 2: e = dag_eval_launch_k2(p, marg, xs, grid, block, smem, st); break;
+        case 1: e = dag_eval_launch_k1(p, marg, xs, grid, block, smem, st); break;
+        default: return set_err(SPN_E_ARG, "bad samples_per_thread");
+    }
+    if (e != cudaSuccess) return cuda_err(e, "dag_eval launch");
+    return SPN_OK;
+}
+
+int occupancy(int K, bool marg, bool xs, int block, size_t smem) {
+    switch (K) {
+        case 4: return dag_eval_occupancy_k4(marg, xs, block, smem);
+        case 2: return dag_eval_occupancy_k2(marg, xs, block, smem);
+        case 1: return dag_eval_occupancy_k1(marg, xs, block, smem);
+    }
+    return 0;
+}
+
+void free_plan(DevicePlan *p) {
+    if (!p) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(p->device);
+    cudaFree(p->d_prog);
+    cudaFree(p->d_task_off);
+    cudaFree(p->d_tables);
+    cudaFree(p->d_edges);
+    cudaFree(p->d_gslots);
+    for (int i = 0; i < 2; ++i) {
+        if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
+        cudaFree(p->hx[i]);
+        cudaFree(p->hout[i]);
+        cudaFree(p->ham[i]);
+    }
+    if (prev >= 0) cudaSetDevice(prev);
+    delete p;
+}
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+template <typename T>
+int upload(T **dst, const std::vector<T> &v) {
+    const size_t bytes = std::max<size_t>(v.size(), 1) * sizeof(T);
+    cudaError_t e = cudaMalloc((void **)dst, bytes);
+    if (e != cudaSuccess) return e == cudaErrorMemoryAllocation ? set_err(SPN_E_OOM, "cudaMalloc")
+                                                                 : cuda_err(e, "cudaMalloc");
+    if (!v.empty()) {
+        e = cudaMemcpy(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return cuda_err(e, "cudaMemcpy");
+    }
+    return SPN_OK;
+}
+
+int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
+                 int32_t *argmax, void *stream, bool marg) {
+    if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
+    DevicePlan &P = *h->plan;
+    if (n < 0) return set_err(SPN_E_ARG, "n < 0");
+    if (n == 0) return SPN_OK;
+    if (!x || !out) return set_err(SPN_E_ARG, "null x/out");
+    if (ld < P.F) return set_err(SPN_E_ARG, "ld < n_features");
+    DeviceGuard dg(P.device);
+    KParams kp;
+    memset(&kp, 0, sizeof(kp));
+    kp.prog = P.d_prog;
+    kp.task_off = P.d_task_off;
+    kp.n_tasks = P.n_tasks;
+    kp.prog_cap = P.prog_cap;
+    kp.first_task_len = P.first_task_len;
+    kp.tables = P.d_tables;
+    kp.edges = P.d_edges;
+    kp.x = x;
+    kp.n = n;
+    kp.ld = ld;
+    kp.F = P.F;
+    kp.R = P.R;
+    kp.out = out;
+    kp.argmax = argmax;
+    kp.gslots = P.d_gslots;
+    kp.n_gslots = (int32_t)P.n_gslots;
+    kp.n_sslots = (int32_t)P.n_sslots;
+    kp.x_in_smem = P.xs;
+    kp.tpw = P.tpw;
+    const int WT = 32 * P.K;
+    kp.n_wtiles = (n + WT - 1) / WT;
+    const int nwarps = P.block / 32;
+    int64_t need;
+    if (P.n_tasks == 1) need = (kp.n_wtiles + nwarps - 1) / nwarps;
+    else need = (n + (int64_t)nwarps * WT - 1) / ((int64_t)nwarps * WT);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, P.grid_max));
+    return launch_kernel(kp, P.K, marg, P.xs, grid, P.block, P.smem, (cudaStream_t)stream);
+}
+
+int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out, int32_t *argmax,
+               bool marg) {
+    if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
+    DevicePlan &P = *h->plan;
+    if (n < 0) return set_err(SPN_E_ARG, "n < 0");
+    if (n == 0) return SPN_OK;
+    if (!x || !out) return set_err(SPN_E_ARG, "null x/out");
+    if (ld < P.F) return set_err(SPN_E_ARG, "ld < n_features");
+    std::lock_guard<std::mutex> lk(P.host_mu);
+    DeviceGuard dg(P.device);
+    cudaError_t e;
+    if (!P.hs[0]) {
+        // chunk sized to ~32 MB of features: big enough to amortise launches,
+        // small enough to overlap H2D / kernel / D2H across the two streams
+        P.host_chunk = std::max<int64_t>(4096, ((int64_t)(32 << 20) / (4 * P.F)) & ~int64_t(4095));
+        for (int i = 0; i < 2; ++i) {
+            if ((e = cudaStreamCreateWithFlags(&P.hs[i], cudaStreamNonBlocking)) != cudaSuccess)
+                return cuda_err(e, "cudaStreamCreate");
+            if ((e = cudaMalloc(&P.hx[i], (size_t)P.host_chunk * P.F * 4)) != cudaSuccess ||
+                (e = cudaMalloc(&P.hout[i], (size_t)P.host_chunk * P.R * 4)) != cudaSuccess ||
+                (e = cudaMalloc(&P.ham[i], (size_t)P.host_chunk * 4)) != cudaSuccess)
+                return set_err(SPN_E_OOM, "host pipeline buffers");
+        }
+    }
+    const int64_t C = P.host_chunk;
+    int rc = SPN_OK;
+    for (int64_t c0 = 0, i = 0; c0 < n; c0 += C, ++i) {
+        const int s = (int)(i & 1);
+        const int64_t m = std::min(C, n - c0);
+        cudaStream_t st = P.hs[s];
+        e = cudaMemcpy2DAsync(P.hx[s], (size_t)P.F * 4, x + c0 * ld, (size_t)ld * 4,
+                              (size_t)P.F * 4, (size_t)m, cudaMemcpyHostToDevice, st);
+        if (e != cudaSuccess) return cuda_err(e, "H2D");
+        rc = infer_device(h, P.hx[s], m, P.F, P.hout[s], argmax ? P.ham[s] : nullptr, st, marg);
+        if (rc != SPN_OK) return rc;
+        e = cudaMemcpyAsync(out + c0 * P.R, P.hout[s], (size_t)m * P.R * 4,
+                            cudaMemcpyDeviceToHost, st);
+        if (e != cudaSuccess) return cuda_err(e, "D2H");
+        if (argmax) {
+            e = cudaMemcpyAsync(argmax + c0, P.ham[s], (size_t)m * 4, cudaMemcpyDeviceToHost, st);
+            if (e != cudaSuccess) return cuda_err(e, "D2H argmax");
+        }
+    }
+    for (int i = 0; i < 2; ++i)
+        if ((e = cudaStreamSynchronize(P.hs[i])) != cudaSuccess) return cuda_err(e, "sync");
+    return SPN_OK;
+}
+
+bool valid_graph_handle(const spn_handle *h) { return h && h->magic == H_GRAPH && h->graph; }
+
+}  // namespace
+
+extern "C" {
+
+void spn_default_options(spn_prepare_options *opt) {
+    if (!opt) return;
+    memset(opt, 0, sizeof(*opt));
+    opt->device = -1;
+}
+
+const char *spn_last_error(void) { return t_err.c_str(); }
+
+int spn_load_graph(const spn_node *nodes, int64_t n_nodes, const int64_t *children,
+                   const double *weights, int64_t n_edges, const double *params,
+                   int64_t n_params, const int64_t *roots, int32_t n_roots, int32_t n_features,
+                   spn_handle **out_graph) {
+    if (!out_graph) return set_err(SPN_E_ARG, "out_graph is NULL");
+    *out_graph = nullptr;
+    if (n_nodes < 0 || n_edges < 0 || n_params < 0 || n_roots < 1 || n_features < 1)
+        return set_err(SPN_E_ARG, "negative size, n_roots < 1 or n_features < 1");
+    if ((n_nodes && !nodes) || (n_edges && (!children || !weights)) || (n_params && !params) ||
+        !roots)
+        return set_err(SPN_E_ARG, "null array with non-zero size");
+    GraphData *g = new (std::nothrow) GraphData();
+    if (!g) return set_err(SPN_E_OOM, "graph allocation");
+    try {
+        g->F = n_features;
+        g->kind.resize(n_nodes);
+        g->feature.resize(n_nodes);
+        g->n_children.resize(n_nodes);
+        g->n_params.resize(n_nodes);
+        g->child_begin.resize(n_nodes);
+        g->param_begin.resize(n_nodes);
+        for (int64_t i = 0; i < n_nodes; ++i) {
+            g->kind[i] = nodes[i].kind;
+            g->feature[i] = nodes[i].feature;
+            g->n_children[i] = nodes[i].n_children;
+            g->n_params[i] = nodes[i].n_params;
+            g->child_begin[i] = nodes[i].child_begin;
+            g->param_begin[i] = nodes[i].param_begin;
+        }
+        g->children.assign(children, children + n_edges);
+        g->weights.assign(weights, weights + n_edges);
+        g->params.assign(params, params + n_params);
+        g->roots.assign(roots, roots + n_roots);
+    } catch (...) {
+        delete g;
+        return set_err(SPN_E_OOM, "graph copy");
+    }
+    std::string msg;
+    const int rc = validate_graph(*g, msg);
+    if (rc != SPN_OK) {
+        delete g;
+        return set_err(rc, msg);
+    }
+    spn_handle *h = new (std::nothrow) spn_handle();
+    if (!h) {
+        delete g;
+        return set_err(SPN_E_OOM, "handle");
+    }
+    h->magic = H_GRAPH;
+    h->graph = g;
+    *out_graph = h;
+    return SPN_OK;
+}
+
+int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
+                spn_handle **out_plan) {
+    if (!out_plan) return set_err(SPN_E_ARG, "out_plan is NULL");
+    *out_plan = nullptr;
+    if (!valid_graph_handle(graph)) return set_err(SPN_E_ARG, "not a graph handle");
+    spn_prepare_options opt;
+    spn_default_options(&opt);
+    if (opt_in) opt = *opt_in;
+    for (int i = 0; i < 8; ++i)
+        if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
+    if (opt.layered_path == 2) return set_err(SPN_E_UNSUPPORTED, "layered path not available for this graph");
+    const auto t0 = std::chrono::steady_clock::now();
+    const GraphData &g = *graph->graph;
+
+    int dev = opt.device;
+    cudaError_t e;
+    if (dev < 0 && (e = cudaGetDevice(&dev)) != cudaSuccess) return cuda_err(e, "cudaGetDevice");
+    DeviceGuard dg(dev);
+    int sms = 0, smem_optin = 0;
+    if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+        return cuda_err(e, "device attributes");
+    cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+
+    int K = opt.samples_per_thread ? opt.samples_per_thread : 4;
+    if (K != 1 && K != 2 && K != 4) return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2 or 4");
+    const int max_block = K == 4 ? 384 : 512;
+    int block = opt.block_threads ? opt.block_threads : max_block;
+    if (block % 32 || block < 32 || block > max_block)
+        return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 within the kernel bound");
+    int nwarps = block / 32;
+    const int WT = 32 * K;
+    const int tpw = WT + 4;
+    const size_t xtile = (size_t)g.F * tpw * 4;
+    // stage features in shared memory when a few warps' tiles fit comfortably
+    bool xs = xtile * std::min(nwarps, 8) <= (size_t)smem_optin * 3 / 4;
+
+    CodegenConfig cfg;
+    cfg.K = K;
+    cfg.x_in_smem = xs;
+    cfg.tpw = tpw;
+    cfg.max_task_ops = opt.max_task_nodes > 0 ? opt.max_task_nodes : -1;
+    cfg.smem_slot_cap = 0;
+    const bool auto_cap = opt.max_task_nodes == 0;
+    PlanProgram prog;
+    std::string msg;
+    size_t smem = 0;
+    for (int iter = 0;; ++iter) {
+        prog = PlanProgram();
+        int rc = build_program(g, cfg, prog, msg);
+        if (rc != SPN_OK) return set_err(rc, msg);
+        auto smem_of = [&](int nw, int64_t sslots) {
+            return (size_t)(prog.max_task_records + 2) * sizeof(Rec) +
+                   (size_t)nw * ((xs ? xtile : 0) + (size_t)sslots * WT * 4);
+        };
+        smem = smem_of(nwarps, prog.n_sslots);
+        if (smem <= (size_t)smem_optin) {
+            // give left-over shared memory to task-local slots (one rebuild)
+            const int64_t spare = ((int64_t)smem_optin - (int64_t)smem_of(nwarps, 0)) /
+                                  ((int64_t)nwarps * WT * 4);
+            if (prog.n_gslots > 0 && cfg.smem_slot_cap == 0 && spare > 0 && iter < 40) {
+                cfg.smem_slot_cap = std::min<int64_t>(spare, 4096);
+                continue;
+            }
+            break;
+        }
+        if (iter > 40) return set_err(SPN_E_UNSUPPORTED, "cannot fit the plan into shared memory");
+        if (xs && nwarps > 8 && !opt.block_threads) {
+            nwarps -= 2;
+            block = nwarps * 32;
+            continue;
+        }
+        if (prog.n_sslots > 0 && cfg.smem_slot_cap > 0) {
+            cfg.smem_slot_cap /= 2;
+            continue;
+        }
+        if (!auto_cap && cfg.max_task_ops > 0 && opt.max_task_nodes > 0)
+            return set_err(SPN_E_UNSUPPORTED, "max_task_nodes too large for shared memory");
+        // partition (or partition finer) so one task's program fits
+        int64_t total_ops = 0;
+        for (int64_t u = 0; u < (int64_t)g.kind.size(); ++u) total_ops += g.n_children[u] * 2;
+        const int64_t budget_rec =
+            ((int64_t)smem_optin - (int64_t)nwarps * (xs ? (int64_t)xtile : 0)) / (int64_t)sizeof(Rec) - 8;
+        if (budget_rec < 64) return set_err(SPN_E_UNSUPPORTED, "no shared memory left for the program");
+        if (cfg.max_task_ops <= 0) cfg.max_task_ops = std::max<int64_t>(64, budget_rec / 2);
+        else cfg.max_task_ops = std::max<int64_t>(32, cfg.max_task_ops * 2 / 3);
+    }
+
+    DevicePlan *P = new (std::nothrow) DevicePlan();
+    if (!P) return set_err(SPN_E_OOM, "plan");
+    P->device = dev;
+    P->K = K;
+    P->xs = xs;
+    P->tpw = tpw;
+    P->block = block;
+    P->smem = smem;
+    P->sms = sms;
+    P->F = g.F;
+    P->R = (int32_t)g.roots.size();
+    P->n_tasks = (int32_t)(prog.task_off.size() - 1);
+    P->first_task_len = (int32_t)(prog.task_off[1] - prog.task_off[0]);
+    P->prog_cap = (int)(prog.max_task_records + 2);
+    P->n_sslots = prog.n_sslots;
+    P->n_gslots = prog.n_gslots;
+    int rc;
+    if ((rc = upload(&P->d_prog, prog.prog)) || (rc = upload(&P->d_task_off, prog.task_off)) ||
+        (rc = upload(&P->d_tables, prog.tables)) || (rc = upload(&P->d_edges, prog.edges))) {
+        free_plan(P);
+        return rc;
+    }
+    int bps = occupancy(K, false, xs, block, smem);
+    if (opt.ctas_per_sm > 0) bps = std::min(bps, opt.ctas_per_sm);
+    if (bps < 1) {
+        free_plan(P);
+        return set_err(SPN_E_UNSUPPORTED, "kernel does not fit on an SM with this configuration");
+    }
+    P->grid_max = sms * bps;
+    if (P->n_gslots > 0) {
+        const size_t bytes = (size_t)P->grid_max * (block / 32) * P->n_gslots * WT * 4;
+        if ((e = cudaMalloc(&P->d_gslots, bytes)) != cudaSuccess) {
+            free_plan(P);
+            return set_err(SPN_E_OOM, "scratch slots");
+        }
+    }
+    spn_plan_stats &s = P->stats;
+    memset(&s, 0, sizeof(s));
+    s.n_nodes = prog.n_nodes;
+    s.n_leaves = prog.n_leaves;
+    s.n_sums = prog.n_sums;
+    s.n_products = prog.n_products;
+    s.n_sum_edges = prog.n_sum_edges;
+    s.n_tasks = P->n_tasks;
+    s.n_cut_values = prog.n_cut_values;
+    s.partition_cost = prog.partition_cost;
+    s.n_records = (int64_t)prog.prog.size();
+    s.n_global_slots = prog.n_gslots;
+    s.n_smem_slots = prog.n_sslots;
+    s.max_stack = prog.max_stack;
+    s.mufu_per_sample = prog.mufu_per_sample;
+    s.fma_per_sample = prog.fma_per_sample;
+    s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)g.roots.size();
+    s.tc_flops_per_sample = 0;
+    s.path = 0;
+    s.block_threads = block;
+    s.samples_per_thread = K;
+    s.grid = P->grid_max;
+    s.smem_bytes = (int32_t)smem;
+    s.x_in_smem = xs;
+    s.prepare_ms =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    spn_handle *h = new (std::nothrow) spn_handle();
+    if (!h) {
+        free_plan(P);
+        return set_err(SPN_E_OOM, "handle");
+    }
+    h->magic = H_PLAN;
+    h->plan = P;
+    *out_plan = h;
+    return SPN_OK;
+}
+
+int spn_infer_joint(spn_handle *plan, const float *x, int64_t n, int64_t ld, float *out,
+                    int32_t *argmax, void *cuda_stream) {
+    return infer_device(plan, x, n, ld, out, argmax, cuda_stream, false);
+}
+
+int spn_infer_marginal(spn_handle *plan, const float *x, int64_t n, int64_t ld, float *out,
+                       int32_t *argmax, void *cuda_stream) {
+    return infer_device(plan, x, n, ld, out, argmax, cuda_stream, true);
+}
+
+int spn_infer_joint_host(spn_handle *plan, const float *x, int64_t n, int64_t ld, float *out,
+                         int32_t *argmax) {
+    return infer_host(plan, x, n, ld, out, argmax, false);
+}
+
+int spn_infer_marginal_host(spn_handle *plan, const float *x, int64_t n, int64_t ld, float *out,
+                            int32_t *argmax) {
+    return infer_host(plan, x, n, ld, out, argmax, true);
+}
+
+int spn_plan_info(const spn_handle *plan, spn_plan_stats *stats) {
+    if (!plan || plan->magic != H_PLAN || !stats) return set_err(SPN_E_ARG, "not a plan handle");
+    *stats = plan->plan->stats;
+    return SPN_OK;
+}
+
+int spn_partition_graph(const spn_handle *graph, int64_t max_task_ops, int32_t *task_of_node,
+                        int32_t *n_tasks, int64_t *cost, int64_t *cut_values) {
+    if (!valid_graph_handle(graph) || !task_of_node) return set_err(SPN_E_ARG, "bad arguments");
+    std::vector<int32_t> t;
+    PartitionResult res;
+    const int rc = partition_graph(*graph->graph, max_task_ops, t, res);
+    if (rc != SPN_OK) return set_err(rc, "partition failed");
+    memcpy(task_of_node, t.data(), t.size() * sizeof(int32_t));
+    if (n_tasks) *n_tasks = res.n_tasks;
+    if (cost) *cost = res.cost;
+    if (cut_values) *cut_values = res.cut_values;
+    return SPN_OK;
+}
+
+int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32_t x_in_smem,
+                      int64_t max_task_ops, int64_t smem_slot_cap, void *records,
+                      int64_t *n_records, int64_t *task_off, int64_t *n_tasks, float *tables,
+                      int64_t *n_tables, void *edges, int64_t *n_edges, int64_t *slots) {
+    if (!valid_graph_handle(graph) || !n_records || !n_tasks || !n_tables || !n_edges)
+        return set_err(SPN_E_ARG, "bad arguments");
+    if (samples_per_thread != 1 && samples_per_thread != 2 && samples_per_thread != 4)
+        return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2 or 4");
+    CodegenConfig cfg;
+    cfg.K = samples_per_thread;
+    cfg.x_in_smem = x_in_smem != 0;
+    cfg.tpw = 32 * cfg.K + 4;
+    cfg.max_task_ops = max_task_ops;
+    cfg.smem_slot_cap = smem_slot_cap;
+    PlanProgram prog;
+    std::string msg;
+    const int rc = build_program(*graph->graph, cfg, prog, msg);
+    if (rc != SPN_OK) return set_err(rc, msg);
+    const int64_t nr = (int64_t)prog.prog.size(), nt = (int64_t)prog.task_off.size() - 1;
+    const int64_t ntab = (int64_t)prog.tables.size(), ne = (int64_t)prog.edges.size();
+    if (records) {
+        if (*n_records < nr || *n_tasks < nt || *n_tables < ntab || *n_edges < ne || !task_off ||
+            !tables || !edges)
+            return set_err(SPN_E_ARG, "buffers too small");
+        memcpy(records, prog.prog.data(), nr * sizeof(Rec));
+        memcpy(task_off, prog.task_off.data(), (nt + 1) * sizeof(int64_t));
+        memcpy(tables, prog.tables.data(), ntab * sizeof(float));
+        memcpy(edges, prog.edges.data(), ne * sizeof(Edge));
+    }
+    *n_records = nr;
+    *n_tasks = nt;
+    *n_tables = ntab;
+    *n_edges = ne;
+    if (slots) {
+        slots[0] = prog.n_sslots;
+        slots[1] = prog.n_gslots;
+        slots[2] = prog.max_stack;
+    }
+    return SPN_OK;
+}
+
+void spn_free(spn_handle *h) {
+    if (!h) return;
+    if (h->magic == H_GRAPH) delete h->graph;
+    else if (h->magic == H_PLAN) free_plan(h->plan);
+    h->magic = 0;
+    delete h;
+}
+
+}  // extern "C"

@@ -1,0 +1,543 @@
+// dag_eval.cuh -- generic SPN DAG evaluator for sm_100a (kernel KA).
+//
+// Computes, for every sample s and root r, log p_r(x_s) by a single bottom-up
+// pass over the DAG (§II-A): leaves query univariate
+// distributions with full (joint) or partial (marginal) evidence, products add
+// log values, weighted sums take a max-shifted log-sum-exp (log space, L86).
+//
+// B200 design:
+//  * The DAG is not compiled to straight-line code per SPN as in the paper's
+//    GPU lowering (L369-382); it is a table-driven node program (program.h)
+//    interpreted by every thread for K samples at once, so one warp-uniform
+//    dispatch is amortised over 32*K samples.  Values live in a register
+//    stack whose depth at each record is static: one dense switch with a case
+//    per (op, sp) compiles to a single jump table (LDC + BRX).
+//  * Each warp owns a tile of 32*K samples; the tile's features are staged in
+//    shared memory transposed to [F][32K+4] so a leaf reads its K inputs with
+//    one vector LDS (the paper's access-pattern-aware loads, L80, L360).
+//  * Sums use the n-ary max-shifted LSE in the log2 domain with MUFU ex2/lg2:
+//    fan-in + 1 MUFU ops per sum (not 2 per edge as binary log-adds).
+//  * Single-task plans: the node program is staged once per CTA and warps run
+//    a persistent static round-robin loop over warp tiles (no CTA barriers).
+//    Multi-task plans (partitioned, L336-346): CTA tiles, each task's program
+//    is staged into shared memory in turn; values crossing tasks go through
+//    per-warp global scratch slots (L2 resident), task-local ones through
+//    shared-memory slots.
+#pragma once
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <stdint.h>
+
+#include "program.h"
+
+namespace spnb {
+
+__device__ __forceinline__ float ex2a(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float lg2a(float x) {
+    float y;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
+__device__ __forceinline__ Rec make_end() {
+    Rec r;
+    r.x = 0; r.y = 0; r.z = 0; r.w = 0;
+    return r;
+}
+
+// 32-bit shared-memory addressing through asm: the addresses are "pinned" in
+// registers (a volatile mov cannot be rematerialised), so the compiler does not
+// recompute the warp's tile base in every switch case.
+__device__ __forceinline__ uint32_t pin_u32(uint32_t v) {
+    uint32_t r;
+    asm volatile("mov.b32 %0, %1;" : "=r"(r) : "r"(v));
+    return r;
+}
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+template <int K>
+struct SIO;  // shared memory, 32-bit byte address
+template <>
+struct SIO<4> {
+    static __device__ __forceinline__ void ld(uint32_t a, float (&v)[4]) {
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]) : "r"(a));
+    }
+    static __device__ __forceinline__ void st(uint32_t a, const float (&v)[4]) {
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};"
+                     :: "r"(a), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]) : "memory");
+    }
+};
+template <>
+struct SIO<2> {
+    static __device__ __forceinline__ void ld(uint32_t a, float (&v)[2]) {
+        asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v[0]), "=f"(v[1]) : "r"(a));
+    }
+    static __device__ __forceinline__ void st(uint32_t a, const float (&v)[2]) {
+        asm volatile("st.shared.v2.f32 [%0], {%1, %2};" :: "r"(a), "f"(v[0]), "f"(v[1])
+                     : "memory");
+    }
+};
+template <>
+struct SIO<1> {
+    static __device__ __forceinline__ void ld(uint32_t a, float (&v)[1]) {
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v[0]) : "r"(a));
+    }
+    static __device__ __forceinline__ void st(uint32_t a, const float (&v)[1]) {
+        asm volatile("st.shared.f32 [%0], %1;" :: "r"(a), "f"(v[0]) : "memory");
+    }
+};
+
+template <int K>
+struct GIO;  // global memory (scratch slots)
+template <>
+struct GIO<4> {
+    static __device__ __forceinline__ void ld(const float *p, float (&v)[4]) {
+        const float4 t = *reinterpret_cast<const float4 *>(p);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+    }
+    static __device__ __forceinline__ void st(float *p, const float (&v)[4]) {
+        *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+};
+template <>
+struct GIO<2> {
+    static __device__ __forceinline__ void ld(const float *p, float (&v)[2]) {
+        const float2 t = *reinterpret_cast<const float2 *>(p);
+        v[0] = t.x; v[1] = t.y;
+    }
+    static __device__ __forceinline__ void st(float *p, const float (&v)[2]) {
+        *reinterpret_cast<float2 *>(p) = make_float2(v[0], v[1]);
+    }
+};
+template <>
+struct GIO<1> {
+    static __device__ __forceinline__ void ld(const float *p, float (&v)[1]) { v[0] = *p; }
+    static __device__ __forceinline__ void st(float *p, const float (&v)[1]) { *p = v[0]; }
+};
+
+// Per-thread execution environment.  Record operands for features and slots
+// are BYTE offsets (pre-multiplied by the preparer).
+template <int K, bool MARG, bool XS>
+struct Env {
+    uint32_t xs;            // XS: shared address of this thread's x column (+lane*K*4)
+    const float *xrow[K];   // !XS: row pointers of this thread's K samples
+    uint32_t ss;            // shared slots of this warp (+lane*K*4)
+    char *gs;               // global slots of this warp (+lane*K*4)
+    const float *tables;
+    const Edge *edges;
+    float *out;             // out + first sample * R
+    int32_t R;
+    int32_t nvalid;         // valid samples of this thread (0..K)
+
+    __device__ __forceinline__ void loadx(uint32_t f, float (&v)[K]) const {
+        if constexpr (XS) {
+            SIO<K>::ld(xs + f, v);
+        } else {
+#pragma unroll
+            for (int j = 0; j < K; ++j)
+                v[j] = __ldg(reinterpret_cast<const float *>(
+                    reinterpret_cast<const char *>(xrow[j]) + f));
+        }
+    }
+    __device__ __forceinline__ void load_slot(uint32_t ref, float (&v)[K]) const {
+        if (ref & SLOT_GLOBAL) GIO<K>::ld(reinterpret_cast<const float *>(gs + (ref & ~SLOT_GLOBAL)), v);
+        else SIO<K>::ld(ss + ref, v);
+    }
+};
+
+#define FOR_K _Pragma("unroll") for (int j = 0; j < K; ++j)
+
+template <int S, bool ACC, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_gauss(float (&r)[MAXD][K], uint32_t arg, uint32_t y,
+                                        uint32_t z, uint32_t w, const Env<K, MARG, XS> &e) {
+    float xv[K];
+    e.loadx(arg, xv);
+    const float a = __uint_as_float(y), b = __uint_as_float(z), cc = __uint_as_float(w);
+    FOR_K {
+        const float t = fmaf(a, xv[j], -b);
+        float v = fmaf(-t, t, cc);
+        if (MARG) v = (xv[j] != xv[j]) ? 0.f : v;
+        if constexpr (ACC) r[S - 1][j] += v;
+        else r[S][j] = v;
+    }
+}
+
+template <int S, bool ACC, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_disc(float (&r)[MAXD][K], uint32_t arg, uint32_t y,
+                                       uint32_t z, uint32_t w, const Env<K, MARG, XS> &e) {
+    float xv[K];
+    e.loadx(arg, xv);
+    const float *tab = e.tables + y;
+    const int lo = (int)z;
+    const int nk = (int)w;
+    const float flo = (float)lo, fhi = (float)(lo + nk);
+    FOR_K {
+        const float x = xv[j];
+        const bool ok = (x >= flo) && (x < fhi);
+        const int idx = ok ? ((int)floorf(x) - lo) : 0;
+        float v = ok ? __ldg(tab + idx) : -CUDART_INF_F;
+        if (x != x) v = MARG ? 0.f : x;
+        if constexpr (ACC) r[S - 1][j] += v;
+        else r[S][j] = v;
+    }
+}
+
+template <int S, int N, int K>
+__device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float w0, float w1, float w2,
+                                      float w3) {
+    FOR_K {
+        if constexpr (N == 1) {
+            r[S - 1][j] += w0;
+        } else {
+            float v[N];
+            v[0] = r[S - N][j] + w0;
+            v[1] = r[S - N + 1][j] + w1;
+            if constexpr (N > 2) v[2] = r[S - N + 2][j] + w2;
+            if constexpr (N > 3) v[3] = r[S - N + 3][j] + w3;
+            float m = v[0];
+#pragma unroll
+            for (int i = 1; i < N; ++i) m = fmaxf(m, v[i]);
+            // all children -inf (or weights 0): keep the shift finite so the
+            // result is -inf rather than NaN (reading c8); NaN children still
+            // propagate through ex2 (reading c7).
+            m = fmaxf(m, -1e30f);
+            float s = 0.f;
+#pragma unroll
+            for (int i = 0; i < N; ++i) s += ex2a(v[i] - m);
+            r[S - N][j] = m + lg2a(s);
+        }
+    }
+}
+
+template <int K>
+struct VecK {
+    float v[K];
+};
+
+// Gather-LSE over slot terms (large fan-in sums whose children are stored).
+// Not inlined: one copy serves every stack depth; arguments and result are
+// passed by value so the caller's register stack stays in registers.
+template <int K>
+__device__ __noinline__ VecK<K> h_glse(const Edge *__restrict__ E, int n, uint32_t ss,
+                                      const char *gs) {
+    auto load = [&](uint32_t ref, float (&v)[K]) {
+        if (ref & SLOT_GLOBAL) GIO<K>::ld(reinterpret_cast<const float *>(gs + (ref & ~SLOT_GLOBAL)), v);
+        else SIO<K>::ld(ss + ref, v);
+    };
+    float m[K];
+    FOR_K m[j] = -CUDART_INF_F;
+    for (int i = 0; i < n; ++i) {
+        const Edge ed = E[i];
+        float v[K];
+        load(ed.a, v);
+        if (ed.b != SLOT_NONE) {
+            float u[K];
+            load(ed.b, u);
+            FOR_K v[j] += u[j];
+        }
+        FOR_K m[j] = fmaxf(m[j], v[j] + ed.lw);
+    }
+    float s[K];
+    FOR_K {
+        m[j] = fmaxf(m[j], -1e30f);
+        s[j] = 0.f;
+    }
+    for (int i = 0; i < n; ++i) {
+        const Edge ed = E[i];
+        float v[K];
+        load(ed.a, v);
+        if (ed.b != SLOT_NONE) {
+            float u[K];
+            load(ed.b, u);
+            FOR_K v[j] += u[j];
+        }
+        FOR_K s[j] += ex2a(v[j] + ed.lw - m[j]);
+    }
+    VecK<K> out;
+    FOR_K out.v[j] = m[j] + lg2a(s[j]);
+    return out;
+}
+
+template <int K>
+struct ArgState {
+    float best[K];
+    int32_t idx[K];
+    __device__ __forceinline__ void init() {
+        FOR_K {
+            best[j] = -CUDART_INF_F;
+            idx[j] = -1;
+        }
+    }
+};
+
+template <int S, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_out(float (&r)[MAXD][K], uint32_t root,
+                                      const Env<K, MARG, XS> &e, ArgState<K> &am) {
+    FOR_K {
+        const float v = r[S - 1][j] * 0.6931471805599453f;
+        if (j < e.nvalid) e.out[j * e.R + (int)root] = v;
+        if (!(v != v) && (am.idx[j] < 0 || v > am.best[j] ||
+                          (v == am.best[j] && (int)root < am.idx[j]))) {
+            am.best[j] = v;
+            am.idx[j] = (int)root;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Valid stack depths per op (sp = depth before the op).
+__host__ __device__ constexpr bool op_valid(int op, int sp) {
+    return (op == OP_GPUSH || op == OP_DPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE)
+               ? (sp >= 0 && sp < MAXD)
+           : (op == OP_GACC || op == OP_DACC || op == OP_LSE1 || op == OP_STS ||
+              op == OP_STG || op == OP_OUT)
+               ? (sp >= 1)
+           : (op == OP_ADD || op == OP_LSE2) ? (sp >= 2)
+           : (op == OP_LSE3) ? (sp >= 3)
+           : (op == OP_LSE4) ? (sp >= 4)
+           : (op == OP_NOP);
+}
+
+#define SPN_ALL_SP(M, O) M(O, 0) M(O, 1) M(O, 2) M(O, 3) M(O, 4) M(O, 5) M(O, 6) M(O, 7) \
+    M(O, 8) M(O, 9) M(O, 10) M(O, 11) M(O, 12) M(O, 13) M(O, 14) M(O, 15) M(O, 16)
+
+// Every case label op*17+sp exists (dense => one jump table); invalid
+// combinations end the task.
+#define SPN_CASE(O, S)                                                           \
+    case O * NSP + S:                                                            \
+        if constexpr (op_valid(O, S)) {                                          \
+            SPN_BODY_##O(S)                                                      \
+        } else {                                                                 \
+            return;                                                              \
+        }                                                                        \
+        break;
+
+#define SPN_BODY_0(S) ;
+#define SPN_UNUSED_CASES case 289: case 290: case 291: case 292: case 293: case 294: case 295: case 296: case 297: case 298: case 299: case 300: case 301: case 302: case 303: case 304: case 305: case 306: case 307: case 308: case 309: case 310: case 311: case 312: case 313: case 314: case 315: case 316: case 317: case 318: case 319: case 320: case 321: case 322: case 323: case 324: case 325: case 326: case 327: case 328: case 329: case 330: case 331: case 332: case 333: case 334: case 335: case 336: case 337: case 338: case 339: case 340: case 341: case 342: case 343: case 344: case 345: case 346: case 347: case 348: case 349: case 350: case 351: case 352: case 353: case 354: case 355: case 356: case 357: case 358: case 359: case 360: case 361: case 362: case 363: case 364: case 365: case 366: case 367: case 368: case 369: case 370: case 371: case 372: case 373: case 374: case 375: case 376: case 377: case 378: case 379: case 380: case 381: case 382: case 383: case 384: case 385: case 386: case 387: case 388: case 389: case 390: case 391: case 392: case 393: case 394: case 395: case 396: case 397: case 398: case 399: case 400: case 401: case 402: case 403: case 404: case 405: case 406: case 407: case 408: case 409: case 410: case 411: case 412: case 413: case 414: case 415: case 416: case 417: case 418: case 419: case 420: case 421: case 422: case 423: case 424: case 425: case 426: case 427: case 428: case 429: case 430: case 431: case 432: case 433: case 434: case 435: case 436: case 437: case 438: case 439: case 440: case 441: case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
+#define SPN_BODY_1(S) h_gauss<(S < MAXD ? S : 0), false>(r, arg, cy, cz, cw, e);
+#define SPN_BODY_2(S) h_gauss<S, true>(r, arg, cy, cz, cw, e);
+#define SPN_BODY_3(S) h_disc<(S < MAXD ? S : 0), false>(r, arg, cy, cz, cw, e);
+#define SPN_BODY_4(S) h_disc<S, true>(r, arg, cy, cz, cw, e);
+#define SPN_BODY_5(S) { FOR_K r[S - 2][j] += r[S - 1][j]; }
+#define SPN_BODY_6(S) h_lse<S, 1>(r, W0, 0.f, 0.f, 0.f);
+#define SPN_BODY_7(S) h_lse<S, 2>(r, W0, W1, 0.f, 0.f);
+#define SPN_BODY_8(S) h_lse<S, 3>(r, W0, W1, W2, 0.f);
+#define SPN_BODY_9(S)                                                            \
+    {                                                                            \
+        uint32_t w3;                                                             \
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w3) : "r"(pc));            \
+        pc += 16;                                                                \
+        h_lse<S, 4>(r, W0, W1, W2, __uint_as_float(w3));                         \
+    }
+#define SPN_BODY_10(S) SIO<K>::ld(e.ss + arg, r[S < MAXD ? S : 0]);
+#define SPN_BODY_11(S) GIO<K>::ld(reinterpret_cast<const float *>(e.gs + arg), r[S < MAXD ? S : 0]);
+#define SPN_BODY_12(S) SIO<K>::st(e.ss + arg, r[S - 1]);
+#define SPN_BODY_13(S) GIO<K>::st(reinterpret_cast<float *>(e.gs + arg), r[S - 1]);
+#define SPN_BODY_14(S)                                                           \
+    {                                                                            \
+        const VecK<K> g = h_glse<K>(e.edges + (((uint64_t)cz << 32) | cy),        \
+                                    (int)cw, e.ss, e.gs);                        \
+        FOR_K r[S < MAXD ? S : 0][j] = g.v[j];                                   \
+    }
+#define SPN_BODY_15(S) h_out<S>(r, arg, e, am);
+#define SPN_BODY_16(S) ;
+
+// Run one task's program (shared memory at byte address prog) for this
+// thread's K samples.  All case labels 0..511 exist, so the dispatch is one
+// unchecked jump-table lookup (build with nvcc -jtd 10).
+template <int K, bool MARG, bool XS>
+__device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &e,
+                                         ArgState<K> &am) {
+    float r[MAXD][K];
+    uint32_t pc = prog;
+    for (;;) {
+        uint32_t cx, cy, cz, cw;
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(cx), "=r"(cy), "=r"(cz), "=r"(cw) : "r"(pc));
+        pc += 16;
+        const uint32_t arg = cx >> CASE_BITS;
+        const float W0 = __uint_as_float(cy);
+        const float W1 = __uint_as_float(cz);
+        const float W2 = __uint_as_float(cw);
+        (void)W0; (void)W1; (void)W2; (void)arg;
+        switch (cx & ((1u << CASE_BITS) - 1u)) {
+            SPN_ALL_SP(SPN_CASE, 0)
+            SPN_ALL_SP(SPN_CASE, 1)
+            SPN_ALL_SP(SPN_CASE, 2)
+            SPN_ALL_SP(SPN_CASE, 3)
+            SPN_ALL_SP(SPN_CASE, 4)
+            SPN_ALL_SP(SPN_CASE, 5)
+            SPN_ALL_SP(SPN_CASE, 6)
+            SPN_ALL_SP(SPN_CASE, 7)
+            SPN_ALL_SP(SPN_CASE, 8)
+            SPN_ALL_SP(SPN_CASE, 9)
+            SPN_ALL_SP(SPN_CASE, 10)
+            SPN_ALL_SP(SPN_CASE, 11)
+            SPN_ALL_SP(SPN_CASE, 12)
+            SPN_ALL_SP(SPN_CASE, 13)
+            SPN_ALL_SP(SPN_CASE, 14)
+            SPN_ALL_SP(SPN_CASE, 15)
+            SPN_ALL_SP(SPN_CASE, 16)
+            SPN_UNUSED_CASES
+            default:
+                __builtin_unreachable();
+        }
+    }
+}
+
+// Load this warp's tile of x (rows [base, base+nrows)) transposed into
+// xw[f * tpw + s] (s = sample within the 32*K tile).
+__device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__restrict__ x,
+                                            int64_t base, int nrows, int64_t ld, int F,
+                                            int lane, int WT) {
+    const int total = WT * F;
+    int s = lane / F;
+    int f = lane - s * F;
+    const float *xb = x + base * ld;
+    const uint32_t xa = smem_u32(xw);
+    for (int idx = lane; idx < total; idx += 32) {
+        const float v = (s < nrows) ? __ldg(xb + (int64_t)s * ld + f) : 0.f;
+        asm volatile("st.shared.f32 [%0], %1;" :: "r"(xa + 4u * (uint32_t)(f * tpw + s)), "f"(v)
+                     : "memory");
+        f += 32;
+        while (f >= F) {
+            f -= F;
+            ++s;
+        }
+    }
+}
+
+template <int K, bool MARG, bool XS>
+__global__ void __launch_bounds__(K == 4 ? 384 : 512) dag_eval_kernel(const KParams p) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    constexpr int WT = 32 * K;
+    Rec *prog_s = reinterpret_cast<Rec *>(smem_raw);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nwarps = blockDim.x >> 5;
+    const size_t xw_floats = XS ? (size_t)p.F * p.tpw : 0;
+    const size_t warp_floats = xw_floats + (size_t)p.n_sslots * WT;
+    float *warp_area = reinterpret_cast<float *>(smem_raw + (size_t)p.prog_cap * sizeof(Rec)) +
+                       (size_t)warp * warp_floats;
+    float *xw = warp_area;
+    float *ss = warp_area + xw_floats;
+    const int64_t gwarp = (int64_t)blockIdx.x * nwarps + warp;
+    const int64_t total_warps = (int64_t)gridDim.x * nwarps;
+
+    Env<K, MARG, XS> e;
+    e.xs = pin_u32(smem_u32(xw + lane * K));
+    e.ss = pin_u32(smem_u32(ss + lane * K));
+    e.gs = reinterpret_cast<char *>(p.gslots + (size_t)gwarp * p.n_gslots * WT + lane * K);
+    const uint32_t prog_a = pin_u32(smem_u32(prog_s));
+    e.tables = p.tables;
+    e.edges = p.edges;
+    e.R = p.R;
+
+    auto tile_begin = [&](int64_t base, ArgState<K> &am) {
+        const int64_t rem = p.n - base;
+        const int nrows = rem < WT ? (int)rem : WT;
+        if constexpr (XS) {
+            load_x_tile(xw, p.tpw, p.x, base, nrows, p.ld, p.F, lane, WT);
+            __syncwarp();
+        } else {
+#pragma unroll
+            for (int j = 0; j < K; ++j) {
+                int64_t row = base + lane * K + j;
+                row = row < p.n ? row : p.n - 1;
+                e.xrow[j] = p.x + row * p.ld;
+            }
+        }
+        const int64_t s0 = base + lane * K;
+        const int64_t rv = p.n - s0;
+        e.nvalid = rv <= 0 ? 0 : (rv < K ? (int)rv : K);
+        e.out = p.out + (size_t)(rv > 0 ? s0 : 0) * p.R;
+        am.init();
+    };
+    auto tile_end = [&](int64_t base, const ArgState<K> &am) {
+        if (p.argmax) {
+            const int64_t s0 = base + lane * K;
+            FOR_K if (j < e.nvalid) p.argmax[s0 + j] = am.idx[j];
+        }
+        if constexpr (XS) __syncwarp();
+    };
+
+    if (p.n_tasks == 1) {
+        const int len = p.first_task_len;
+        for (int i = threadIdx.x; i < len + 2; i += blockDim.x)
+            prog_s[i] = i < len ? p.prog[i] : make_end();
+        __syncthreads();
+        for (int64_t wt = gwarp; wt < p.n_wtiles; wt += total_warps) {
+            const int64_t base = wt * WT;
+            ArgState<K> am;
+            tile_begin(base, am);
+            run_task<K, MARG, XS>(prog_a, e, am);
+            tile_end(base, am);
+        }
+    } else {
+        const int64_t CT = (int64_t)nwarps * WT;
+        const int64_t n_ctiles = (p.n + CT - 1) / CT;
+        for (int64_t ct = blockIdx.x; ct < n_ctiles; ct += gridDim.x) {
+            const int64_t base = ct * CT + (int64_t)warp * WT;
+            const bool active = base < p.n;
+            ArgState<K> am;
+            if (active) tile_begin(base, am);
+            for (int t = 0; t < p.n_tasks; ++t) {
+                const int64_t b = p.task_off[t], len = p.task_off[t + 1] - b;
+                __syncthreads();
+                for (int64_t i = threadIdx.x; i < len + 2; i += blockDim.x)
+                    prog_s[i] = i < len ? p.prog[b + i] : make_end();
+                __syncthreads();
+                if (active) run_task<K, MARG, XS>(prog_a, e, am);
+            }
+            if (active) tile_end(base, am);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Host-side helpers, instantiated per K in dag_eval_k{1,2,4}.cu.
+template <int K, bool MARG, bool XS>
+cudaError_t dag_eval_launch_t(const KParams &p, int grid, int block, size_t smem,
+                              cudaStream_t st) {
+    auto fn = dag_eval_kernel<K, MARG, XS>;
+    cudaError_t err =
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (err != cudaSuccess) return err;
+    fn<<<grid, block, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <int K, bool MARG, bool XS>
+int dag_eval_occupancy_t(int block, size_t smem) {
+    auto fn = dag_eval_kernel<K, MARG, XS>;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess)
+        return 0;
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, block, smem) != cudaSuccess)
+        return 0;
+    return nb;
+}
+
+#define SPNB_INSTANTIATE_K(K)                                                             \
+    cudaError_t dag_eval_launch_k##K(const KParams &p, bool marg, bool xs, int grid,       \
+                                     int block, size_t smem, cudaStream_t st) {            \
+        if (marg) return xs ? dag_eval_launch_t<K, true, true>(p, grid, block, smem, st)  \
+                            : dag_eval_launch_t<K, true, false>(p, grid, block, smem, st); \
+        return xs ? dag_eval_launch_t<K, false, true>(p, grid, block, smem, st)           \
+                  : dag_eval_launch_t<K, false, false>(p, grid, block, smem, st);         \
+    }                                                                                     \
+    int dag_eval_occupancy_k##K(bool marg, bool xs, int block, size_t smem) {             \
+        if (marg) return xs ? dag_eval_occupancy_t<K, true, true>(block, smem)            \
+                            : dag_eval_occupancy_t<K, true, false>(block, smem);          \
+        return xs ? dag_eval_occupancy_t<K, false, true>(block, smem)                     \
+                  : dag_eval_occupancy_t<K, false, false>(block, smem);                   \
+    }
+
+}  // namespace spnb

@@ -1,0 +1,213 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the fp64 oracle on
+the same seeded inputs.  Tolerance (north_star): |g - o| <= 1e-4 max(1, |o|);
+-inf must match -inf, NaN must match NaN.  Argmax must agree wherever the
+oracle's top-2 gap exceeds twice the tolerance (ties are legitimately
+decided by rounding)."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_cgo_sommera022_b200 as spnb  # noqa: E402
+from oracle import oracle_eval  # noqa: E402
+from spn_inputs import (toy_spn, speaker_spn, speaker_set, rat_spn, tiny_discrete_spn,  # noqa: E402
+                        ancestral_sample, add_outliers, nan_mask, toy_data, GraphBuilder)
+
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    from paper_conf_cgo_sommera022_b200.build import build
+    build()
+    spnb.load_library()
+
+
+def _cmp(gpu, ref, tol=TOL):
+    gpu = np.asarray(gpu, dtype=np.float64)
+    both_nan = np.isnan(gpu) & np.isnan(ref)
+    both_inf = np.isneginf(gpu) & np.isneginf(ref)
+    with np.errstate(invalid="ignore"):
+        err = np.abs(gpu - ref) / np.maximum(1.0, np.abs(ref))
+        ok = both_nan | both_inf | (err <= tol)
+    assert ok.all(), (f"{(~ok).sum()} mismatches; first at {np.argwhere(~ok)[:3].tolist()}: "
+                      f"gpu={gpu[~ok][:3]} ref={ref[~ok][:3]}")
+    return float(np.nanmax(np.where(both_nan | both_inf, 0.0, err))) if err.size else 0.0
+
+
+def _cmp_argmax(am_gpu, ref, am_ref, tol=TOL):
+    if ref.shape[1] < 2:
+        return
+    s = np.sort(np.where(np.isnan(ref), -np.inf, ref), axis=1)
+    gap = s[:, -1] - s[:, -2]
+    decided = gap > 2 * tol * np.maximum(1.0, np.abs(s[:, -1]))
+    assert np.array_equal(am_gpu[decided], am_ref[decided])
+
+
+def _run(g, x, marginal=False, **opt):
+    G = spnb.Graph(g)
+    P = spnb.Plan(G, **opt)
+    xt = torch.from_numpy(x).cuda()
+    out, am = P.infer(xt, marginal=marginal)
+    torch.cuda.synchronize()
+    return out.cpu().numpy(), am.cpu().numpy(), P
+
+
+def _parity(g, x, marginal=False, **opt):
+    out, am, P = _run(g, x, marginal, **opt)
+    ref, am_ref = oracle_eval(g, x, marginal=marginal)
+    err = _cmp(out, ref)
+    _cmp_argmax(am, ref, am_ref)
+    return err, P
+
+
+# ----------------------------------------------------------------- config 1
+def test_c1_toy_all_assignments_and_golden():
+    g = toy_spn()
+    grid = np.array([[a, b, c] for a in range(-1, 3) for b in range(-1, 4) for c in range(-1, 5)],
+                    np.float32)
+    _parity(g, grid)
+    pats = np.array([[a, b, c] for a in [np.nan, 0, 1] for b in [np.nan, 0, 1, 2]
+                     for c in [np.nan, 0, 1, 2, 3]], np.float32)
+    _parity(g, pats, marginal=True)
+
+
+def test_c1_toy_100k_joint_and_marginal():
+    g = toy_spn()
+    x = toy_data(100_000, seed=1001)
+    _parity(g, x)
+    _parity(g, nan_mask(x, 0.2, 1002), marginal=True)
+
+
+# ----------------------------------------------------------------- config 2
+@pytest.mark.parametrize("n", [1, 31, 128, 129, 1000, 4099])
+def test_c2_ragged_sizes(n):
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, n, 2002)
+    _parity(g, add_outliers(x, 0.01, 7))
+
+
+@pytest.mark.parametrize("K", [1, 2, 4])
+def test_c2_samples_per_thread_variants(K):
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 3000, 11)
+    _parity(g, add_outliers(x, 0.01, 7), samples_per_thread=K)
+
+
+def test_c2_full_size_sampled():
+    """1M samples in the bench's launch configuration; oracle on a sample."""
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 1_000_000, 2002)
+    x = add_outliers(x, 0.01, 2003)
+    out, _, P = _run(g, x)
+    idx = np.random.default_rng(0).choice(len(x), 4000, replace=False)
+    ref, _ = oracle_eval(g, x[idx])
+    _cmp(out[idx], ref)
+    assert np.isfinite(out).all()
+
+
+def test_c2_marginal_without_nan_is_bitwise_joint():
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 5000, 3)
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    xt = torch.from_numpy(x).cuda()
+    j, _ = P.infer(xt)
+    m, _ = P.infer(xt, marginal=True)
+    assert torch.equal(j, m)
+
+
+def test_c2_full_marginal_is_zero():
+    g = speaker_spn(2001)
+    x = np.full((257, 26), np.nan, np.float32)
+    out, _, _ = _run(g, x, marginal=True)
+    assert np.abs(out).max() < 1e-4
+
+
+# ----------------------------------------------------------------- config 3
+def test_c3_speaker_set_marginal_argmax():
+    g = speaker_set(list(range(3001, 3033)))
+    x, labels = ancestral_sample(g, 3000, 3002)
+    x = nan_mask(x, 0.2, 3100)
+    err, P = _parity(g, x, marginal=True)
+    assert P.info()["n_tasks"] >= 1
+
+
+def test_c3_partition_sizes_agree():
+    g = speaker_set(list(range(3001, 3009)))
+    x, _ = ancestral_sample(g, 2000, 5)
+    x = nan_mask(x, 0.2, 6)
+    outs = []
+    for cap in (0, 300, 2000):
+        out, am, P = _run(g, x, True, max_task_nodes=cap)
+        outs.append(out)
+        ref, am_ref = oracle_eval(g, x, marginal=True)
+        _cmp(out, ref)
+    for o in outs[1:]:
+        _cmp(o, outs[0].astype(np.float64), tol=1e-5)
+
+
+# ----------------------------------------------------------------- config 4 (generic path)
+def test_c4_rat_generic_path_small():
+    g = rat_spn(4001, F=784, D=5, R=2, S=8, I=10, C=10)
+    x, _ = ancestral_sample(g, 600, 4002)
+    _parity(g, x)
+
+
+def test_rat_generic_with_partitioning():
+    g = rat_spn(7, F=64, D=3, R=3, S=6, I=8, C=4)
+    x, _ = ancestral_sample(g, 700, 8)
+    for cap in (0, 500):
+        _parity(g, x, max_task_nodes=cap)
+
+
+# ----------------------------------------------------------------- edges
+def test_empty_batch_and_strided_input():
+    g = speaker_spn(2001)
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    x, _ = ancestral_sample(g, 500, 1)
+    big = torch.zeros((500, 40), dtype=torch.float32, device="cuda")
+    big[:, :26] = torch.from_numpy(x).cuda()
+    out, _ = P.infer(big)                       # ld = 40 > F
+    ref, _ = oracle_eval(g, x)
+    _cmp(out.cpu().numpy(), ref)
+    e, _ = P.infer(big[:0])                     # n = 0 no-op
+    assert e.shape == (0, 1)
+    with pytest.raises(spnb.SPNError):
+        P.infer(big[:, :20])                    # ld < F
+
+
+def test_shard_invariance_bitwise():
+    g = speaker_set(list(range(3001, 3005)))
+    x, _ = ancestral_sample(g, 10_000, 2)
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    xt = torch.from_numpy(x).cuda()
+    full, amf = P.infer(xt)
+    parts = [P.infer(xt[a:b]) for a, b in ((0, 3333), (3333, 7001), (7001, 10_000))]
+    assert torch.equal(full, torch.cat([p[0] for p in parts]))
+    assert torch.equal(amf, torch.cat([p[1] for p in parts]))
+
+
+def test_host_pipeline_matches_device():
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 300_000, 5)
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    dev, _ = P.infer(torch.from_numpy(x).cuda())
+    xh = torch.from_numpy(x).pin_memory()
+    out, am = P.infer_host(xh)
+    assert np.array_equal(out, dev.cpu().numpy())
+
+
+def test_tiny_discrete_exact():
+    import itertools
+    for seed in range(4):
+        g = tiny_discrete_spn(seed)
+        doms = g.meta["domains"]
+        x = np.array(list(itertools.product(*[range(-1, k + 1) for k in doms])), np.float32)
+        _parity(g, x)
+        _parity(g, nan_mask(x, 0.3, seed), marginal=True)

@@ -188,6 +188,8 @@ class Plan:
         import torch
         if not (x.is_cuda and x.dtype == torch.float32 and x.dim() == 2 and x.stride(1) == 1):
             raise ValueError("x must be a CUDA float32 [N, F] tensor with unit feature stride")
+        if x.shape[1] < self.n_features:
+            raise ValueError(f"x has {x.shape[1]} features, the SPN needs {self.n_features}")
         N = x.shape[0]
         if out is None:
             out = torch.empty((N, self.n_roots), dtype=torch.float32, device=x.device)
@@ -209,6 +211,8 @@ class Plan:
         if not (isinstance(xa, np.ndarray) and xa.dtype == np.float32 and xa.ndim == 2
                 and xa.strides[1] == 4):
             raise ValueError("x must be a float32 [N, F] host array with unit feature stride")
+        if xa.shape[1] < self.n_features:
+            raise ValueError(f"x has {xa.shape[1]} features, the SPN needs {self.n_features}")
         N = xa.shape[0]
         if out is None:
             out = np.empty((N, self.n_roots), dtype=np.float32)

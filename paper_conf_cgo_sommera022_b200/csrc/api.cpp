@@ -219,8 +219,11 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
         const int s = (int)(i & 1);
         const int64_t m = std::min(C, n - c0);
         cudaStream_t st = P.hs[s];
-        e = cudaMemcpy2DAsync(P.hx[s], (size_t)P.F * 4, x + c0 * ld, (size_t)ld * 4,
-                              (size_t)P.F * 4, (size_t)m, cudaMemcpyHostToDevice, st);
+        if (ld == P.F)  // contiguous rows: one linear copy (2-D copies of 104-byte rows are slow)
+            e = cudaMemcpyAsync(P.hx[s], x + c0 * ld, (size_t)m * P.F * 4, cudaMemcpyHostToDevice, st);
+        else
+            e = cudaMemcpy2DAsync(P.hx[s], (size_t)P.F * 4, x + c0 * ld, (size_t)ld * 4,
+                                  (size_t)P.F * 4, (size_t)m, cudaMemcpyHostToDevice, st);
         if (e != cudaSuccess) return cuda_err(e, "H2D");
         rc = infer_device(h, P.hx[s], m, P.F, P.hout[s], argmax ? P.ham[s] : nullptr, st, marg);
         if (rc != SPN_OK) return rc;

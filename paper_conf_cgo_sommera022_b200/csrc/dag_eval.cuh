@@ -154,65 +154,154 @@ struct Env {
 
 #define FOR_K _Pragma("unroll") for (int j = 0; j < K; ++j)
 
-template <int S, bool ACC, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_gauss(float (&r)[MAXD][K], uint32_t arg, uint32_t y,
-                                        uint32_t z, uint32_t w, const Env<K, MARG, XS> &e) {
-    float xv[K];
-    e.loadx(arg, xv);
-    const float a = __uint_as_float(y), b = __uint_as_float(z), cc = __uint_as_float(w);
-    FOR_K {
-        const float t = fmaf(a, xv[j], -b);
-        float v = fmaf(-t, t, cc);
-        if (MARG) v = (xv[j] != xv[j]) ? 0.f : v;
-        if constexpr (ACC) r[S - 1][j] += v;
-        else r[S][j] = v;
-    }
+__device__ __forceinline__ void lds4(uint32_t a, uint32_t &x, uint32_t &y, uint32_t &z,
+                                     uint32_t &w) {
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w) : "r"(a));
 }
 
+// Leaf product: acc = C + sum_i leaf_i over the parameter records at pp
+// (ng Gaussian then nd discrete).  Returns the address after the last one.
 template <int S, bool ACC, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_disc(float (&r)[MAXD][K], uint32_t arg, uint32_t y,
-                                       uint32_t z, uint32_t w, const Env<K, MARG, XS> &e) {
-    float xv[K];
-    e.loadx(arg, xv);
-    const float *tab = e.tables + y;
-    const int lo = (int)z;
-    const int nk = (int)w;
-    const float flo = (float)lo, fhi = (float)(lo + nk);
-    FOR_K {
-        const float x = xv[j];
-        const bool ok = (x >= flo) && (x < fhi);
-        const int idx = ok ? ((int)floorf(x) - lo) : 0;
-        float v = ok ? __ldg(tab + idx) : -CUDART_INF_F;
-        if (x != x) v = MARG ? 0.f : x;
-        if constexpr (ACC) r[S - 1][j] += v;
-        else r[S][j] = v;
+__device__ __forceinline__ uint32_t h_lprod(float (&r)[MAXD][K], uint32_t ng, float C,
+                                            uint32_t nd, uint32_t pp,
+                                            const Env<K, MARG, XS> &e) {
+    float acc[K];
+    if constexpr (ACC) {
+        FOR_K acc[j] = r[S - 1][j] + C;
+    } else {
+        FOR_K acc[j] = C;
     }
+#pragma unroll 2
+    for (uint32_t i = 0; i < ng; ++i, pp += 16) {
+        uint32_t f, ya, zb, wc;
+        lds4(pp, f, ya, zb, wc);
+        float xv[K];
+        e.loadx(f, xv);
+        const float a = __uint_as_float(ya), b = __uint_as_float(zb);
+        FOR_K {
+            const float t = fmaf(a, xv[j], -b);
+            if constexpr (MARG) {
+                // NaN input: subtract this leaf's c from the pre-summed C instead
+                // of t^2, i.e. the leaf contributes log 1 = 0 (reading c6)
+                const bool nan = xv[j] != xv[j];
+                const float pv = nan ? __uint_as_float(wc) : t;
+                const float qv = nan ? 1.f : t;
+                acc[j] = fmaf(-pv, qv, acc[j]);
+            } else {
+                acc[j] = fmaf(-t, t, acc[j]);
+            }
+        }
+    }
+    for (uint32_t i = 0; i < nd; ++i, pp += 16) {
+        uint32_t f, tb, lo_u, nk;
+        lds4(pp, f, tb, lo_u, nk);
+        float xv[K];
+        e.loadx(f, xv);
+        const float *tab = e.tables + tb;
+        const int lo = (int)lo_u;
+        const float flo = (float)lo, fhi = (float)(lo + (int)nk);
+        FOR_K {
+            const float x = xv[j];
+            const bool ok = (x >= flo) && (x < fhi);
+            const int idx = ok ? ((int)floorf(x) - lo) : 0;
+            float v = ok ? __ldg(tab + idx) : -CUDART_INF_F;
+            if (x != x) v = MARG ? 0.f : x;
+            acc[j] += v;
+        }
+    }
+    if constexpr (ACC) {
+        FOR_K r[S - 1][j] = acc[j];
+    } else {
+        FOR_K r[S][j] = acc[j];
+    }
+    return pp;
 }
 
+__device__ __forceinline__ float max_nan(float a, float b) {  // NaN-propagating max
+    float r;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+
+// n-ary max-shifted log-sum-exp in the log2 domain.  The largest input hi is
+// the shift, so its term ex2(0) = 1 is exact and needs no MUFU: the n-1 other
+// inputs (selected with a min/max network) cost one ex2 each, plus one lg2.
+//   r = hi + bias + lg2(1 + sum_i ex2(lo_i - hi))
+// hi is NaN-propagating (reading c7); with all inputs -inf the shift is
+// clamped so the result is -inf, not NaN (reading c8).
 template <int S, int N, int K>
-__device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float w0, float w1, float w2,
-                                      float w3) {
+__device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float bias) {
     FOR_K {
         if constexpr (N == 1) {
-            r[S - 1][j] += w0;
+            r[S - 1][j] += bias;
         } else {
             float v[N];
-            v[0] = r[S - N][j] + w0;
-            v[1] = r[S - N + 1][j] + w1;
-            if constexpr (N > 2) v[2] = r[S - N + 2][j] + w2;
-            if constexpr (N > 3) v[3] = r[S - N + 3][j] + w3;
-            float m = v[0];
 #pragma unroll
-            for (int i = 1; i < N; ++i) m = fmaxf(m, v[i]);
-            // all children -inf (or weights 0): keep the shift finite so the
-            // result is -inf rather than NaN (reading c8); NaN children still
-            // propagate through ex2 (reading c7).
-            m = fmaxf(m, -1e30f);
-            float s = 0.f;
+            for (int i = 0; i < N; ++i) v[i] = r[S - N + i][j];
+            float hi, lo[N - 1];
+            if constexpr (N == 2) {
+                hi = max_nan(v[0], v[1]);
+                lo[0] = fminf(v[0], v[1]);
+            } else if constexpr (N == 3) {
+                const float m01 = fmaxf(v[0], v[1]);
+                lo[0] = fminf(v[0], v[1]);
+                lo[1] = fminf(m01, v[2]);
+                hi = max_nan(max_nan(v[0], v[1]), v[2]);
+            } else {
+                const float m01 = fmaxf(v[0], v[1]), m23 = fmaxf(v[2], v[3]);
+                lo[0] = fminf(v[0], v[1]);
+                lo[1] = fminf(v[2], v[3]);
+                lo[2] = fminf(m01, m23);
+                hi = max_nan(max_nan(v[0], v[1]), max_nan(v[2], v[3]));
+            }
+            const float hc = fmaxf(hi, -1e30f);
+            float s = 1.f;
 #pragma unroll
-            for (int i = 0; i < N; ++i) s += ex2a(v[i] - m);
-            r[S - N][j] = m + lg2a(s);
+            for (int i = 0; i < N - 1; ++i) s += ex2a(lo[i] - hc);
+            r[S - N][j] = (hi + bias) + lg2a(s);
         }
+    }
+}
+
+// Straight-line product of exactly N Gaussian leaves (parameter records at pp).
+// The next program record (at pp + 16 N) is loaded alongside the parameters.
+template <int S, bool ACC, int N, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_gprod(float (&r)[MAXD][K], float C, uint32_t pp,
+                                        const Env<K, MARG, XS> &e, uint32_t &nx, uint32_t &ny,
+                                        uint32_t &nz, uint32_t &nw) {
+    uint32_t f[N], ya[N], zb[N], wc[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) lds4(pp + 16 * i, f[i], ya[i], zb[i], wc[i]);
+    lds4(pp + 16 * N, nx, ny, nz, nw);
+    float xv[N][K];
+#pragma unroll
+    for (int i = 0; i < N; ++i) e.loadx(f[i], xv[i]);
+    float acc[K];
+    if constexpr (ACC) {
+        FOR_K acc[j] = r[S - 1][j] + C;
+    } else {
+        FOR_K acc[j] = C;
+    }
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+        const float a = __uint_as_float(ya[i]), b = __uint_as_float(zb[i]);
+        FOR_K {
+            const float t = fmaf(a, xv[i][j], -b);
+            if constexpr (MARG) {
+                const bool nan = xv[i][j] != xv[i][j];
+                const float pv = nan ? __uint_as_float(wc[i]) : t;
+                const float qv = nan ? 1.f : t;
+                acc[j] = fmaf(-pv, qv, acc[j]);
+            } else {
+                acc[j] = fmaf(-t, t, acc[j]);
+            }
+        }
+    }
+    if constexpr (ACC) {
+        FOR_K r[S - 1][j] = acc[j];
+    } else {
+        FOR_K r[S][j] = acc[j];
     }
 }
 
@@ -294,10 +383,11 @@ __device__ __forceinline__ void h_out(float (&r)[MAXD][K], uint32_t root,
 // ---------------------------------------------------------------------------
 // Valid stack depths per op (sp = depth before the op).
 __host__ __device__ constexpr bool op_valid(int op, int sp) {
-    return (op == OP_GPUSH || op == OP_DPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE)
+    return (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
+            (op >= OP_GPUSH1 && op <= OP_GPUSH4))
                ? (sp >= 0 && sp < MAXD)
-           : (op == OP_GACC || op == OP_DACC || op == OP_LSE1 || op == OP_STS ||
-              op == OP_STG || op == OP_OUT)
+           : (op == OP_LACC || op == OP_LSE1 || op == OP_STS || op == OP_STG || op == OP_OUT ||
+              (op >= OP_GACC1 && op <= OP_GACC4))
                ? (sp >= 1)
            : (op == OP_ADD || op == OP_LSE2) ? (sp >= 2)
            : (op == OP_LSE3) ? (sp >= 3)
@@ -320,53 +410,79 @@ __host__ __device__ constexpr bool op_valid(int op, int sp) {
         break;
 
 #define SPN_BODY_0(S) ;
-#define SPN_UNUSED_CASES case 289: case 290: case 291: case 292: case 293: case 294: case 295: case 296: case 297: case 298: case 299: case 300: case 301: case 302: case 303: case 304: case 305: case 306: case 307: case 308: case 309: case 310: case 311: case 312: case 313: case 314: case 315: case 316: case 317: case 318: case 319: case 320: case 321: case 322: case 323: case 324: case 325: case 326: case 327: case 328: case 329: case 330: case 331: case 332: case 333: case 334: case 335: case 336: case 337: case 338: case 339: case 340: case 341: case 342: case 343: case 344: case 345: case 346: case 347: case 348: case 349: case 350: case 351: case 352: case 353: case 354: case 355: case 356: case 357: case 358: case 359: case 360: case 361: case 362: case 363: case 364: case 365: case 366: case 367: case 368: case 369: case 370: case 371: case 372: case 373: case 374: case 375: case 376: case 377: case 378: case 379: case 380: case 381: case 382: case 383: case 384: case 385: case 386: case 387: case 388: case 389: case 390: case 391: case 392: case 393: case 394: case 395: case 396: case 397: case 398: case 399: case 400: case 401: case 402: case 403: case 404: case 405: case 406: case 407: case 408: case 409: case 410: case 411: case 412: case 413: case 414: case 415: case 416: case 417: case 418: case 419: case 420: case 421: case 422: case 423: case 424: case 425: case 426: case 427: case 428: case 429: case 430: case 431: case 432: case 433: case 434: case 435: case 436: case 437: case 438: case 439: case 440: case 441: case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
-#define SPN_BODY_1(S) h_gauss<(S < MAXD ? S : 0), false>(r, arg, cy, cz, cw, e);
-#define SPN_BODY_2(S) h_gauss<S, true>(r, arg, cy, cz, cw, e);
-#define SPN_BODY_3(S) h_disc<(S < MAXD ? S : 0), false>(r, arg, cy, cz, cw, e);
-#define SPN_BODY_4(S) h_disc<S, true>(r, arg, cy, cz, cw, e);
-#define SPN_BODY_5(S) { FOR_K r[S - 2][j] += r[S - 1][j]; }
-#define SPN_BODY_6(S) h_lse<S, 1>(r, W0, 0.f, 0.f, 0.f);
-#define SPN_BODY_7(S) h_lse<S, 2>(r, W0, W1, 0.f, 0.f);
-#define SPN_BODY_8(S) h_lse<S, 3>(r, W0, W1, W2, 0.f);
+#define SPN_BODY_1(S)                                                            \
+    pc = h_lprod<(S < MAXD ? S : 0), false>(r, arg, __uint_as_float(cy), cz, pc + 16, e) - 16; \
+    lds4(pc + 16, nx, ny, nz, nw);
+#define SPN_BODY_2(S)                                                            \
+    pc = h_lprod<S, true>(r, arg, __uint_as_float(cy), cz, pc + 16, e) - 16;      \
+    lds4(pc + 16, nx, ny, nz, nw);
+#define SPN_BODY_3(S) { FOR_K r[S - 2][j] += r[S - 1][j] + __uint_as_float(cy); }
+#define SPN_BODY_4(S) h_lse<S, 1>(r, __uint_as_float(cy));
+#define SPN_BODY_5(S) h_lse<S, 2>(r, __uint_as_float(cy));
+#define SPN_BODY_6(S) h_lse<S, 3>(r, __uint_as_float(cy));
+#define SPN_BODY_7(S) h_lse<S, 4>(r, __uint_as_float(cy));
+#define SPN_BODY_8(S)                                                            \
+    {                                                                            \
+        SIO<K>::ld(e.ss + arg, r[S < MAXD ? S : 0]);                             \
+        FOR_K r[S < MAXD ? S : 0][j] += __uint_as_float(cy);                     \
+    }
 #define SPN_BODY_9(S)                                                            \
     {                                                                            \
-        uint32_t w3;                                                             \
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w3) : "r"(pc));            \
-        pc += 16;                                                                \
-        h_lse<S, 4>(r, W0, W1, W2, __uint_as_float(w3));                         \
+        GIO<K>::ld(reinterpret_cast<const float *>(e.gs + arg), r[S < MAXD ? S : 0]); \
+        FOR_K r[S < MAXD ? S : 0][j] += __uint_as_float(cy);                     \
     }
-#define SPN_BODY_10(S) SIO<K>::ld(e.ss + arg, r[S < MAXD ? S : 0]);
-#define SPN_BODY_11(S) GIO<K>::ld(reinterpret_cast<const float *>(e.gs + arg), r[S < MAXD ? S : 0]);
-#define SPN_BODY_12(S) SIO<K>::st(e.ss + arg, r[S - 1]);
-#define SPN_BODY_13(S) GIO<K>::st(reinterpret_cast<float *>(e.gs + arg), r[S - 1]);
-#define SPN_BODY_14(S)                                                           \
+#define SPN_BODY_10(S) SIO<K>::st(e.ss + arg, r[S - 1]);
+#define SPN_BODY_11(S) GIO<K>::st(reinterpret_cast<float *>(e.gs + arg), r[S - 1]);
+#define SPN_BODY_12(S)                                                           \
     {                                                                            \
         const VecK<K> g = h_glse<K>(e.edges + (((uint64_t)cz << 32) | cy),        \
                                     (int)cw, e.ss, e.gs);                        \
         FOR_K r[S < MAXD ? S : 0][j] = g.v[j];                                   \
     }
-#define SPN_BODY_15(S) h_out<S>(r, arg, e, am);
-#define SPN_BODY_16(S) ;
+#define SPN_BODY_13(S) h_out<S>(r, arg, e, am);
+#define SPN_BODY_14(S) ;
+#define SPN_BODY_15(S)                                                       \
+    h_gprod<(S < MAXD ? S : 0), false, 1>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
+    pc += 16;
+#define SPN_BODY_16(S)                                                       \
+    h_gprod<(S < MAXD ? S : 0), false, 2>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
+    pc += 32;
+#define SPN_BODY_17(S)                                                       \
+    h_gprod<(S < MAXD ? S : 0), false, 3>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
+    pc += 48;
+#define SPN_BODY_18(S)                                                       \
+    h_gprod<(S < MAXD ? S : 0), false, 4>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
+    pc += 64;
+#define SPN_BODY_19(S)                                                       \
+    h_gprod<S, true, 1>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
+    pc += 16;
+#define SPN_BODY_20(S)                                                       \
+    h_gprod<S, true, 2>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
+    pc += 32;
+#define SPN_BODY_21(S)                                                       \
+    h_gprod<S, true, 3>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
+    pc += 48;
+#define SPN_BODY_22(S)                                                       \
+    h_gprod<S, true, 4>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
+    pc += 64;
+#define SPN_UNUSED_CASES case 391: case 392: case 393: case 394: case 395: case 396: case 397: case 398: case 399: case 400: case 401: case 402: case 403: case 404: case 405: case 406: case 407: case 408: case 409: case 410: case 411: case 412: case 413: case 414: case 415: case 416: case 417: case 418: case 419: case 420: case 421: case 422: case 423: case 424: case 425: case 426: case 427: case 428: case 429: case 430: case 431: case 432: case 433: case 434: case 435: case 436: case 437: case 438: case 439: case 440: case 441: case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
 
 // Run one task's program (shared memory at byte address prog) for this
 // thread's K samples.  All case labels 0..511 exist, so the dispatch is one
-// unchecked jump-table lookup (build with nvcc -jtd 10).
+// unchecked jump-table lookup (build with nvcc -jtd 10).  The next record is
+// loaded before the current one is dispatched (software prefetch).
 template <int K, bool MARG, bool XS>
 __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &e,
                                          ArgState<K> &am) {
     float r[MAXD][K];
     uint32_t pc = prog;
+    uint32_t cx, cy, cz, cw;
+    lds4(pc, cx, cy, cz, cw);
     for (;;) {
-        uint32_t cx, cy, cz, cw;
-        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
-                     : "=r"(cx), "=r"(cy), "=r"(cz), "=r"(cw) : "r"(pc));
-        pc += 16;
+        uint32_t nx, ny, nz, nw;
+        lds4(pc + 16, nx, ny, nz, nw);
         const uint32_t arg = cx >> CASE_BITS;
-        const float W0 = __uint_as_float(cy);
-        const float W1 = __uint_as_float(cz);
-        const float W2 = __uint_as_float(cw);
-        (void)W0; (void)W1; (void)W2; (void)arg;
+        (void)arg;
         switch (cx & ((1u << CASE_BITS) - 1u)) {
             SPN_ALL_SP(SPN_CASE, 0)
             SPN_ALL_SP(SPN_CASE, 1)
@@ -385,15 +501,25 @@ __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &
             SPN_ALL_SP(SPN_CASE, 14)
             SPN_ALL_SP(SPN_CASE, 15)
             SPN_ALL_SP(SPN_CASE, 16)
+            SPN_ALL_SP(SPN_CASE, 17)
+            SPN_ALL_SP(SPN_CASE, 18)
+            SPN_ALL_SP(SPN_CASE, 19)
+            SPN_ALL_SP(SPN_CASE, 20)
+            SPN_ALL_SP(SPN_CASE, 21)
+            SPN_ALL_SP(SPN_CASE, 22)
             SPN_UNUSED_CASES
             default:
                 __builtin_unreachable();
         }
+        pc += 16;
+        cx = nx; cy = ny; cz = nz; cw = nw;
     }
 }
 
 // Load this warp's tile of x (rows [base, base+nrows)) transposed into
-// xw[f * tpw + s] (s = sample within the 32*K tile).
+// xw[f * tpw + s] (s = sample within the 32*K tile) with asynchronous 4-byte
+// copies (cp.async, LDGSTS): all of them are in flight at once, then one wait.
+// Rows past the end are zero-filled (src-size 0).
 __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__restrict__ x,
                                             int64_t base, int nrows, int64_t ld, int F,
                                             int lane, int WT) {
@@ -403,8 +529,11 @@ __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__r
     const float *xb = x + base * ld;
     const uint32_t xa = smem_u32(xw);
     for (int idx = lane; idx < total; idx += 32) {
-        const float v = (s < nrows) ? __ldg(xb + (int64_t)s * ld + f) : 0.f;
-        asm volatile("st.shared.f32 [%0], %1;" :: "r"(xa + 4u * (uint32_t)(f * tpw + s)), "f"(v)
+        const bool ok = s < nrows;
+        const float *src = ok ? xb + (int64_t)s * ld + f : x;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(
+                         xa + 4u * (uint32_t)(f * tpw + s)),
+                     "l"(src), "r"(ok ? 4 : 0)
                      : "memory");
         f += 32;
         while (f >= F) {
@@ -412,6 +541,7 @@ __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__r
             ++s;
         }
     }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
 }
 
 template <int K, bool MARG, bool XS>
@@ -506,9 +636,14 @@ template <int K, bool MARG, bool XS>
 cudaError_t dag_eval_launch_t(const KParams &p, int grid, int block, size_t smem,
                               cudaStream_t st) {
     auto fn = dag_eval_kernel<K, MARG, XS>;
-    cudaError_t err =
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (err != cudaSuccess) return err;
+    // the attribute persists per function: set it only when a larger size is needed
+    static size_t configured = 0;
+    if (smem > configured) {
+        cudaError_t err =
+            cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (err != cudaSuccess) return err;
+        configured = smem;
+    }
     fn<<<grid, block, smem, st>>>(p);
     return cudaGetLastError();
 }

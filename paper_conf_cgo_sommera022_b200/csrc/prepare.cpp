@@ -369,9 +369,10 @@ PartitionResult partition(const CGraph &c, int64_t cap) {
 
 // Pack a leaf's parameters.
 struct LeafPack {
-    uint32_t op;   // OP_GPUSH or OP_DPUSH (ACC = +1)
+    bool gauss;    // Gaussian (else discrete table)
     uint32_t f;    // feature
     uint32_t y, z, w;
+    double c;      // Gaussian: -log2(sigma sqrt(2 pi)) (pre-summed into LPUSH's C)
 };
 
 }  // namespace
@@ -417,7 +418,8 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             const double a = 1.0 / (sd * std::sqrt(2.0 * M_LN2));
             const double b = a * mu;
             const double cc = -std::log2(sd * std::sqrt(2.0 * M_PI));
-            lp.op = OP_GPUSH;
+            lp.gauss = true;
+            lp.c = cc;
             lp.y = fbits((float)a);
             lp.z = fbits((float)b);
             lp.w = fbits((float)cc);
@@ -442,7 +444,8 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
                     for (int64_t v = (int64_t)p[b]; v < (int64_t)p[b + 1]; ++v)
                         tab[v - lo] = (float)std::log2(p[b + 2]);
             }
-            lp.op = OP_DPUSH;
+            lp.gauss = false;
+            lp.c = 0.0;
             lp.y = (uint32_t)out.tables.size();
             lp.z = (uint32_t)(int32_t)lo;
             lp.w = (uint32_t)nk;
@@ -566,6 +569,9 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
     }
 
     // ---- code generation ----
+    // emit_value(u, sp, bias) leaves value(u) + bias at stack position sp.
+    // bias carries the parent sum's log2 weight (weights are folded into the
+    // records producing the children, so LSE records need no weight adds).
     struct Fix {
         int64_t idx;      // record index or edge index
         int64_t node;
@@ -574,35 +580,57 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
     std::vector<Fix> fixes;
     std::vector<Rec> &prog = out.prog;
     int64_t max_sp = 0;
+    bool overflow = false;
     auto rec_of = [&](uint32_t op, int sp, uint32_t arg, uint32_t y = 0, uint32_t z = 0,
                       uint32_t w = 0) {
-        if (sp > MAXD || sp < 0) return false;
+        if (sp > MAXD || sp < 0 || arg > ARG_MAX) {
+            overflow = true;
+            return;
+        }
         prog.push_back(make_rec(op, (uint32_t)sp, arg, y, z, w));
-        return true;
     };
     auto feat_arg = [&](uint32_t f) -> uint32_t {
         return cfg.x_in_smem ? f * (uint32_t)cfg.tpw * 4u : f * 4u;
     };
-    auto lw2 = [](double w) -> uint32_t { return fbits((float)std::log2(w)); };
-    bool overflow = false;
-
-    std::function<void(int64_t, int)> emit_value;
-    auto emit_leaf = [&](int64_t u, int sp, bool acc) {
-        const LeafPack &lp = leaf[u];
-        const int rsp = acc ? sp + 1 : sp;  // ACC: accumulator at r[sp], depth sp+1
+    auto lw2 = [](double w) -> double { return std::log2(w); };
+    // leaf product: LPUSH (acc=false, pushes at sp) or LACC (adds to r[sp])
+    auto emit_leaves = [&](const std::vector<int64_t> &lv, int sp, bool acc, double bias) {
+        double C = bias;
+        uint32_t ng = 0, nd = 0;
+        for (int64_t u : lv) {
+            if (leaf[u].gauss) {
+                C += leaf[u].c;
+                ++ng;
+            } else {
+                ++nd;
+            }
+        }
         if (!acc) max_sp = std::max<int64_t>(max_sp, sp + 1);
-        if (!rec_of(lp.op + (acc ? 1 : 0), rsp, feat_arg(lp.f), lp.y, lp.z, lp.w)) overflow = true;
+        if (nd == 0 && ng >= 1 && ng <= 4)  // straight-line variants
+            rec_of((acc ? OP_GACC1 : OP_GPUSH1) + ng - 1, acc ? sp + 1 : sp, 0, fbits((float)C));
+        else
+            rec_of(acc ? OP_LACC : OP_LPUSH, acc ? sp + 1 : sp, ng, fbits((float)C), nd);
+        for (int pass = 0; pass < 2; ++pass)
+            for (int64_t u : lv) {
+                const LeafPack &lp = leaf[u];
+                if (lp.gauss != (pass == 0)) continue;
+                prog.push_back(Rec{feat_arg(lp.f), lp.y, lp.z, lp.w});
+            }
     };
-    auto emit_load = [&](int64_t u, int sp) {
+    auto emit_load = [&](int64_t u, int sp, double bias) {
         max_sp = std::max<int64_t>(max_sp, sp + 1);
         fixes.push_back({(int64_t)prog.size(), u, 0});
-        if (!rec_of(OP_LDS, sp, 0)) overflow = true;
+        rec_of(OP_LDS, sp, 0, fbits((float)bias));
     };
-    std::vector<std::pair<int32_t, int64_t>> tmp;
-    emit_value = [&](int64_t u, int sp) {
+    std::function<void(int64_t, int, double)> emit_value;
+    auto emit_child = [&](int64_t ch, int sp, double bias) {
+        if (!is_leaf(c.kind[ch]) && mat[ch]) emit_load(ch, sp, bias);
+        else emit_value(ch, sp, bias);
+    };
+    emit_value = [&](int64_t u, int sp, double bias) {
         const int32_t k = c.kind[u];
         if (is_leaf(k)) {
-            emit_leaf(u, sp, false);
+            emit_leaves({u}, sp, false, bias);
             return;
         }
         if (k == SPN_PRODUCT) {
@@ -615,33 +643,34 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             }
             std::stable_sort(inner.begin(), inner.end(),
                              [](auto &a, auto &b) { return a.first > b.first; });
-            bool first = true;
-            for (auto &pr : inner) {
-                const int64_t ch = pr.second;
-                if (first) {
-                    if (mat[ch]) emit_load(ch, sp);
-                    else emit_value(ch, sp);
-                    first = false;
+            if (inner.empty()) {
+                emit_leaves(leaves, sp, false, bias);
+                return;
+            }
+            for (size_t i = 0; i < inner.size(); ++i) {
+                const bool last_add = leaves.empty() && i + 1 == inner.size();
+                if (i == 0) {
+                    emit_child(inner[i].second, sp, inner.size() == 1 && leaves.empty() ? bias : 0.0);
                 } else {
-                    if (mat[ch]) emit_load(ch, sp + 1);
-                    else emit_value(ch, sp + 1);
-                    if (!rec_of(OP_ADD, sp + 2, 0)) overflow = true;
+                    emit_child(inner[i].second, sp + 1, 0.0);
+                    rec_of(OP_ADD, sp + 2, 0, fbits((float)(last_add ? bias : 0.0)));
                 }
             }
-            for (int64_t lf : leaves) {
-                emit_leaf(lf, sp, !first);
-                first = false;
-            }
+            if (!leaves.empty()) emit_leaves(leaves, sp, true, bias);
             return;
         }
         // weighted sum
         const int64_t n = fan(u);
+        if (n == 1) {  // single-input sum with weight != 1: value + log2 w
+            emit_child(c.ch[c.cb[u]], sp, bias + lw2(c.w[c.cb[u]]));
+            return;
+        }
         if (glse[u]) {
             const int64_t off = (int64_t)out.edges.size();
             for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) {
                 const int64_t ch = c.ch[e];
                 Edge ed;
-                ed.lw = (float)std::log2(c.w[e]);
+                ed.lw = (float)(lw2(c.w[e]) + bias);
                 ed.pad = 0;
                 ed.a = 0;
                 ed.b = SLOT_NONE;
@@ -655,51 +684,29 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
                 out.edges.push_back(ed);
             }
             max_sp = std::max<int64_t>(max_sp, sp + 1);
-            if (!rec_of(OP_GLSE, sp, 0, (uint32_t)(off & 0xffffffffu), (uint32_t)(off >> 32),
-                        (uint32_t)n))
-                overflow = true;
+            rec_of(OP_GLSE, sp, 0, (uint32_t)(off & 0xffffffffu), (uint32_t)(off >> 32), (uint32_t)n);
             return;
         }
         std::vector<std::pair<int32_t, int64_t>> kids;  // (need, edge)
         for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) kids.push_back({child_need(c.ch[e]), e});
         std::stable_sort(kids.begin(), kids.end(),
                          [](auto &a, auto &b) { return a.first > b.first; });
-        auto push_child = [&](int64_t e, int at) {
-            const int64_t ch = c.ch[e];
-            if (!is_leaf(c.kind[ch]) && mat[ch]) emit_load(ch, at);
-            else emit_value(ch, at);
-        };
         if (n <= cfg.lse_max) {
-            uint32_t w[4] = {0, 0, 0, 0};
-            for (int64_t i = 0; i < n; ++i) {
-                push_child(kids[i].second, sp + (int)i);
-                w[i] = lw2(c.w[kids[i].second]);
-            }
-            const uint32_t op = OP_LSE1 + (uint32_t)(n - 1);
-            if (!rec_of(op, sp + (int)n, 0, w[0], w[1], w[2])) overflow = true;
-            if (n == 4) prog.push_back(Rec{w[3], 0, 0, 0});
+            for (int64_t i = 0; i < n; ++i)
+                emit_child(c.ch[kids[i].second], sp + (int)i, lw2(c.w[kids[i].second]));
+            rec_of(OP_LSE1 + (uint32_t)(n - 1), sp + (int)n, 0, fbits((float)bias));
             return;
         }
-        // chunked: first 4 children, then (accumulator + 3 children) per chunk
-        {
-            uint32_t w[4];
-            for (int i = 0; i < 4; ++i) {
-                push_child(kids[i].second, sp + i);
-                w[i] = lw2(c.w[kids[i].second]);
-            }
-            if (!rec_of(OP_LSE4, sp + 4, 0, w[0], w[1], w[2])) overflow = true;
-            prog.push_back(Rec{w[3], 0, 0, 0});
-        }
+        // chunked: first 4 children, then (accumulator + up to 3 children)
+        for (int i = 0; i < 4; ++i)
+            emit_child(c.ch[kids[i].second], sp + i, lw2(c.w[kids[i].second]));
+        rec_of(OP_LSE4, sp + 4, 0, fbits(n == 4 ? (float)bias : 0.f));
         for (int64_t i = 4; i < n; i += 3) {
             const int64_t m = std::min<int64_t>(3, n - i);
-            uint32_t w[4] = {fbits(0.f), 0, 0, 0};
-            for (int64_t j = 0; j < m; ++j) {
-                push_child(kids[i + j].second, sp + 1 + (int)j);
-                w[j + 1] = lw2(c.w[kids[i + j].second]);
-            }
-            const uint32_t op = OP_LSE1 + (uint32_t)m;  // m+1 inputs
-            if (!rec_of(op, sp + 1 + (int)m, 0, w[0], w[1], w[2])) overflow = true;
-            if (m + 1 == 4) prog.push_back(Rec{w[3], 0, 0, 0});
+            for (int64_t j = 0; j < m; ++j)
+                emit_child(c.ch[kids[i + j].second], sp + 1 + (int)j, lw2(c.w[kids[i + j].second]));
+            const bool last = i + m >= n;
+            rec_of(OP_LSE1 + (uint32_t)m, sp + 1 + (int)m, 0, fbits(last ? (float)bias : 0.f));
         }
     };
 
@@ -713,11 +720,11 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             const bool is_root = !c.rootrefs[u].empty();
             if (is_leaf(c.kind[u])) {
                 if (!is_root) continue;
-                emit_leaf(u, 0, false);
+                emit_leaves({u}, 0, false, 0.0);
             } else {
                 if (virt[u]) continue;
                 if (!mat[u] && !is_root) continue;  // emitted inside its consumer
-                emit_value(u, 0);
+                emit_value(u, 0, 0.0);
                 if (mat[u]) {
                     store_rec[u] = (int64_t)prog.size();
                     fixes.push_back({(int64_t)prog.size(), u, 1});
@@ -745,7 +752,12 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             const int64_t off = ((int64_t)prog[i].z << 32) | prog[i].y;
             for (int64_t e = off; e < off + (int64_t)prog[i].w; ++e) edge_rec[e] = i;
         }
-        if (cs / NSP == OP_LSE4 && cs < OP_COUNT * NSP) ++i;  // skip weight record
+        if ((cs / NSP == OP_LPUSH || cs / NSP == OP_LACC) && cs < OP_COUNT * NSP)
+            i += (int64_t)(prog[i].x >> CASE_BITS) + (int64_t)prog[i].z;  // skip leaf params
+        else if (cs / NSP >= OP_GPUSH1 && cs / NSP <= OP_GPUSH4)
+            i += cs / NSP - OP_GPUSH1 + 1;
+        else if (cs / NSP >= OP_GACC1 && cs / NSP <= OP_GACC4)
+            i += cs / NSP - OP_GACC1 + 1;
     }
     for (const Fix &f : fixes) {
         if (f.kind == 0) last_use[f.node] = std::max(last_use[f.node], f.idx);

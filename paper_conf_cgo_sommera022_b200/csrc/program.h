@@ -8,24 +8,29 @@
 // case = op * 17 + sp and sp = stack depth BEFORE the op (0..16); y, z, w are
 // operands.  The static sp lets the kernel keep the stack in registers: every
 // (op, sp) pair is its own case of one dense switch (a single jump table), with
-// constant register indices.  Feature and slot operands are pre-multiplied by
-// the preparer into float offsets (feature * tile stride, slot * 32K).
+// constant register indices.  Feature and slot operands are byte offsets
+// pre-multiplied by the preparer (feature * 4 * tile stride, slot * 128 * K).
+// Sum weights are folded into the records producing the children ("bias"),
+// so the LSE records carry no weights.
 //
-//   GPUSH  f | a, b, c      r[sp]   = c - (a*x_f - b)^2         Gaussian leaf
-//   GACC   f | a, b, c      r[sp-1] += c - (a*x_f - b)^2        leaf into product
-//   DPUSH  f | tab, lo, K   r[sp]   = x in [lo,lo+K) ? tab[floor(x)-lo] : -inf
-//   DACC   f | tab, lo, K   r[sp-1] += (same)                   discrete leaf
-//   ADD                     r[sp-2] += r[sp-1]                   product edge
-//   LSE1..4  | w0, w1, w2   r[sp-n] = LSE_i(r[sp-n+i] + w_i)     weighted sum
-//              (LSE4: w3 in the x word of the following record)
-//   LDS/LDG s               r[sp]   = slot_s   (shared / global scratch)
-//   STS/STG s               slot_s  = r[sp-1]  (the next record's sp pops)
-//   GLSE     | off_lo, off_hi, n   r[sp] = LSE over edge terms (slots)
-//   OUT    r                out[., r] = ln2 * r[sp-1]
+//   LPUSH  ng | C, nd        r[sp]   = C + sum of ng Gaussian + nd discrete leaves
+//   LACC   ng | C, nd        r[sp-1] += (same)          (leaf children of a product)
+//   GPUSHn / GACCn  | C      same for exactly n <= 4 Gaussian leaves (no loop)
+//       followed by ng Gaussian parameter records {f, a, b, c} and nd discrete
+//       records {f, table, lo, K}.  Gaussian: c - (a*x_f - b)^2 = log2 N(x; mu, s)
+//       with a = 1/(s sqrt(2 ln2)), b = a mu, c = -log2(s sqrt(2 pi)); the c's
+//       (and the bias) are pre-summed into C, so a leaf costs 2 FFMA: t = a x - b,
+//       acc -= t*t.  Marginal kernels subtract c instead of t^2 for a NaN input
+//       (log 1 = 0).  Discrete: x in [lo, lo+K) ? table[floor(x)-lo] : -inf.
+//   ADD      | bias          r[sp-2] += r[sp-1] + bias           product edge
+//   LSE1..4  | bias          r[sp-n] = LSE_i(r[sp-n+i]) + bias   weighted sum: the
+//                            largest input is the shift m, so its ex2(0)=1 needs no
+//                            MUFU: n-1 ex2 + 1 lg2 per sum
+//   LDS/LDG s | bias         r[sp]   = slot_s + bias   (shared / global scratch)
+//   STS/STG s                slot_s  = r[sp-1]  (the next record's sp pops)
+//   GLSE     | off_lo, off_hi, n   r[sp] = LSE over edge terms slot(a)[+slot(b)]+lw
+//   OUT    r                 out[., r] = ln2 * r[sp-1]
 //   END
-// Leaves: a = 1/(sigma*sqrt(2 ln 2)), b = a*mu, c = -log2(sigma*sqrt(2 pi)),
-// so c - (a x - b)^2 = log2 N(x; mu, sigma).  Marginal kernels replace a leaf
-// whose input is NaN by 0 (= log 1).
 #pragma once
 #include <stdint.h>
 
@@ -33,23 +38,29 @@ namespace spnb {
 
 enum Op : uint32_t {
     OP_END = 0,
-    OP_GPUSH = 1,
-    OP_GACC = 2,
-    OP_DPUSH = 3,
-    OP_DACC = 4,
-    OP_ADD = 5,
-    OP_LSE1 = 6,
-    OP_LSE2 = 7,
-    OP_LSE3 = 8,
-    OP_LSE4 = 9,
-    OP_LDS = 10,
-    OP_LDG = 11,
-    OP_STS = 12,
-    OP_STG = 13,
-    OP_GLSE = 14,
-    OP_OUT = 15,
-    OP_NOP = 16,
-    OP_COUNT = 17
+    OP_LPUSH = 1,   // generic leaf product (loop; Gaussian + discrete leaves)
+    OP_LACC = 2,
+    OP_ADD = 3,
+    OP_LSE1 = 4,
+    OP_LSE2 = 5,
+    OP_LSE3 = 6,
+    OP_LSE4 = 7,
+    OP_LDS = 8,
+    OP_LDG = 9,
+    OP_STS = 10,
+    OP_STG = 11,
+    OP_GLSE = 12,
+    OP_OUT = 13,
+    OP_NOP = 14,
+    OP_GPUSH1 = 15, // straight-line products of 1..4 Gaussian leaves
+    OP_GPUSH2 = 16,
+    OP_GPUSH3 = 17,
+    OP_GPUSH4 = 18,
+    OP_GACC1 = 19,
+    OP_GACC2 = 20,
+    OP_GACC3 = 21,
+    OP_GACC4 = 22,
+    OP_COUNT = 23
 };
 
 constexpr int MAXD = 16;              // register stack depth

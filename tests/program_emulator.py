@@ -12,8 +12,9 @@ from __future__ import annotations
 import numpy as np
 
 NSP = 17
-OPS = ["END", "GPUSH", "GACC", "DPUSH", "DACC", "ADD", "LSE1", "LSE2", "LSE3", "LSE4",
-       "LDS", "LDG", "STS", "STG", "GLSE", "OUT", "NOP"]
+OPS = ["END", "LPUSH", "LACC", "ADD", "LSE1", "LSE2", "LSE3", "LSE4",
+       "LDS", "LDG", "STS", "STG", "GLSE", "OUT", "NOP",
+       "GPUSH1", "GPUSH2", "GPUSH3", "GPUSH4", "GACC1", "GACC2", "GACC3", "GACC4"]
 SLOT_GLOBAL = 0x80000000
 SLOT_NONE = 0xFFFFFFFF
 
@@ -66,43 +67,51 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
             op, sp = OPS[case // NSP] if case // NSP < len(OPS) else "BAD", case % NSP
             if op == "END":
                 break
-            if op in ("GPUSH", "GACC"):
-                xv = xd[:, feat(arg)]
-                a, b, c = _f32(r["y"]), _f32(r["z"]), _f32(r["w"])
-                v = c - (a * xv - b) ** 2
-                if marginal:
-                    v = np.where(np.isnan(xv), 0.0, v)
-                if op == "GPUSH":
-                    stack[sp] = v
+            if op[:5] in ("GPUSH", "GACC1", "GACC2", "GACC3", "GACC4"):
+                ng, nd = int(op[-1]), 0
+                op = "LPUSH" if op.startswith("GPUSH") else "LACC"
+            elif op in ("LPUSH", "LACC"):
+                ng, nd = arg, int(r["z"])
+            if op in ("LPUSH", "LACC"):
+                C = _f32(r["y"])
+                acc = np.full(N, C)
+                for i in range(ng):
+                    q = rec[pc]
+                    pc += 1
+                    xv = xd[:, feat(int(q["x"]))]
+                    a, b, c = _f32(q["y"]), _f32(q["z"]), _f32(q["w"])
+                    t = a * xv - b
+                    if marginal:
+                        acc = acc - np.where(np.isnan(xv), c, t * t)
+                    else:
+                        acc = acc - t * t
+                for i in range(nd):
+                    q = rec[pc]
+                    pc += 1
+                    xv = xd[:, feat(int(q["x"]))]
+                    off, lo, nk = int(q["y"]), int(np.int32(np.uint32(q["z"]))), int(q["w"])
+                    ok = (xv >= lo) & (xv < lo + nk)
+                    idx = np.where(ok, np.floor(np.where(ok, xv, lo)) - lo, 0).astype(np.int64)
+                    v = np.where(ok, tables[off + idx], -np.inf)
+                    v = np.where(np.isnan(xv), 0.0 if marginal else np.nan, v)
+                    acc = acc + v
+                if op == "LPUSH":
+                    stack[sp] = acc
                 else:
-                    stack[sp - 1] = stack[sp - 1] + v
-            elif op in ("DPUSH", "DACC"):
-                xv = xd[:, feat(arg)]
-                off, lo, nk = int(r["y"]), int(np.int32(np.uint32(r["z"]))), int(r["w"])
-                ok = (xv >= lo) & (xv < lo + nk)
-                idx = np.where(ok, np.floor(np.where(ok, xv, lo)) - lo, 0).astype(np.int64)
-                v = np.where(ok, tables[off + idx], -np.inf)
-                v = np.where(np.isnan(xv), 0.0 if marginal else np.nan, v)
-                if op == "DPUSH":
-                    stack[sp] = v
-                else:
-                    stack[sp - 1] = stack[sp - 1] + v
+                    stack[sp - 1] = stack[sp - 1] + acc
             elif op == "ADD":
-                stack[sp - 2] = stack[sp - 2] + stack[sp - 1]
+                stack[sp - 2] = stack[sp - 2] + stack[sp - 1] + _f32(r["y"])
             elif op.startswith("LSE"):
                 n = int(op[3])
-                w = [_f32(r["y"]), _f32(r["z"]), _f32(r["w"])]
-                if n == 4:
-                    w.append(_f32(rec[pc]["x"]))
-                    pc += 1
+                bias = _f32(r["y"])
                 if n == 1:
-                    stack[sp - 1] = stack[sp - 1] + w[0]
+                    stack[sp - 1] = stack[sp - 1] + bias
                 else:
-                    stack[sp - n] = _lse([stack[sp - n + i] + w[i] for i in range(n)])
+                    stack[sp - n] = _lse([stack[sp - n + i] for i in range(n)]) + bias
             elif op == "LDS":
-                stack[sp] = sslots[arg // slot_bytes]
+                stack[sp] = sslots[arg // slot_bytes] + _f32(r["y"])
             elif op == "LDG":
-                stack[sp] = gslots[arg // slot_bytes]
+                stack[sp] = gslots[arg // slot_bytes] + _f32(r["y"])
             elif op == "STS":
                 sslots[arg // slot_bytes] = stack[sp - 1].copy()
             elif op == "STG":

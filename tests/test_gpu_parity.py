@@ -176,8 +176,13 @@ def test_empty_batch_and_strided_input():
     _cmp(out.cpu().numpy(), ref)
     e, _ = P.infer(big[:0])                     # n = 0 no-op
     assert e.shape == (0, 1)
-    with pytest.raises(spnb.SPNError):
-        P.infer(big[:, :20])                    # ld < F
+    with pytest.raises(ValueError):
+        P.infer(big[:, :20])                    # fewer columns than features
+    lib = spnb.load_library()
+    import ctypes
+    rc = lib.spn_infer_joint(P._h, ctypes.c_void_p(big.data_ptr()), 10, 20,
+                             ctypes.c_void_p(out.data_ptr()), None, None)
+    assert rc == -1                             # SPN_E_ARG: ld < n_features
 
 
 def test_shard_invariance_bitwise():

@@ -230,6 +230,31 @@ __device__ __forceinline__ float max_nan(float a, float b) {  // NaN-propagating
 //   r = hi + bias + lg2(1 + sum_i ex2(lo_i - hi))
 // hi is NaN-propagating (reading c7); with all inputs -inf the shift is
 // clamped so the result is -inf, not NaN (reading c8).
+template <int N>
+__device__ __forceinline__ float lse_vals(const float (&v)[N], float bias) {
+    float hi, lo[N - 1];
+    if constexpr (N == 2) {
+        hi = max_nan(v[0], v[1]);
+        lo[0] = fminf(v[0], v[1]);
+    } else if constexpr (N == 3) {
+        const float m01 = fmaxf(v[0], v[1]);
+        lo[0] = fminf(v[0], v[1]);
+        lo[1] = fminf(m01, v[2]);
+        hi = max_nan(max_nan(v[0], v[1]), v[2]);
+    } else {
+        const float m01 = fmaxf(v[0], v[1]), m23 = fmaxf(v[2], v[3]);
+        lo[0] = fminf(v[0], v[1]);
+        lo[1] = fminf(v[2], v[3]);
+        lo[2] = fminf(m01, m23);
+        hi = max_nan(max_nan(v[0], v[1]), max_nan(v[2], v[3]));
+    }
+    const float hc = fmaxf(hi, -1e30f);
+    float s = 1.f;
+#pragma unroll
+    for (int i = 0; i < N - 1; ++i) s += ex2a(lo[i] - hc);
+    return (hi + bias) + lg2a(s);
+}
+
 template <int S, int N, int K>
 __device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float bias) {
     FOR_K {
@@ -239,41 +264,62 @@ __device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float bias) {
             float v[N];
 #pragma unroll
             for (int i = 0; i < N; ++i) v[i] = r[S - N + i][j];
-            float hi, lo[N - 1];
-            if constexpr (N == 2) {
-                hi = max_nan(v[0], v[1]);
-                lo[0] = fminf(v[0], v[1]);
-            } else if constexpr (N == 3) {
-                const float m01 = fmaxf(v[0], v[1]);
-                lo[0] = fminf(v[0], v[1]);
-                lo[1] = fminf(m01, v[2]);
-                hi = max_nan(max_nan(v[0], v[1]), v[2]);
-            } else {
-                const float m01 = fmaxf(v[0], v[1]), m23 = fmaxf(v[2], v[3]);
-                lo[0] = fminf(v[0], v[1]);
-                lo[1] = fminf(v[2], v[3]);
-                lo[2] = fminf(m01, m23);
-                hi = max_nan(max_nan(v[0], v[1]), max_nan(v[2], v[3]));
-            }
-            const float hc = fmaxf(hi, -1e30f);
-            float s = 1.f;
-#pragma unroll
-            for (int i = 0; i < N - 1; ++i) s += ex2a(lo[i] - hc);
-            r[S - N][j] = (hi + bias) + lg2a(s);
+            r[S - N][j] = lse_vals<N>(v, bias);
         }
     }
 }
 
+// One Gaussian leaf (parameter record at pp) accumulated into acc.
+template <int K, bool MARG, bool XS>
+__device__ __forceinline__ void gauss_acc(float (&acc)[K], uint32_t pp, const Env<K, MARG, XS> &e) {
+    uint32_t f, ya, zb, wc;
+    lds4(pp, f, ya, zb, wc);
+    float xv[K];
+    e.loadx(f, xv);
+    const float a = __uint_as_float(ya), b = __uint_as_float(zb);
+    FOR_K {
+        const float t = fmaf(a, xv[j], -b);
+        if constexpr (MARG) {
+            const bool nan = xv[j] != xv[j];
+            const float pv = nan ? __uint_as_float(wc) : t;
+            const float qv = nan ? 1.f : t;
+            acc[j] = fmaf(-pv, qv, acc[j]);
+        } else {
+            acc[j] = fmaf(-t, t, acc[j]);
+        }
+    }
+}
+
+// Fused weighted sum over KC Gaussian leaf products (SLPk record).
+template <int S, int KC, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_slp(float (&r)[MAXD][K], uint32_t counts, float bias,
+                                      const float (&Cs)[4], uint32_t pp,
+                                      const Env<K, MARG, XS> &e) {
+    float v[KC][K];
+#pragma unroll
+    for (int c = 0; c < KC; ++c) {
+        const uint32_t nc = (counts >> (3 * c)) & 7u;
+        float acc[K];
+        FOR_K acc[j] = Cs[c];
+#pragma unroll 1
+        for (uint32_t i = 0; i < nc; ++i, pp += 16) gauss_acc<K, MARG, XS>(acc, pp, e);
+        FOR_K v[c][j] = acc[j];
+    }
+    FOR_K {
+        float w[KC];
+#pragma unroll
+        for (int c = 0; c < KC; ++c) w[c] = v[c][j];
+        r[S][j] = lse_vals<KC>(w, bias);
+    }
+}
+
 // Straight-line product of exactly N Gaussian leaves (parameter records at pp).
-// The next program record (at pp + 16 N) is loaded alongside the parameters.
 template <int S, bool ACC, int N, int K, bool MARG, bool XS>
 __device__ __forceinline__ void h_gprod(float (&r)[MAXD][K], float C, uint32_t pp,
-                                        const Env<K, MARG, XS> &e, uint32_t &nx, uint32_t &ny,
-                                        uint32_t &nz, uint32_t &nw) {
+                                        const Env<K, MARG, XS> &e) {
     uint32_t f[N], ya[N], zb[N], wc[N];
 #pragma unroll
     for (int i = 0; i < N; ++i) lds4(pp + 16 * i, f[i], ya[i], zb[i], wc[i]);
-    lds4(pp + 16 * N, nx, ny, nz, nw);
     float xv[N][K];
 #pragma unroll
     for (int i = 0; i < N; ++i) e.loadx(f[i], xv[i]);
@@ -384,7 +430,7 @@ __device__ __forceinline__ void h_out(float (&r)[MAXD][K], uint32_t root,
 // Valid stack depths per op (sp = depth before the op).
 __host__ __device__ constexpr bool op_valid(int op, int sp) {
     return (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
-            (op >= OP_GPUSH1 && op <= OP_GPUSH4))
+            (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4))
                ? (sp >= 0 && sp < MAXD)
            : (op == OP_LACC || op == OP_LSE1 || op == OP_STS || op == OP_STG || op == OP_OUT ||
               (op >= OP_GACC1 && op <= OP_GACC4))
@@ -410,67 +456,132 @@ __host__ __device__ constexpr bool op_valid(int op, int sp) {
         break;
 
 #define SPN_BODY_0(S) ;
+// Every body captures its operands, advances pc, issues the load of the next
+// record into (cx, cy, cz, cw) -- so its latency overlaps the body -- and then
+// computes.
+#define SPN_NEXT(NEWPC)                                                          \
+    pc = (NEWPC);                                                                \
+    lds4(pc, cx, cy, cz, cw);
+#define SPN_SS(S) (S < MAXD ? S : 0)
 #define SPN_BODY_1(S)                                                            \
-    pc = h_lprod<(S < MAXD ? S : 0), false>(r, arg, __uint_as_float(cy), cz, pc + 16, e) - 16; \
-    lds4(pc + 16, nx, ny, nz, nw);
+    {                                                                            \
+        const uint32_t ng = cx >> CASE_BITS, nd = cz, pp = pc + 16;              \
+        const float C = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16 * (1 + ng + nd))                                        \
+        h_lprod<SPN_SS(S), false>(r, ng, C, nd, pp, e);                          \
+    }
 #define SPN_BODY_2(S)                                                            \
-    pc = h_lprod<S, true>(r, arg, __uint_as_float(cy), cz, pc + 16, e) - 16;      \
-    lds4(pc + 16, nx, ny, nz, nw);
-#define SPN_BODY_3(S) { FOR_K r[S - 2][j] += r[S - 1][j] + __uint_as_float(cy); }
-#define SPN_BODY_4(S) h_lse<S, 1>(r, __uint_as_float(cy));
-#define SPN_BODY_5(S) h_lse<S, 2>(r, __uint_as_float(cy));
-#define SPN_BODY_6(S) h_lse<S, 3>(r, __uint_as_float(cy));
-#define SPN_BODY_7(S) h_lse<S, 4>(r, __uint_as_float(cy));
+    {                                                                            \
+        const uint32_t ng = cx >> CASE_BITS, nd = cz, pp = pc + 16;              \
+        const float C = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16 * (1 + ng + nd))                                        \
+        h_lprod<S, true>(r, ng, C, nd, pp, e);                                   \
+    }
+#define SPN_BODY_3(S)                                                            \
+    {                                                                            \
+        const float b = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16)                                                        \
+        FOR_K r[S - 2][j] += r[S - 1][j] + b;                                    \
+    }
+#define SPN_LSE_BODY(S, N)                                                       \
+    {                                                                            \
+        const float b = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16)                                                        \
+        h_lse<S, N>(r, b);                                                       \
+    }
+#define SPN_BODY_4(S) SPN_LSE_BODY(S, 1)
+#define SPN_BODY_5(S) SPN_LSE_BODY(S, 2)
+#define SPN_BODY_6(S) SPN_LSE_BODY(S, 3)
+#define SPN_BODY_7(S) SPN_LSE_BODY(S, 4)
 #define SPN_BODY_8(S)                                                            \
     {                                                                            \
-        SIO<K>::ld(e.ss + arg, r[S < MAXD ? S : 0]);                             \
-        FOR_K r[S < MAXD ? S : 0][j] += __uint_as_float(cy);                     \
+        const uint32_t a = cx >> CASE_BITS;                                      \
+        const float b = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16)                                                        \
+        SIO<K>::ld(e.ss + a, r[SPN_SS(S)]);                                      \
+        FOR_K r[SPN_SS(S)][j] += b;                                              \
     }
 #define SPN_BODY_9(S)                                                            \
     {                                                                            \
-        GIO<K>::ld(reinterpret_cast<const float *>(e.gs + arg), r[S < MAXD ? S : 0]); \
-        FOR_K r[S < MAXD ? S : 0][j] += __uint_as_float(cy);                     \
+        const uint32_t a = cx >> CASE_BITS;                                      \
+        const float b = __uint_as_float(cy);                                     \
+        SPN_NEXT(pc + 16)                                                        \
+        GIO<K>::ld(reinterpret_cast<const float *>(e.gs + a), r[SPN_SS(S)]);     \
+        FOR_K r[SPN_SS(S)][j] += b;                                              \
     }
-#define SPN_BODY_10(S) SIO<K>::st(e.ss + arg, r[S - 1]);
-#define SPN_BODY_11(S) GIO<K>::st(reinterpret_cast<float *>(e.gs + arg), r[S - 1]);
+#define SPN_BODY_10(S)                                                           \
+    {                                                                            \
+        const uint32_t a = cx >> CASE_BITS;                                      \
+        SPN_NEXT(pc + 16)                                                        \
+        SIO<K>::st(e.ss + a, r[S - 1]);                                          \
+    }
+#define SPN_BODY_11(S)                                                           \
+    {                                                                            \
+        const uint32_t a = cx >> CASE_BITS;                                      \
+        SPN_NEXT(pc + 16)                                                        \
+        GIO<K>::st(reinterpret_cast<float *>(e.gs + a), r[S - 1]);               \
+    }
 #define SPN_BODY_12(S)                                                           \
     {                                                                            \
-        const VecK<K> g = h_glse<K>(e.edges + (((uint64_t)cz << 32) | cy),        \
-                                    (int)cw, e.ss, e.gs);                        \
-        FOR_K r[S < MAXD ? S : 0][j] = g.v[j];                                   \
+        const Edge *E = e.edges + (((uint64_t)cz << 32) | cy);                   \
+        const int n = (int)cw;                                                   \
+        SPN_NEXT(pc + 16)                                                        \
+        const VecK<K> g = h_glse<K>(E, n, e.ss, e.gs);                           \
+        FOR_K r[SPN_SS(S)][j] = g.v[j];                                          \
     }
-#define SPN_BODY_13(S) h_out<S>(r, arg, e, am);
-#define SPN_BODY_14(S) ;
-#define SPN_BODY_15(S)                                                       \
-    h_gprod<(S < MAXD ? S : 0), false, 1>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
-    pc += 16;
-#define SPN_BODY_16(S)                                                       \
-    h_gprod<(S < MAXD ? S : 0), false, 2>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
-    pc += 32;
-#define SPN_BODY_17(S)                                                       \
-    h_gprod<(S < MAXD ? S : 0), false, 3>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
-    pc += 48;
-#define SPN_BODY_18(S)                                                       \
-    h_gprod<(S < MAXD ? S : 0), false, 4>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw); \
-    pc += 64;
-#define SPN_BODY_19(S)                                                       \
-    h_gprod<S, true, 1>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
-    pc += 16;
-#define SPN_BODY_20(S)                                                       \
-    h_gprod<S, true, 2>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
-    pc += 32;
-#define SPN_BODY_21(S)                                                       \
-    h_gprod<S, true, 3>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
-    pc += 48;
-#define SPN_BODY_22(S)                                                       \
-    h_gprod<S, true, 4>(r, __uint_as_float(cy), pc + 16, e, nx, ny, nz, nw);    \
-    pc += 64;
-#define SPN_UNUSED_CASES case 391: case 392: case 393: case 394: case 395: case 396: case 397: case 398: case 399: case 400: case 401: case 402: case 403: case 404: case 405: case 406: case 407: case 408: case 409: case 410: case 411: case 412: case 413: case 414: case 415: case 416: case 417: case 418: case 419: case 420: case 421: case 422: case 423: case 424: case 425: case 426: case 427: case 428: case 429: case 430: case 431: case 432: case 433: case 434: case 435: case 436: case 437: case 438: case 439: case 440: case 441: case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
+#define SPN_BODY_13(S)                                                           \
+    {                                                                            \
+        const uint32_t root = cx >> CASE_BITS;                                   \
+        SPN_NEXT(pc + 16)                                                        \
+        h_out<S>(r, root, e, am);                                                \
+    }
+#define SPN_BODY_14(S) SPN_NEXT(pc + 16)
+#define SPN_GPROD_BODY(S, ACC, N)                                                \
+    {                                                                            \
+        const float C = __uint_as_float(cy);                                     \
+        const uint32_t pp = pc + 16;                                             \
+        SPN_NEXT(pc + 16 * (N + 1))                                              \
+        h_gprod<S, ACC, N>(r, C, pp, e);                                         \
+    }
+#define SPN_BODY_15(S) SPN_GPROD_BODY(SPN_SS(S), false, 1)
+#define SPN_BODY_16(S) SPN_GPROD_BODY(SPN_SS(S), false, 2)
+#define SPN_BODY_17(S) SPN_GPROD_BODY(SPN_SS(S), false, 3)
+#define SPN_BODY_18(S) SPN_GPROD_BODY(SPN_SS(S), false, 4)
+#define SPN_BODY_19(S) SPN_GPROD_BODY(S, true, 1)
+#define SPN_BODY_20(S) SPN_GPROD_BODY(S, true, 2)
+#define SPN_BODY_21(S) SPN_GPROD_BODY(S, true, 3)
+#define SPN_BODY_22(S) SPN_GPROD_BODY(S, true, 4)
+#define SPN_SLP_BODY(S, KC)                                                      \
+    {                                                                            \
+        const uint32_t counts = cx >> CASE_BITS;                                 \
+        float Cs[4];                                                             \
+        Cs[0] = __uint_as_float(cz);                                             \
+        Cs[1] = __uint_as_float(cw);                                             \
+        Cs[2] = 0.f;                                                             \
+        Cs[3] = 0.f;                                                             \
+        const float bias = __uint_as_float(cy);                                  \
+        uint32_t pp = pc + 16;                                                   \
+        if (KC >= 3) {                                                           \
+            uint32_t c2, c3, u0, u1;                                             \
+            lds4(pp, c2, c3, u0, u1);                                            \
+            Cs[2] = __uint_as_float(c2);                                         \
+            Cs[3] = __uint_as_float(c3);                                         \
+            pp += 16;                                                            \
+        }                                                                        \
+        const uint32_t tot = (counts & 7u) + ((counts >> 3) & 7u) +              \
+                             ((counts >> 6) & 7u) + ((counts >> 9) & 7u);         \
+        SPN_NEXT(pp + 16 * tot)                                                  \
+        h_slp<SPN_SS(S), KC>(r, counts, bias, Cs, pp, e);                        \
+    }
+#define SPN_BODY_23(S) SPN_SLP_BODY(S, 2)
+#define SPN_BODY_24(S) SPN_SLP_BODY(S, 3)
+#define SPN_BODY_25(S) SPN_SLP_BODY(S, 4)
+#define SPN_UNUSED_CASES case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
 
 // Run one task's program (shared memory at byte address prog) for this
 // thread's K samples.  All case labels 0..511 exist, so the dispatch is one
-// unchecked jump-table lookup (build with nvcc -jtd 10).  The next record is
-// loaded before the current one is dispatched (software prefetch).
+// unchecked jump-table lookup (build with nvcc -jtd 10).  Each case loads the
+// next record right after reading its own operands (see SPN_NEXT).
 template <int K, bool MARG, bool XS>
 __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &e,
                                          ArgState<K> &am) {
@@ -479,10 +590,6 @@ __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &
     uint32_t cx, cy, cz, cw;
     lds4(pc, cx, cy, cz, cw);
     for (;;) {
-        uint32_t nx, ny, nz, nw;
-        lds4(pc + 16, nx, ny, nz, nw);
-        const uint32_t arg = cx >> CASE_BITS;
-        (void)arg;
         switch (cx & ((1u << CASE_BITS) - 1u)) {
             SPN_ALL_SP(SPN_CASE, 0)
             SPN_ALL_SP(SPN_CASE, 1)
@@ -507,12 +614,13 @@ __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &
             SPN_ALL_SP(SPN_CASE, 20)
             SPN_ALL_SP(SPN_CASE, 21)
             SPN_ALL_SP(SPN_CASE, 22)
+            SPN_ALL_SP(SPN_CASE, 23)
+            SPN_ALL_SP(SPN_CASE, 24)
+            SPN_ALL_SP(SPN_CASE, 25)
             SPN_UNUSED_CASES
             default:
                 __builtin_unreachable();
         }
-        pc += 16;
-        cx = nx; cy = ny; cz = nz; cw = nw;
     }
 }
 

@@ -1,0 +1,444 @@
+// layered.cpp -- detection of RAT-SPN-style region graphs and construction of
+// the tensor-core plan (see layered.h, rat_eval.cu).
+#include "layered.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <unordered_map>
+
+#include "spnb.h"
+
+namespace spnb {
+
+namespace {
+
+inline bool is_leafk(int32_t k) {
+    return k == SPN_GAUSSIAN || k == SPN_CATEGORICAL || k == SPN_HISTOGRAM;
+}
+
+uint16_t f32_to_f16(float f) {
+    // round-to-nearest-even conversion (host)
+    uint32_t x;
+    memcpy(&x, &f, 4);
+    const uint32_t sign = (x >> 16) & 0x8000u;
+    int32_t exp = (int32_t)((x >> 23) & 0xff) - 127 + 15;
+    uint32_t man = x & 0x7fffffu;
+    if (((x >> 23) & 0xff) == 0xff) return (uint16_t)(sign | 0x7c00u | (man ? 0x200u : 0));
+    if (exp >= 31) return (uint16_t)(sign | 0x7c00u);
+    if (exp <= 0) {
+        if (exp < -10) return (uint16_t)sign;
+        man |= 0x800000u;
+        const int shift = 14 - exp;
+        uint32_t h = man >> shift;
+        const uint32_t rem = man & ((1u << shift) - 1);
+        const uint32_t half = 1u << (shift - 1);
+        if (rem > half || (rem == half && (h & 1))) ++h;
+        return (uint16_t)(sign | h);
+    }
+    uint32_t h = ((uint32_t)exp << 10) | (man >> 13);
+    const uint32_t rem = man & 0x1fffu;
+    if (rem > 0x1000u || (rem == 0x1000u && (h & 1))) ++h;
+    return (uint16_t)(sign | h);
+}
+
+float f16_to_f32(uint16_t h) {
+    const uint32_t sign = (uint32_t)(h & 0x8000u) << 16;
+    uint32_t exp = (h >> 10) & 0x1f, man = h & 0x3ffu;
+    uint32_t x;
+    if (exp == 0) {
+        if (man == 0) {
+            x = sign;
+        } else {
+            int e = -1;
+            do {
+                ++e;
+                man <<= 1;
+            } while (!(man & 0x400u));
+            x = sign | ((uint32_t)(127 - 15 - e) << 23) | ((man & 0x3ffu) << 13);
+        }
+    } else if (exp == 31) {
+        x = sign | 0x7f800000u | (man << 13);
+    } else {
+        x = sign | ((exp - 15 + 127) << 23) | (man << 13);
+    }
+    float f;
+    memcpy(&f, &x, 4);
+    return f;
+}
+
+uint64_t hash_vec(const std::vector<int64_t> &v) {
+    uint64_t h = 1469598103934665603ull;
+    for (int64_t x : v) {
+        h ^= (uint64_t)x + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
+        h *= 1099511628211ull;
+    }
+    return h;
+}
+
+struct Region {
+    bool leaf = false;
+    std::vector<int64_t> nodes;          // value index -> canonical node
+    std::vector<int32_t> vars;           // leaf regions: sorted features
+    std::vector<int32_t> partitions;     // sum regions: partitions feeding the sums
+    int32_t consumer_partition = -1;
+};
+
+struct Partition {
+    int32_t ra = -1, rb = -1;            // child regions (ra < rb)
+    std::vector<int64_t> prods;          // cell (i*nb + j) -> product node
+    int32_t consumer_region = -1;
+};
+
+}  // namespace
+
+void detect_layered(const GraphData &g, LayeredPlan &plan) {
+    plan = LayeredPlan();
+    CGraph c;
+    canonicalise(g, c);
+    auto fail = [&](const std::string &why) {
+        plan.ok = false;
+        plan.why = why;
+    };
+    auto fan = [&](int64_t u) { return c.cb[u + 1] - c.cb[u]; };
+    const int64_t n = c.n;
+    std::vector<int32_t> region_of(n, -1), index_in(n, -1);
+    std::vector<Region> regions;
+
+    // ---- leaf regions: Gaussian leaves / products of Gaussian leaves over
+    //      distinct variables, grouped by variable set
+    std::map<std::vector<int32_t>, int32_t> by_vars;
+    std::vector<int32_t> feats;
+    for (int64_t u = 0; u < n; ++u) {
+        feats.clear();
+        if (c.kind[u] == SPN_GAUSSIAN) {
+            // a Gaussian consumed by anything but products of leaves is a 1-var dist
+            bool in_leaf_product = c.pb[u + 1] > c.pb[u];
+            for (int64_t e = c.pb[u]; e < c.pb[u + 1]; ++e) {
+                const int64_t p = c.par[e];
+                bool all_g = c.kind[p] == SPN_PRODUCT;
+                for (int64_t f = c.cb[p]; all_g && f < c.cb[p + 1]; ++f)
+                    all_g = c.kind[c.ch[f]] == SPN_GAUSSIAN;
+                if (!all_g) in_leaf_product = false;
+            }
+            if (in_leaf_product) continue;  // part of a factorised distribution
+            feats.push_back(g.feature[c.orig[u]]);
+        } else if (c.kind[u] == SPN_PRODUCT) {
+            bool all_g = true;
+            for (int64_t e = c.cb[u]; e < c.cb[u + 1] && all_g; ++e) {
+                const int64_t ch = c.ch[e];
+                all_g = c.kind[ch] == SPN_GAUSSIAN;
+                if (all_g) feats.push_back(g.feature[c.orig[ch]]);
+            }
+            if (!all_g) continue;
+            std::sort(feats.begin(), feats.end());
+            if (std::adjacent_find(feats.begin(), feats.end()) != feats.end())
+                return fail("leaf product repeats a variable");
+        } else {
+            if (is_leafk(c.kind[u])) return fail("discrete leaves are not layered");
+            continue;
+        }
+        auto it = by_vars.find(feats);
+        int32_t r;
+        if (it == by_vars.end()) {
+            r = (int32_t)regions.size();
+            regions.emplace_back();
+            regions[r].leaf = true;
+            regions[r].vars = feats;
+            by_vars[feats] = r;
+        } else {
+            r = it->second;
+        }
+        region_of[u] = r;
+        index_in[u] = (int32_t)regions[r].nodes.size();
+        regions[r].nodes.push_back(u);
+    }
+    if (regions.empty()) return fail("no leaf regions");
+
+    // ---- sum regions: sums with identical child sets
+    std::unordered_map<uint64_t, std::vector<int32_t>> by_children;
+    std::vector<int64_t> kids;
+    std::vector<std::vector<int64_t>> region_kids;  // sorted child list per sum region
+    std::vector<int32_t> sum_region_ids;
+    for (int64_t u = 0; u < n; ++u) {
+        if (c.kind[u] != SPN_SUM) continue;
+        kids.assign(c.ch.begin() + c.cb[u], c.ch.begin() + c.cb[u + 1]);
+        std::sort(kids.begin(), kids.end());
+        if (std::adjacent_find(kids.begin(), kids.end()) != kids.end())
+            return fail("sum with a repeated child");
+        const uint64_t h = hash_vec(kids);
+        int32_t r = -1;
+        for (int32_t cand : by_children[h])
+            if (region_kids[cand] == kids) r = cand;
+        if (r < 0) {
+            r = (int32_t)region_kids.size();
+            region_kids.push_back(kids);
+            by_children[h].push_back(r);
+            sum_region_ids.push_back((int32_t)regions.size());
+            regions.emplace_back();
+        }
+        const int32_t rid = sum_region_ids[r];
+        region_of[u] = rid;
+        index_in[u] = (int32_t)regions[rid].nodes.size();
+        regions[rid].nodes.push_back(u);
+    }
+
+    // ---- partitions: products of two region values
+    std::map<std::pair<int32_t, int32_t>, int32_t> by_pair;
+    std::vector<Partition> parts;
+    std::vector<int32_t> part_of(n, -1);
+    std::vector<int32_t> cell_of(n, -1);
+    for (int64_t u = 0; u < n; ++u) {
+        if (c.kind[u] != SPN_PRODUCT || region_of[u] >= 0) continue;
+        if (fan(u) != 2) return fail("inner product without two region children");
+        int64_t a = c.ch[c.cb[u]], b = c.ch[c.cb[u] + 1];
+        if (region_of[a] < 0 || region_of[b] < 0) return fail("product child outside regions");
+        if (region_of[a] > region_of[b]) std::swap(a, b);
+        if (region_of[a] == region_of[b]) return fail("product of one region with itself");
+        const auto key = std::make_pair(region_of[a], region_of[b]);
+        auto it = by_pair.find(key);
+        int32_t p;
+        if (it == by_pair.end()) {
+            p = (int32_t)parts.size();
+            parts.emplace_back();
+            parts[p].ra = key.first;
+            parts[p].rb = key.second;
+            by_pair[key] = p;
+        } else {
+            p = it->second;
+        }
+        Partition &P = parts[p];
+        const int64_t na = (int64_t)regions[P.ra].nodes.size(), nb = (int64_t)regions[P.rb].nodes.size();
+        if (P.prods.empty()) P.prods.assign(na * nb, -1);
+        const int64_t cell = (int64_t)index_in[a] * nb + index_in[b];
+        if (P.prods[cell] >= 0) return fail("duplicate product in a partition");
+        P.prods[cell] = u;
+        part_of[u] = p;
+        cell_of[u] = (int32_t)cell;
+    }
+    for (auto &P : parts)
+        for (int64_t x : P.prods)
+            if (x < 0) return fail("partition is not a complete cross product");
+    // every region consumed by exactly one partition (except the root region)
+    for (int32_t p = 0; p < (int32_t)parts.size(); ++p) {
+        for (int32_t r : {parts[p].ra, parts[p].rb}) {
+            if (regions[r].consumer_partition >= 0 && regions[r].consumer_partition != p)
+                return fail("region consumed by two partitions");
+            regions[r].consumer_partition = p;
+        }
+    }
+    // region values consumed only by their partition's products
+    for (int32_t r = 0; r < (int32_t)regions.size(); ++r)
+        for (int64_t u : regions[r].nodes)
+            for (int64_t e = c.pb[u]; e < c.pb[u + 1]; ++e)
+                if (part_of[c.par[e]] != regions[r].consumer_partition)
+                    return fail("region value with a foreign consumer");
+    // sum regions: children = union of complete partitions
+    for (size_t k = 0; k < region_kids.size(); ++k) {
+        const int32_t rid = sum_region_ids[k];
+        std::vector<int32_t> ps;
+        for (int64_t ch : region_kids[k]) {
+            if (part_of[ch] < 0) return fail("sum child is not a partition product");
+            ps.push_back(part_of[ch]);
+        }
+        std::sort(ps.begin(), ps.end());
+        ps.erase(std::unique(ps.begin(), ps.end()), ps.end());
+        size_t total = 0;
+        for (int32_t p : ps) {
+            total += parts[p].prods.size();
+            if (parts[p].consumer_region >= 0) return fail("partition consumed by two regions");
+            parts[p].consumer_region = rid;
+        }
+        if (total != region_kids[k].size()) return fail("sum region covers a partial partition");
+        regions[rid].partitions = ps;
+    }
+    // the roots: exactly the sums of one region, each root once
+    const int32_t R0 = (int32_t)g.roots.size();
+    int32_t root_region = -1;
+    std::vector<int32_t> root_value(R0, -1);
+    for (int64_t u = 0; u < n; ++u) {
+        if (c.rootrefs[u].empty()) continue;
+        if (c.kind[u] != SPN_SUM || region_of[u] < 0) return fail("root is not a layered sum");
+        if (c.rootrefs[u].size() != 1) return fail("repeated root");
+        if (root_region >= 0 && region_of[u] != root_region) return fail("roots in several regions");
+        root_region = region_of[u];
+    }
+    if (root_region < 0) return fail("no root region");
+    if ((int32_t)regions[root_region].nodes.size() != R0) return fail("root region has non-root sums");
+    if (regions[root_region].consumer_partition >= 0) return fail("root region is consumed");
+    for (int32_t r = 0; r < (int32_t)regions.size(); ++r)
+        if (r != root_region && regions[r].consumer_partition < 0)
+            return fail("dangling region");
+    for (int32_t r = 0; r < (int32_t)regions.size(); ++r)
+        if (!regions[r].leaf && r != root_region && regions[r].partitions.size() != 1)
+            return fail("internal sum region with several partitions");
+    for (auto &reg : regions) {
+        if (reg.nodes.size() > 64) return fail("region with more than 64 values");
+        if (reg.leaf && reg.nodes.size() % 4) return fail("leaf region size must be a multiple of 4");
+        if (!reg.leaf && reg.nodes.size() < 1) return fail("empty region");
+    }
+    for (auto &P : parts) {
+        const size_t na = regions[P.ra].nodes.size(), nb = regions[P.rb].nodes.size();
+        if (na % 8 || nb > 64 || na > 56) return fail("region sizes need na % 8 == 0, <= 56");
+        (void)nb;
+    }
+
+    // ---- build the schedule (post-order over each repetition's region tree)
+    plan.F = g.F;
+    plan.C = R0;
+    plan.R = (int32_t)regions[root_region].partitions.size();
+    std::vector<int32_t> root_order(R0);  // root region value index -> root index
+    for (int64_t u : regions[root_region].nodes) root_order[index_in[u]] = c.rootrefs[u][0];
+    const int TILE = 128;
+    int32_t buf_top = 0, buf_peak = 0;
+    std::vector<double> cvals;
+    auto add_weights = [&](LStep &st, int32_t rid, int32_t p, bool root) {
+        const Partition &P = parts[p];
+        const int32_t na = (int32_t)regions[P.ra].nodes.size();
+        const int32_t nb = (int32_t)regions[P.rb].nodes.size();
+        const int32_t S = (int32_t)regions[rid].nodes.size();
+        st.na = na;
+        st.nb = nb;
+        st.n_out = S;
+        st.k_pad = (nb + 15) / 16 * 16;
+        st.s_per_group = std::max(1, std::min(S, 240 / na));
+        st.n_groups = (S + st.s_per_group - 1) / st.s_per_group;
+        st.n_group = (st.s_per_group * na + 15) / 16 * 16;
+        st.w_group_bytes = (int64_t)st.n_group * st.k_pad * 2;
+        // align the weight images to 16 bytes
+        while (plan.wimg.size() % 8) plan.wimg.push_back(0);
+        st.w_off = (int64_t)plan.wimg.size() * 2;
+        // weights W[s][i][j] for value s of region rid (root: value index of the root)
+        std::vector<double> W((size_t)S * na * nb, 0.0);
+        for (int64_t sn : regions[rid].nodes) {
+            const int32_t s = index_in[sn];
+            for (int64_t e = c.cb[sn]; e < c.cb[sn + 1]; ++e) {
+                const int64_t ch = c.ch[e];
+                if (part_of[ch] != p) continue;
+                const int32_t cell = cell_of[ch];
+                W[(size_t)s * na * nb + cell] = c.w[e];  // cell = i * nb + j
+            }
+        }
+        (void)root;
+        for (int32_t gi = 0; gi < st.n_groups; ++gi) {
+            std::vector<uint16_t> hi((size_t)st.n_group * st.k_pad, 0), lo(hi.size(), 0);
+            for (int32_t sl = 0; sl < st.s_per_group; ++sl) {
+                const int32_t s = gi * st.s_per_group + sl;
+                if (s >= S) break;
+                for (int32_t i = 0; i < na; ++i)
+                    for (int32_t j = 0; j < nb; ++j) {
+                        const int32_t row = sl * na + i;  // N index
+                        const double w = W[(size_t)s * na * nb + (size_t)i * nb + j];
+                        const uint16_t h = f32_to_f16((float)w);
+                        const uint16_t l = f32_to_f16((float)(w - (double)f16_to_f32(h)));
+                        // K-major no-swizzle core-matrix image: (k/8)*LBO + (row/8)*128 + (row%8)*16 + (k%8)*2
+                        const size_t lbo = (size_t)(st.n_group / 8) * 64;  // in f16 elements
+                        const size_t idx = (size_t)(j / 8) * lbo + (size_t)(row / 8) * 64 +
+                                           (size_t)(row % 8) * 8 + (size_t)(j % 8);
+                        hi[idx] = h;
+                        lo[idx] = l;
+                    }
+            }
+            plan.wimg.insert(plan.wimg.end(), hi.begin(), hi.end());
+            plan.wimg.insert(plan.wimg.end(), lo.begin(), lo.end());
+        }
+        plan.tc_flops_per_sample += 2LL * na * nb * S;
+        plan.fma_per_sample += (int64_t)S * na;
+        plan.mufu_per_sample += na + nb + S;
+    };
+    // Stack allocation of the activation buffers: a region's output is placed
+    // at the stack top it was started with.  A SUM step reads its inputs only
+    // in its first phase, so its output may overwrite them.
+    std::function<int32_t(int32_t)> visit = [&](int32_t rid) -> int32_t {
+        Region &reg = regions[rid];
+        const int32_t top0 = buf_top;
+        LStep st;
+        memset(&st, 0, sizeof(st));
+        if (reg.leaf) {
+            st.type = 0;
+            const int32_t I = (int32_t)reg.nodes.size();
+            const int32_t V = (int32_t)reg.vars.size();
+            st.n_out = I;
+            st.n_vars = V;
+            st.vars_off = (int64_t)plan.vars.size();
+            plan.vars.insert(plan.vars.end(), reg.vars.begin(), reg.vars.end());
+            // params [v][i'] float2 (a, b); i' = half * Ih + k for dist i = half * Ih + k
+            while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
+            st.par_off = (int64_t)plan.fparams.size();
+            const int32_t Ih = (I + 1) / 2;
+            std::vector<float> ab((size_t)V * 2 * Ih * 2, 0.f);
+            std::vector<float> cv((size_t)V * 2 * Ih, 0.f);
+            std::vector<double> Cs(I, 0.0);
+            for (int32_t i = 0; i < I; ++i) {
+                const int64_t u = reg.nodes[i];
+                std::vector<int64_t> leaves;
+                if (c.kind[u] == SPN_GAUSSIAN) leaves.push_back(u);
+                else leaves.assign(c.ch.begin() + c.cb[u], c.ch.begin() + c.cb[u + 1]);
+                for (int64_t lf : leaves) {
+                    const int64_t o = c.orig[lf];
+                    const int32_t f = g.feature[o];
+                    const int32_t v = (int32_t)(std::lower_bound(reg.vars.begin(), reg.vars.end(), f) -
+                                                reg.vars.begin());
+                    const double *pp = g.params.data() + g.param_begin[o];
+                    const double a = 1.0 / (pp[1] * std::sqrt(2.0 * M_LN2));
+                    const double cc = -std::log2(pp[1] * std::sqrt(2.0 * M_PI));
+                    Cs[i] += cc;
+                    cv[(size_t)v * 2 * Ih + i] = (float)cc;
+                    const size_t idx = ((size_t)v * 2 * Ih + (size_t)i) * 2;
+                    ab[idx] = (float)a;
+                    ab[idx + 1] = (float)(a * pp[0]);
+                }
+            }
+            plan.fparams.insert(plan.fparams.end(), ab.begin(), ab.end());
+            while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
+            st.cst_off = (int64_t)plan.fparams.size();
+            for (int32_t i = 0; i < 2 * Ih; ++i) plan.fparams.push_back(i < I ? (float)Cs[i] : 0.f);
+            st.w_off = (int64_t)plan.fparams.size();  // LEAF: per-(v,i) c (marginal)
+            plan.fparams.insert(plan.fparams.end(), cv.begin(), cv.end());
+            st.buf_out = top0;
+            buf_top = top0 + I * TILE;
+            buf_peak = std::max(buf_peak, buf_top);
+            plan.fma_per_sample += 2LL * I * V;
+            plan.n_leaf_regions++;
+            plan.steps.push_back(st);
+            return st.buf_out;
+        }
+        const Partition &P = parts[reg.partitions[0]];
+        st.buf_a = visit(P.ra);
+        st.buf_b = visit(P.rb);
+        st.type = 1;
+        add_weights(st, rid, reg.partitions[0], false);
+        st.buf_out = top0;
+        buf_top = top0 + st.n_out * TILE;
+        buf_peak = std::max(buf_peak, buf_top);
+        plan.n_sum_regions++;
+        plan.steps.push_back(st);
+        return st.buf_out;
+    };
+    for (int32_t p : regions[root_region].partitions) {
+        const Partition &P = parts[p];
+        const int32_t top0 = buf_top;
+        LStep st;
+        memset(&st, 0, sizeof(st));
+        st.buf_a = visit(P.ra);
+        st.buf_b = visit(P.rb);
+        st.type = 2;
+        add_weights(st, root_region, p, true);
+        st.buf_out = -1;
+        plan.steps.push_back(st);
+        buf_top = top0;
+    }
+    // root values must be emitted in root-index order: remap via root_order
+    plan.root_map = root_order;
+    plan.smem_floats = buf_peak;
+    for (auto &st : plan.steps) {
+        plan.max_kpad = std::max(plan.max_kpad, st.k_pad);
+        plan.max_ngroup = std::max(plan.max_ngroup, st.n_group);
+        plan.max_na = std::max(plan.max_na, st.na);
+    }
+    plan.ok = true;
+}
+
+}  // namespace spnb

@@ -1,0 +1,65 @@
+// layered.h -- detection of layered (RAT-SPN-style) region-graph structure
+// in a flat SPN DAG and the plan of the tensor-core path (kernel KB/KC).
+//
+// A layered SPN (§V-B: RAT-SPNs, "random tensorized"
+// region graphs) consists of
+//   * leaf regions: I "distributions", each a product of Gaussian leaves over
+//     the region's variable set (or a single Gaussian leaf);
+//   * partitions: the cross product of two child regions' values (product
+//     nodes with exactly two children, one per child region);
+//   * sum regions: S weighted sums over all products of one partition;
+//   * the root region: the graph roots, C sums over the products of one or
+//     more partitions (one per repetition).
+// Every region feeds exactly one partition (a tree of regions per
+// repetition).  The preparer recognises this structure from the DAG alone.
+#pragma once
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "prepare.h"
+
+namespace spnb {
+
+// One step of the per-tile schedule (see rat_eval.cu).
+struct LStep {
+    int32_t type;        // 0 LEAF, 1 SUM, 2 ROOT
+    int32_t n_out;       // values produced (I, S or C)
+    int32_t na, nb;      // child region sizes (SUM / ROOT)
+    int32_t buf_a, buf_b, buf_out;  // shared-memory buffer offsets (floats)
+    int32_t k_pad;       // nb rounded up to 16 (f16 K-step)
+    int32_t s_per_group; // sums per N-group
+    int32_t n_groups;
+    int32_t n_group;     // N columns per group (multiple of 16)
+    int32_t n_vars;      // LEAF: variables of the region
+    int64_t vars_off;    // LEAF: int32 offset into vars[]
+    int64_t par_off;     // LEAF: float2 (a, b) [n_vars][n_out]; C at cst_off
+    int64_t cst_off;     // LEAF: float C[n_out]
+    int64_t w_off;       // SUM/ROOT: byte offset of the f16 weight images
+    int64_t w_group_bytes;  // bytes per (group, part) image
+    int32_t rep;         // repetition (ROOT)
+    int32_t pad_;
+};
+
+struct LayeredPlan {
+    bool ok = false;
+    std::string why;             // reason when not layered
+    int32_t F = 0, C = 0, R = 0; // features, classes (roots), repetitions
+    std::vector<LStep> steps;
+    std::vector<int32_t> vars;
+    std::vector<float> fparams;  // leaf (a,b) pairs and C constants
+    std::vector<uint16_t> wimg;  // f16 weight images (hi then lo per group)
+    int32_t smem_floats = 0;     // activation buffers
+    int32_t max_kpad = 0, max_ngroup = 0, max_na = 0;
+    std::vector<int32_t> root_map;  // root-region value index -> output column
+    int64_t tc_flops_per_sample = 0;  // one precision pass
+    int64_t fma_per_sample = 0;
+    int64_t mufu_per_sample = 0;
+    int64_t n_leaf_regions = 0, n_sum_regions = 0;
+};
+
+// Detects the structure; on success fills plan (ok = true).
+void detect_layered(const GraphData &g, LayeredPlan &plan);
+
+}  // namespace spnb

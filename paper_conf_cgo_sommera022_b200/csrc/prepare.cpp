@@ -157,19 +157,7 @@ int validate_graph(const GraphData &g, std::string &msg) {
 // ---------------------------------------------------------------------------
 namespace {
 
-// Canonical DAG: reachable nodes in post-order (children first), single-input
-// nodes removed where exact (products always; sums only if the weight is 1).
-struct CGraph {
-    int64_t n = 0;
-    std::vector<int32_t> kind;
-    std::vector<int64_t> orig;          // original node id
-    std::vector<int64_t> cb;            // CSR children
-    std::vector<int64_t> ch;
-    std::vector<double> w;
-    std::vector<int64_t> pb;            // CSR parents
-    std::vector<int64_t> par;
-    std::vector<std::vector<int32_t>> rootrefs;
-};
+}  // namespace
 
 void canonicalise(const GraphData &g, CGraph &c) {
     const int64_t n = (int64_t)g.kind.size();
@@ -248,6 +236,8 @@ void canonicalise(const GraphData &g, CGraph &c) {
     c.rootrefs.assign(c.n, {});
     for (size_t r = 0; r < g.roots.size(); ++r) c.rootrefs[newid[rep[g.roots[r]]]].push_back((int32_t)r);
 }
+
+namespace {
 
 // LoSPN-operation size of an inner node (binary mul/add after lowering,
 // weighted sums become n muls + n-1 adds); leaf uses count 1.
@@ -516,10 +506,30 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
         if (is_leaf(c.kind[ch]) || mat[ch]) return 1;
         return need[ch];
     };
+    // fused sum of Gaussian leaf products (SLPk): 2..4 children, each a
+    // Gaussian leaf or an unshared product of 1..7 Gaussian leaves
+    auto gprod_leaves = [&](int64_t ch) -> int {
+        if (c.kind[ch] == SPN_GAUSSIAN) return 1;
+        if (c.kind[ch] != SPN_PRODUCT || mat[ch] || virt[ch]) return 0;
+        int cnt = 0;
+        for (int64_t e = c.cb[ch]; e < c.cb[ch + 1]; ++e) {
+            if (c.kind[c.ch[e]] != SPN_GAUSSIAN) return 0;
+            ++cnt;
+        }
+        return cnt <= 7 ? cnt : 0;
+    };
+    auto slp_ok = [&](int64_t u) -> bool {
+        if (c.kind[u] != SPN_SUM || glse[u]) return false;
+        const int64_t n = fan(u);
+        if (n < 2 || n > 4) return false;
+        for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e)
+            if (!gprod_leaves(c.ch[e])) return false;
+        return true;
+    };
     auto compute_need = [&](int64_t u) -> int32_t {
         const int32_t k = c.kind[u];
         if (is_leaf(k) || virt[u]) return 1;
-        if (k == SPN_SUM && glse[u]) return 1;
+        if (k == SPN_SUM && (glse[u] || slp_ok(u))) return 1;
         std::vector<int32_t> nv;
         int nleaf = 0;
         for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) {
@@ -687,6 +697,26 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             rec_of(OP_GLSE, sp, 0, (uint32_t)(off & 0xffffffffu), (uint32_t)(off >> 32), (uint32_t)n);
             return;
         }
+        if (slp_ok(u)) {
+            uint32_t counts = 0, Cb[4] = {0, 0, 0, 0};
+            std::vector<int64_t> lv;
+            for (int64_t e = c.cb[u], ci = 0; e < c.cb[u + 1]; ++e, ++ci) {
+                const int64_t ch = c.ch[e];
+                std::vector<int64_t> cl;
+                if (c.kind[ch] == SPN_GAUSSIAN) cl.push_back(ch);
+                else cl.assign(c.ch.begin() + c.cb[ch], c.ch.begin() + c.cb[ch + 1]);
+                double C = lw2(c.w[e]);
+                for (int64_t l : cl) C += leaf[l].c;
+                Cb[ci] = fbits((float)C);
+                counts |= (uint32_t)cl.size() << (3 * ci);
+                lv.insert(lv.end(), cl.begin(), cl.end());
+            }
+            max_sp = std::max<int64_t>(max_sp, sp + 1);
+            rec_of(OP_SLP2 + (uint32_t)(n - 2), sp, counts, fbits((float)bias), Cb[0], Cb[1]);
+            if (n >= 3) prog.push_back(Rec{Cb[2], Cb[3], 0, 0});
+            for (int64_t l : lv) prog.push_back(Rec{feat_arg(leaf[l].f), leaf[l].y, leaf[l].z, leaf[l].w});
+            return;
+        }
         std::vector<std::pair<int32_t, int64_t>> kids;  // (need, edge)
         for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) kids.push_back({child_need(c.ch[e]), e});
         std::stable_sort(kids.begin(), kids.end(),
@@ -758,6 +788,11 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             i += cs / NSP - OP_GPUSH1 + 1;
         else if (cs / NSP >= OP_GACC1 && cs / NSP <= OP_GACC4)
             i += cs / NSP - OP_GACC1 + 1;
+        else if (cs / NSP >= OP_SLP2 && cs / NSP <= OP_SLP4 && cs < OP_COUNT * NSP) {
+            const uint32_t cnt = prog[i].x >> CASE_BITS;
+            i += (cs / NSP >= OP_SLP3 ? 1 : 0) + (cnt & 7u) + ((cnt >> 3) & 7u) +
+                 ((cnt >> 6) & 7u) + ((cnt >> 9) & 7u);
+        }
     }
     for (const Fix &f : fixes) {
         if (f.kind == 0) last_use[f.node] = std::max(last_use[f.node], f.idx);

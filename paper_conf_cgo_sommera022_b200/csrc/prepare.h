@@ -43,6 +43,21 @@ struct PlanProgram {
     int64_t n_roots = 0;
 };
 
+// Canonical DAG: reachable nodes in post-order (children first), single-input
+// nodes removed where exact (products always; sums only if the weight is 1).
+struct CGraph {
+    int64_t n = 0;
+    std::vector<int32_t> kind;
+    std::vector<int64_t> orig;          // original node id
+    std::vector<int64_t> cb;            // CSR children
+    std::vector<int64_t> ch;
+    std::vector<double> w;
+    std::vector<int64_t> pb;            // CSR parents
+    std::vector<int64_t> par;
+    std::vector<std::vector<int32_t>> rootrefs;
+};
+void canonicalise(const GraphData &g, CGraph &c);
+
 // Returns 0 or a negative spn_status with msg set.
 int validate_graph(const GraphData &g, std::string &msg);
 

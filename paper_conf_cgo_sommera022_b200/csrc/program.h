@@ -16,6 +16,9 @@
 //   LPUSH  ng | C, nd        r[sp]   = C + sum of ng Gaussian + nd discrete leaves
 //   LACC   ng | C, nd        r[sp-1] += (same)          (leaf children of a product)
 //   GPUSHn / GACCn  | C      same for exactly n <= 4 Gaussian leaves (no loop)
+//   SLPk  counts | bias, C0, C1   r[sp] = LSE_c(C_c + sum of n_c Gaussian leaves) + bias
+//       for k = 2..4 children (n_c in 1..7 packed 3 bits each in arg); for k >= 3
+//       a record {C2, C3} follows, then the children's parameter records.
 //       followed by ng Gaussian parameter records {f, a, b, c} and nd discrete
 //       records {f, table, lo, K}.  Gaussian: c - (a*x_f - b)^2 = log2 N(x; mu, s)
 //       with a = 1/(s sqrt(2 ln2)), b = a mu, c = -log2(s sqrt(2 pi)); the c's
@@ -60,7 +63,10 @@ enum Op : uint32_t {
     OP_GACC2 = 20,
     OP_GACC3 = 21,
     OP_GACC4 = 22,
-    OP_COUNT = 23
+    OP_SLP2 = 23,   // fused weighted sum of 2..4 Gaussian leaf products
+    OP_SLP3 = 24,
+    OP_SLP4 = 25,
+    OP_COUNT = 26
 };
 
 constexpr int MAXD = 16;              // register stack depth

@@ -14,7 +14,8 @@ import numpy as np
 NSP = 17
 OPS = ["END", "LPUSH", "LACC", "ADD", "LSE1", "LSE2", "LSE3", "LSE4",
        "LDS", "LDG", "STS", "STG", "GLSE", "OUT", "NOP",
-       "GPUSH1", "GPUSH2", "GPUSH3", "GPUSH4", "GACC1", "GACC2", "GACC3", "GACC4"]
+       "GPUSH1", "GPUSH2", "GPUSH3", "GPUSH4", "GACC1", "GACC2", "GACC3", "GACC4",
+       "SLP2", "SLP3", "SLP4"]
 SLOT_GLOBAL = 0x80000000
 SLOT_NONE = 0xFFFFFFFF
 
@@ -67,6 +68,25 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
             op, sp = OPS[case // NSP] if case // NSP < len(OPS) else "BAD", case % NSP
             if op == "END":
                 break
+            if op.startswith("SLP"):
+                k = int(op[3])
+                Cs = [_f32(r["z"]), _f32(r["w"])]
+                if k >= 3:
+                    Cs += [_f32(rec[pc]["x"]), _f32(rec[pc]["y"])]
+                    pc += 1
+                vals = []
+                for ci in range(k):
+                    acc = np.full(N, Cs[ci])
+                    for _ in range((arg >> (3 * ci)) & 7):
+                        q = rec[pc]
+                        pc += 1
+                        xv = xd[:, feat(int(q["x"]))]
+                        a, b, c = _f32(q["y"]), _f32(q["z"]), _f32(q["w"])
+                        t = a * xv - b
+                        acc = acc - (np.where(np.isnan(xv), c, t * t) if marginal else t * t)
+                    vals.append(acc)
+                stack[sp] = _lse(vals) + _f32(r["y"])
+                continue
             if op[:5] in ("GPUSH", "GACC1", "GACC2", "GACC3", "GACC4"):
                 ng, nd = int(op[-1]), 0
                 op = "LPUSH" if op.startswith("GPUSH") else "LACC"

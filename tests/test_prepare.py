@@ -207,8 +207,9 @@ def test_codegen_rat_uses_gather_terms():
 
 
 def test_codegen_deep_balanced_tree_forces_materialisation():
-    """A balanced 4-ary sum tree of depth 6 needs 1 + 3*6 = 19 stack entries
-    (Sethi-Ullman), more than the 16-deep register stack: the preparer must
+    """A balanced 4-ary sum tree of depth 7 needs 1 + 3*6 = 19 stack entries
+    (Sethi-Ullman; the bottom level is one fused SLP4 record), more than the
+    16-deep register stack: the preparer must
     split it through slots."""
     b = GraphBuilder(4)
     rng = np.random.default_rng(0)
@@ -218,7 +219,7 @@ def test_codegen_deep_balanced_tree_forces_materialisation():
             return b.gaussian(int(rng.integers(0, 4)), float(rng.normal()), 1.0)
         return b.sum([deep(d - 1) for _ in range(4)], [0.25] * 4)
 
-    g = b.build([deep(6)])
+    g = b.build([deep(7)])
     x = rng.normal(size=(64, 4)).astype(np.float32)
     p = _check_program(g, x, False)
     assert p["n_sslots"] + p["n_gslots"] > 0 and p["max_stack"] <= 16

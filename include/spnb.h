@@ -72,10 +72,13 @@ typedef struct spn_prepare_options {
     int32_t device;             /* CUDA device ordinal; -1 = current device    */
     int32_t block_threads;      /* threads per CTA, multiple of 32; 0 = auto   */
     int32_t samples_per_thread; /* K in {1,2,4}; 0 = auto                      */
-    int32_t layered_path;       /* 0 auto, 1 off (generic only), 2 force       */
+    int32_t layered_path;       /* 0 auto, 1 off (generic only), 2 force the
+                                   tensor-core RAT-SPN path (E_UNSUPPORTED if
+                                   the DAG is not a layered region graph)    */
     int64_t max_task_nodes;     /* partition cap in LoSPN ops;
                                    0 = auto (shared-memory budget), -1 = none  */
-    int32_t tc_precision;       /* layered path: 0 tf32, 1 3xtf32, 2 f16       */
+    int32_t tc_precision;       /* layered path: 0 auto (= 2), 1 f16 single
+                                   pass, 2 f16 hi/lo split (3 MMAs, ~fp32)    */
     int32_t ctas_per_sm;        /* 0 = auto                                    */
     int32_t reserved[8];        /* must be zero                                */
 } spn_prepare_options;
@@ -198,6 +201,18 @@ int spn_plan_info(const spn_handle *plan, spn_plan_stats *stats);
  *   number of shared-memory slots, slots[1] global slots, slots[2] the max
  *   stack depth.
  */
+/*
+ * spn_build_layered: run the layered (RAT-SPN region graph) detector and
+ *   plan builder of the tensor-core path without a GPU.  Returns SPN_OK and
+ *   *is_layered = 0/1 (why[why_len] receives the reason when 0).  With NULL
+ *   buffers only the sizes are returned: sizes[0] steps (each
+ *   sizeof_step bytes), sizes[1] vars (int32), sizes[2] fparams (float),
+ *   sizes[3] weight-image bytes, sizes[4] roots, sizes[5] activation floats,
+ *   sizes[6] sizeof_step.  Then call again with buffers of those sizes.
+ */
+int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, int64_t why_len,
+                      int64_t *sizes, void *steps, int32_t *vars, float *fparams, void *wimg,
+                      int32_t *root_map);
 int spn_partition_graph(const spn_handle *graph, int64_t max_task_ops, int32_t *task_of_node,
                         int32_t *n_tasks, int64_t *cost, int64_t *cut_values);
 int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32_t x_in_smem,

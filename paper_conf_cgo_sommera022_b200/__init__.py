@@ -22,7 +22,7 @@ import numpy as np
 from .build import LIB as _LIB_PATH
 
 __all__ = ["SPNError", "Graph", "Plan", "load_library", "partition_graph",
-           "build_program", "NODE_DTYPE", "REC_DTYPE", "EDGE_DTYPE",
+           "build_program", "build_layered", "LSTEP_DTYPE", "NODE_DTYPE", "REC_DTYPE", "EDGE_DTYPE",
            "GAUSSIAN", "CATEGORICAL", "HISTOGRAM", "SUM", "PRODUCT"]
 
 GAUSSIAN, CATEGORICAL, HISTOGRAM, SUM, PRODUCT = 0, 1, 2, 3, 4
@@ -32,6 +32,12 @@ NODE_DTYPE = np.dtype([("kind", "<i4"), ("feature", "<i4"), ("child_begin", "<i8
 assert NODE_DTYPE.itemsize == 32
 REC_DTYPE = np.dtype([("x", "<u4"), ("y", "<u4"), ("z", "<u4"), ("w", "<u4")])
 EDGE_DTYPE = np.dtype([("a", "<u4"), ("b", "<u4"), ("lw", "<f4"), ("pad", "<u4")])
+LSTEP_DTYPE = np.dtype([(n, "<i4") for n in ("type", "n_out", "na", "nb", "buf_a", "buf_b",
+                                             "buf_out", "k_pad", "s_per_group", "n_groups",
+                                             "n_group", "n_vars")] +
+                       [(n, "<i8") for n in ("vars_off", "par_off", "cst_off", "w_off",
+                                             "w_group_bytes")] +
+                       [("rep", "<i4"), ("pad_", "<i4")])
 
 _STATUS = {0: "SPN_OK", -1: "SPN_E_ARG", -2: "SPN_E_GRAPH", -3: "SPN_E_CUDA",
            -4: "SPN_E_OOM", -5: "SPN_E_UNSUPPORTED"}
@@ -87,9 +93,10 @@ def load_library(path: str | None = None):
     lib.spn_free.restype = None
     lib.spn_partition_graph.argtypes = [P, I64, P, P, P, P]
     lib.spn_build_program.argtypes = [P, I32, I32, I64, I64, P, P, P, P, P, P, P, P, P]
+    lib.spn_build_layered.argtypes = [P, P, P, I64, P, P, P, P, P, P]
     for name in ("spn_load_graph", "spn_prepare", "spn_infer_joint", "spn_infer_marginal",
                  "spn_infer_joint_host", "spn_infer_marginal_host", "spn_plan_info",
-                 "spn_partition_graph", "spn_build_program"):
+                 "spn_partition_graph", "spn_build_program", "spn_build_layered"):
         getattr(lib, name).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -272,3 +279,26 @@ def build_program(graph: Graph, samples_per_thread: int = 4, x_in_smem: bool = T
                                  ctypes.byref(ne), _ptr(slots)))
     return {"records": rec, "task_off": toff, "tables": tab, "edges": edg,
             "n_sslots": int(slots[0]), "n_gslots": int(slots[1]), "max_stack": int(slots[2])}
+
+
+def build_layered(graph: Graph):
+    """Host-only: the layered (RAT-SPN) tensor-core plan (``spn_build_layered``).
+    Returns None (and the reason) if the DAG is not a layered region graph."""
+    lib = load_library()
+    ok = ctypes.c_int32()
+    why = ctypes.create_string_buffer(256)
+    sizes = np.zeros(7, dtype=np.int64)
+    _check(lib.spn_build_layered(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                 None, None, None, None, None))
+    if not ok.value:
+        return None, why.value.decode()
+    assert sizes[6] == LSTEP_DTYPE.itemsize, (sizes[6], LSTEP_DTYPE.itemsize)
+    steps = np.zeros(sizes[0], dtype=LSTEP_DTYPE)
+    vars_ = np.zeros(sizes[1], dtype=np.int32)
+    fp = np.zeros(sizes[2], dtype=np.float32)
+    w = np.zeros(sizes[3] // 2, dtype=np.float16)
+    rm = np.zeros(sizes[4], dtype=np.int32)
+    _check(lib.spn_build_layered(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                 _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w), _ptr(rm)))
+    return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
+            "smem_floats": int(sizes[5])}, ""

@@ -13,6 +13,7 @@
 #include <string>
 #include <vector>
 
+#include "layered.h"
 #include "prepare.h"
 #include "program.h"
 #include "spnb.h"
@@ -24,6 +25,26 @@ cudaError_t dag_eval_launch_k4(const KParams &, bool, bool, int, int, size_t, cu
 int dag_eval_occupancy_k1(bool, bool, int, size_t);
 int dag_eval_occupancy_k2(bool, bool, int, size_t);
 int dag_eval_occupancy_k4(bool, bool, int, size_t);
+struct RParams {
+    const LStep *steps;
+    int32_t n_steps;
+    int32_t C;
+    const int32_t *vars;
+    const float *fparams;
+    const uint8_t *wimg;
+    const int32_t *root_map;
+    const float *xT;
+    int64_t ldT;
+    int64_t n;
+    float *out;
+    int32_t *argmax;
+    int32_t prec;
+    int32_t smem_floats, max_kpad, max_ngroup, max_na;
+};
+size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup);
+cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
+cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
+                             int64_t rows_pad, cudaStream_t st);
 }  // namespace spnb
 
 using namespace spnb;
@@ -68,6 +89,18 @@ struct DevicePlan {
     float *hout[2] = {nullptr, nullptr};
     int32_t *ham[2] = {nullptr, nullptr};
     int64_t host_chunk = 0;
+    // layered (RAT-SPN) path
+    int path = 0;
+    LStep *d_steps = nullptr;
+    int32_t n_steps = 0;
+    int32_t *d_vars = nullptr;
+    float *d_fparams = nullptr;
+    uint8_t *d_wimg = nullptr;
+    int32_t *d_root_map = nullptr;
+    float *d_xT = nullptr;
+    int64_t chunk = 0;
+    int32_t prec = 3;
+    int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
     spn_plan_stats stats;
 };
 
@@ -113,6 +146,12 @@ void free_plan(DevicePlan *p) {
     cudaFree(p->d_tables);
     cudaFree(p->d_edges);
     cudaFree(p->d_gslots);
+    cudaFree(p->d_steps);
+    cudaFree(p->d_vars);
+    cudaFree(p->d_fparams);
+    cudaFree(p->d_wimg);
+    cudaFree(p->d_root_map);
+    cudaFree(p->d_xT);
     for (int i = 0; i < 2; ++i) {
         if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
         cudaFree(p->hx[i]);
@@ -158,6 +197,38 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
     if (!x || !out) return set_err(SPN_E_ARG, "null x/out");
     if (ld < P.F) return set_err(SPN_E_ARG, "ld < n_features");
     DeviceGuard dg(P.device);
+    if (P.path == 1) {
+        RParams rp;
+        memset(&rp, 0, sizeof(rp));
+        rp.steps = P.d_steps;
+        rp.n_steps = P.n_steps;
+        rp.C = P.R;
+        rp.vars = P.d_vars;
+        rp.fparams = P.d_fparams;
+        rp.wimg = P.d_wimg;
+        rp.root_map = P.d_root_map;
+        rp.xT = P.d_xT;
+        rp.ldT = P.chunk;
+        rp.prec = P.prec;
+        rp.smem_floats = P.smem_floats;
+        rp.max_kpad = P.max_kpad;
+        rp.max_ngroup = P.max_ngroup;
+        rp.max_na = P.max_na;
+        for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
+            const int64_t m = std::min(P.chunk, n - c0);
+            const int64_t rows_pad = (m + 127) / 128 * 128;
+            cudaError_t e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
+                                             (cudaStream_t)stream);
+            if (e != cudaSuccess) return cuda_err(e, "transpose launch");
+            rp.n = m;
+            rp.out = out + c0 * P.R;
+            rp.argmax = argmax ? argmax + c0 : nullptr;
+            const int grid = (int)std::min<int64_t>((m + 127) / 128, P.grid_max);
+            e = rat_launch(rp, marg, grid, P.smem, (cudaStream_t)stream);
+            if (e != cudaSuccess) return cuda_err(e, "rat_eval launch");
+        }
+        return SPN_OK;
+    }
     KParams kp;
     memset(&kp, 0, sizeof(kp));
     kp.prog = P.d_prog;
@@ -242,6 +313,82 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
 
 bool valid_graph_handle(const spn_handle *h) { return h && h->magic == H_GRAPH && h->graph; }
 
+int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare_options &opt,
+                    int dev, int sms, size_t smem, std::chrono::steady_clock::time_point t0,
+                    spn_handle **out_plan) {
+    DevicePlan *P = new (std::nothrow) DevicePlan();
+    if (!P) return set_err(SPN_E_OOM, "plan");
+    P->device = dev;
+    P->path = 1;
+    P->F = g.F;
+    P->R = lp.C;
+    P->sms = sms;
+    P->smem = smem;
+    P->grid_max = sms;
+    P->block = 256;
+    P->n_steps = (int32_t)lp.steps.size();
+    P->prec = opt.tc_precision == 1 ? 1 : 3;
+    P->smem_floats = lp.smem_floats;
+    P->max_kpad = lp.max_kpad;
+    P->max_ngroup = lp.max_ngroup;
+    P->max_na = lp.max_na;
+    // transposed-feature scratch: chunks of up to 64k samples (or ~256 MB)
+    int64_t chunk = 65536;
+    while (chunk > 1024 && (int64_t)g.F * chunk * 4 > ((int64_t)256 << 20)) chunk /= 2;
+    P->chunk = chunk;
+    int rc;
+    std::vector<uint8_t> w8(lp.wimg.size() * 2);
+    if (!w8.empty()) memcpy(w8.data(), lp.wimg.data(), w8.size());
+    if ((rc = upload(&P->d_steps, lp.steps)) || (rc = upload(&P->d_vars, lp.vars)) ||
+        (rc = upload(&P->d_fparams, lp.fparams)) || (rc = upload(&P->d_wimg, w8)) ||
+        (rc = upload(&P->d_root_map, lp.root_map))) {
+        free_plan(P);
+        return rc;
+    }
+    cudaError_t e = cudaMalloc(&P->d_xT, (size_t)g.F * chunk * 4);
+    if (e != cudaSuccess) {
+        free_plan(P);
+        return set_err(SPN_E_OOM, "transposed feature scratch");
+    }
+    spn_plan_stats &s = P->stats;
+    memset(&s, 0, sizeof(s));
+    CGraph c;
+    canonicalise(g, c);
+    s.n_nodes = c.n;
+    for (int64_t u = 0; u < c.n; ++u) {
+        if (c.kind[u] == SPN_SUM) {
+            s.n_sums++;
+            s.n_sum_edges += c.cb[u + 1] - c.cb[u];
+            s.mufu_per_sample += c.cb[u + 1] - c.cb[u] + 1;
+        } else if (c.kind[u] == SPN_PRODUCT) {
+            s.n_products++;
+        } else {
+            s.n_leaves++;
+        }
+    }
+    s.n_tasks = (int64_t)lp.steps.size();
+    s.fma_per_sample = lp.fma_per_sample;
+    s.tc_flops_per_sample = lp.tc_flops_per_sample * (P->prec == 3 ? 3 : 1);
+    s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)lp.C + 4;
+    s.path = 1;
+    s.block_threads = 256;
+    s.samples_per_thread = 0;
+    s.grid = P->grid_max;
+    s.smem_bytes = (int32_t)smem;
+    s.x_in_smem = 0;
+    s.prepare_ms =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    spn_handle *h = new (std::nothrow) spn_handle();
+    if (!h) {
+        free_plan(P);
+        return set_err(SPN_E_OOM, "handle");
+    }
+    h->magic = H_PLAN;
+    h->plan = P;
+    *out_plan = h;
+    return SPN_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -318,7 +465,6 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     if (opt_in) opt = *opt_in;
     for (int i = 0; i < 8; ++i)
         if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
-    if (opt.layered_path == 2) return set_err(SPN_E_UNSUPPORTED, "layered path not available for this graph");
     const auto t0 = std::chrono::steady_clock::now();
     const GraphData &g = *graph->graph;
 
@@ -331,6 +477,22 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         return cuda_err(e, "device attributes");
     cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
 
+    // ---- layered (RAT-SPN) tensor-core path ----
+    if (opt.layered_path != 1) {
+        LayeredPlan lp;
+        detect_layered(g, lp);
+        size_t lsmem = 0;
+        if (lp.ok) {
+            lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup);
+            if (lsmem > (size_t)smem_optin) {
+                lp.ok = false;
+                lp.why = "activations do not fit in shared memory";
+            }
+        }
+        if (!lp.ok && opt.layered_path == 2)
+            return set_err(SPN_E_UNSUPPORTED, "layered path not applicable: " + lp.why);
+        if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, t0, out_plan);
+    }
     int K = opt.samples_per_thread ? opt.samples_per_thread : 4;
     if (K != 1 && K != 2 && K != 4) return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2 or 4");
     const int max_block = K == 4 ? 384 : 512;
@@ -546,6 +708,32 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
         slots[1] = prog.n_gslots;
         slots[2] = prog.max_stack;
     }
+    return SPN_OK;
+}
+
+int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, int64_t why_len,
+                      int64_t *sizes, void *steps, int32_t *vars, float *fparams, void *wimg,
+                      int32_t *root_map) {
+    if (!valid_graph_handle(graph) || !is_layered || !sizes) return set_err(SPN_E_ARG, "bad arguments");
+    LayeredPlan lp;
+    detect_layered(*graph->graph, lp);
+    *is_layered = lp.ok ? 1 : 0;
+    if (why && why_len > 0) {
+        strncpy(why, lp.why.c_str(), (size_t)why_len - 1);
+        why[why_len - 1] = 0;
+    }
+    sizes[0] = (int64_t)lp.steps.size();
+    sizes[1] = (int64_t)lp.vars.size();
+    sizes[2] = (int64_t)lp.fparams.size();
+    sizes[3] = (int64_t)lp.wimg.size() * 2;
+    sizes[4] = (int64_t)lp.root_map.size();
+    sizes[5] = lp.smem_floats;
+    sizes[6] = (int64_t)sizeof(LStep);
+    if (steps) memcpy(steps, lp.steps.data(), lp.steps.size() * sizeof(LStep));
+    if (vars) memcpy(vars, lp.vars.data(), lp.vars.size() * 4);
+    if (fparams) memcpy(fparams, lp.fparams.data(), lp.fparams.size() * 4);
+    if (wimg) memcpy(wimg, lp.wimg.data(), lp.wimg.size() * 2);
+    if (root_map) memcpy(root_map, lp.root_map.data(), lp.root_map.size() * 4);
     return SPN_OK;
 }
 

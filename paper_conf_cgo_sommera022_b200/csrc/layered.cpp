@@ -281,7 +281,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
     }
     for (auto &P : parts) {
         const size_t na = regions[P.ra].nodes.size(), nb = regions[P.rb].nodes.size();
-        if (na % 8 || nb > 64 || na > 56) return fail("region sizes need na % 8 == 0, <= 56");
+        if (na % 4 || nb > 64 || na > 60) return fail("region sizes need na % 4 == 0, <= 60");
         (void)nb;
     }
 

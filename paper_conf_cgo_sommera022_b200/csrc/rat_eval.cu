@@ -1,0 +1,428 @@
+// rat_eval.cu -- layered RAT-SPN path for sm_100a (kernels KB + KC).
+//
+// For layered SPNs (RAT-SPNs, §V-B) the preparer
+// (layered.cpp) turns the DAG into a per-repetition schedule of region steps.
+// One persistent CTA owns a tile of 128 samples and walks the schedule:
+//
+//  LEAF (KB, FP32 pipe): L[i][m] = C_i - sum_v (a_iv x_mv - b_iv)^2, the log2
+//       density of each of the region's I factorised Gaussians; the features
+//       come from a transposed copy xT[F][N] (the LoSPN `transposed` batch
+//       access, L204-227) so a region's variables are coalesced rows.
+//  SUM  (KC, tensor cores): for a partition of regions A (na values a_i) and
+//       B (nb values b_j) and S sums with linear weights W[s][i][j]:
+//         out_s = ha + hb + log2 sum_{i,j} W[s,i,j] 2^(a_i-ha) 2^(b_j-hb)
+//       (exp distributes over the product node, so the max-shifted sum over
+//       the na*nb products factorises).  Stage 1 on tcgen05:
+//         T[m, (s,i)] = sum_j eb[m,j] W[s,i,j]   (M=128, K=nb, N=S*na groups)
+//       with A = eb (f16, K-major in shared memory), B = the prepared weight
+//       image, D accumulated in TMEM; stage 2 per sample on FP32:
+//         out_s = ha + hb + lg2(sum_i ea[m,i] T[m,(s,i)])   (tcgen05.ld).
+//       Precision: f16 operands, optionally split hi+lo (3 MMAs:
+//       hi*hi + lo*hi + hi*lo, ~2^-22 relative) -- spn_prepare_options.tc_precision.
+//  ROOT: the same contraction for the root region's partition of each
+//       repetition, accumulated over repetitions by an online log-sum-exp;
+//       the C class log-likelihoods and their argmax are written at the end.
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <stdint.h>
+
+#include "layered.h"
+
+namespace spnb {
+
+struct RParams {
+    const LStep *steps;
+    int32_t n_steps;
+    int32_t C;
+    const int32_t *vars;
+    const float *fparams;
+    const uint8_t *wimg;
+    const int32_t *root_map;
+    const float *xT;
+    int64_t ldT;
+    int64_t n;
+    float *out;
+    int32_t *argmax;
+    int32_t prec;       // 1: single f16 pass; 3: hi/lo split
+    int32_t smem_floats, max_kpad, max_ngroup, max_na;
+};
+
+constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
+constexpr int RTH = 256;  // threads per CTA
+constexpr uint32_t TMEM_COLS = 256;
+
+__device__ __forceinline__ float r_ex2(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float r_lg2(float x) {
+    float y;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float r_maxnan(float a, float b) {
+    float r;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+// log2(2^a + 2^b), NaN-propagating, -inf safe
+__device__ __forceinline__ float r_lse2(float a, float b) {
+    const float hi = r_maxnan(a, b), lo = fminf(a, b);
+    return hi + r_lg2(1.f + r_ex2(lo - fmaxf(hi, -1e30f)));
+}
+
+__device__ __forceinline__ uint32_t r_smem(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// UMMA shared-memory descriptor, K-major, no swizzle (canonical layout
+// ((8,m),(T,2)):((16B,SBO),(1,LBO)); version 1 for sm_100).
+__device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    uint64_t d = 0;
+    d |= (uint64_t)((addr >> 4) & 0x3FFFu);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+    d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+    d |= (uint64_t)1 << 46;
+    return d;
+}
+
+__device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc,
+                                         uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
+        "l"(a), "l"(b), "r"(idesc), "r"(accumulate));
+}
+
+__device__ __forceinline__ void umma_commit(uint32_t mbar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                     mbar)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}\n"
+            : "=r"(done)
+            : "r"(mbar), "r"(parity)
+            : "memory");
+    }
+}
+
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, float (&v)[8]) {
+    uint32_t r[8];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = __uint_as_float(r[k]);
+}
+__device__ __forceinline__ void tmem_ld4(uint32_t taddr, float (&v)[4]) {
+    uint32_t r[4];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+                 : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = __uint_as_float(r[k]);
+}
+__device__ __forceinline__ void tmem_wait_ld() {
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void fence_before() {
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void fence_after() {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void fence_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// element (row, k) of a K-major no-swizzle f16 operand image with `rows` rows
+__device__ __forceinline__ uint32_t img_off(int row, int k, int rows) {
+    return (uint32_t)((k >> 3) * (rows * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
+}
+
+template <bool MARG>
+__device__ void leaf_step(const LStep &st, const RParams &p, float *act, int64_t base, int tid) {
+    const int I = st.n_out, V = st.n_vars;
+    const int nq = I >> 2;
+    const int units = (RT / 2) * nq;
+    const float2 *ab = reinterpret_cast<const float2 *>(p.fparams + st.par_off);
+    const float *cv = p.fparams + st.w_off;
+    const int32_t *vars = p.vars + st.vars_off;
+    for (int u = tid; u < units; u += RTH) {
+        const int m = (u % (RT / 2)) * 2, q = u / (RT / 2);
+        const float4 cst = *reinterpret_cast<const float4 *>(p.fparams + st.cst_off + 4 * q);
+        float a0[4] = {cst.x, cst.y, cst.z, cst.w};
+        float a1[4] = {cst.x, cst.y, cst.z, cst.w};
+#pragma unroll 2
+        for (int v = 0; v < V; ++v) {
+            const int f = __ldg(vars + v);
+            const float2 xx = __ldg(reinterpret_cast<const float2 *>(p.xT + (int64_t)f * p.ldT + base + m));
+            const float4 p01 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q));
+            const float4 p23 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q + 2));
+            const float aa[4] = {p01.x, p01.z, p23.x, p23.z};
+            const float bb[4] = {p01.y, p01.w, p23.y, p23.w};
+            if constexpr (MARG) {
+                const float4 c4 = __ldg(reinterpret_cast<const float4 *>(cv + (int64_t)v * I + 4 * q));
+                const float cc[4] = {c4.x, c4.y, c4.z, c4.w};
+                const bool n0 = xx.x != xx.x, n1 = xx.y != xx.y;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const float t0 = fmaf(aa[k], xx.x, -bb[k]);
+                    const float t1 = fmaf(aa[k], xx.y, -bb[k]);
+                    a0[k] = fmaf(-(n0 ? cc[k] : t0), n0 ? 1.f : t0, a0[k]);
+                    a1[k] = fmaf(-(n1 ? cc[k] : t1), n1 ? 1.f : t1, a1[k]);
+                }
+            } else {
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const float t0 = fmaf(aa[k], xx.x, -bb[k]);
+                    const float t1 = fmaf(aa[k], xx.y, -bb[k]);
+                    a0[k] = fmaf(-t0, t0, a0[k]);
+                    a1[k] = fmaf(-t1, t1, a1[k]);
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+            *reinterpret_cast<float2 *>(act + st.buf_out + (4 * q + k) * RT + m) =
+                make_float2(a0[k], a1[k]);
+    }
+}
+
+template <bool MARG>
+__global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    // ---- shared-memory carve-up (offsets mirrored by rat_smem_bytes) ----
+    uint64_t *mbar = reinterpret_cast<uint64_t *>(smem);
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 8);
+    size_t off = 128;
+    float *act = reinterpret_cast<float *>(smem + off);
+    off += (size_t)p.smem_floats * 4;
+    float *racc = reinterpret_cast<float *>(smem + off);
+    off += (size_t)p.C * RT * 4;
+    float *ea = reinterpret_cast<float *>(smem + off);
+    off += (size_t)p.max_na * RT * 4;
+    float *sa = reinterpret_cast<float *>(smem + off);
+    float *sb = sa + RT;
+    off += 2 * RT * 4;
+    off = (off + 1023) & ~(size_t)1023;
+    uint8_t *aimg = smem + off;  // [2][RT x kpad] f16 (hi, lo)
+    const size_t aimg_part = (size_t)RT * p.max_kpad * 2;
+    off += 2 * aimg_part;
+    off = (off + 1023) & ~(size_t)1023;
+    uint8_t *wsm = smem + off;   // [2][n_group x kpad] f16 (hi, lo)
+    const size_t w_part_max = (size_t)p.max_ngroup * p.max_kpad * 2;
+
+    const uint32_t mbar_a = r_smem(mbar);
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                         r_smem(tmem_slot)),
+                     "r"(TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mbar_a), "r"(1));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tmem = *tmem_slot;
+    uint32_t phase = 0;
+
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        const int64_t base = tile * RT;
+        for (int i = tid; i < p.C * RT; i += RTH) racc[i] = -CUDART_INF_F;
+        __syncthreads();
+        for (int si = 0; si < p.n_steps; ++si) {
+            const LStep &st = p.steps[si];
+            if (st.type == 0) {
+                leaf_step<MARG>(st, p, act, base, tid);
+                __syncthreads();
+                continue;
+            }
+            // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
+            const int na = st.na, nb = st.nb, kpad = st.k_pad;
+            if (tid < RT) {
+                const int m = tid;
+                const float *VA = act + st.buf_a;
+                float hi = -CUDART_INF_F;
+                for (int i = 0; i < na; ++i) hi = r_maxnan(hi, VA[i * RT + m]);
+                const float hc = fmaxf(hi, -1e30f);
+                for (int i = 0; i < na; ++i) ea[i * RT + m] = r_ex2(VA[i * RT + m] - hc);
+                sa[m] = hi;
+            } else {
+                const int m = tid - RT;
+                const float *VB = act + st.buf_b;
+                float hi = -CUDART_INF_F;
+                for (int j = 0; j < nb; ++j) hi = r_maxnan(hi, VB[j * RT + m]);
+                const float hc = fmaxf(hi, -1e30f);
+                for (int j = 0; j < kpad; ++j) {
+                    const float e = j < nb ? r_ex2(VB[j * RT + m] - hc) : 0.f;
+                    const __half h = __float2half_rn(e);
+                    const __half l = __float2half_rn(e - __half2float(h));
+                    const uint32_t o = img_off(m, j, RT);
+                    *reinterpret_cast<__half *>(aimg + o) = h;
+                    *reinterpret_cast<__half *>(aimg + aimg_part + o) = l;
+                }
+                sb[m] = hi;
+            }
+            fence_async_smem();
+            __syncthreads();
+            // ---------------- phase 2: per N-group MMA + epilogue -------------
+            const uint32_t lbo_a = RT * 16;
+            const uint32_t lbo_b = (uint32_t)st.n_group * 16;
+            const uint32_t idesc = (1u << 4) | ((uint32_t)(st.n_group >> 3) << 17) |
+                                   ((uint32_t)(RT >> 4) << 24);
+            const uint32_t a_hi = r_smem(aimg), a_lo = a_hi + (uint32_t)aimg_part;
+            const uint32_t w_hi = r_smem(wsm), w_lo = w_hi + (uint32_t)w_part_max;
+            const size_t gbytes = (size_t)st.w_group_bytes;
+            for (int g = 0; g < st.n_groups; ++g) {
+                const uint4 *src = reinterpret_cast<const uint4 *>(p.wimg + st.w_off + 2 * gbytes * g);
+                const int nvec = (int)(gbytes / 16);
+                uint4 *dhi = reinterpret_cast<uint4 *>(wsm);
+                uint4 *dlo = reinterpret_cast<uint4 *>(wsm + w_part_max);
+                for (int i = tid; i < nvec; i += RTH) dhi[i] = __ldg(src + i);
+                if (p.prec == 3)
+                    for (int i = tid; i < nvec; i += RTH) dlo[i] = __ldg(src + nvec + i);
+                fence_async_smem();
+                __syncthreads();
+                if (tid == 0) {
+                    fence_after();
+                    for (int kk = 0; kk < kpad / 16; ++kk) {
+                        const uint32_t ka = kk * 2 * lbo_a, kb = kk * 2 * lbo_b;
+                        umma_f16(tmem, umma_desc(a_hi + ka, lbo_a, 128), umma_desc(w_hi + kb, lbo_b, 128),
+                                 idesc, kk > 0);
+                        if (p.prec == 3) {
+                            umma_f16(tmem, umma_desc(a_lo + ka, lbo_a, 128),
+                                     umma_desc(w_hi + kb, lbo_b, 128), idesc, 1);
+                            umma_f16(tmem, umma_desc(a_hi + ka, lbo_a, 128),
+                                     umma_desc(w_lo + kb, lbo_b, 128), idesc, 1);
+                        }
+                    }
+                    umma_commit(mbar_a);
+                }
+                __syncwarp();
+                mbar_wait(mbar_a, phase);
+                phase ^= 1;
+                fence_after();
+                // epilogue: warp quarter q reads TMEM lanes 32q..32q+31 (= samples)
+                const int qd = warp & 3, half = warp >> 2;
+                const int m = qd * 32 + lane;
+                const int s0 = g * st.s_per_group;
+                const int ns = min(st.s_per_group, st.n_out - s0);
+                const int hcut = (ns + 1) >> 1;
+                const int sl0 = half ? hcut : 0, sl1 = half ? ns : hcut;
+                const float shift = sa[m] + sb[m];
+                for (int sl = sl0; sl < sl1; ++sl) {
+                    float acc = 0.f;
+                    const uint32_t trow = tmem + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
+                    int c0 = 0;
+                    for (; c0 + 8 <= na; c0 += 8) {
+                        float t[8];
+                        tmem_ld8(trow + c0, t);
+                        tmem_wait_ld();
+#pragma unroll
+                        for (int k = 0; k < 8; ++k) acc = fmaf(ea[(c0 + k) * RT + m], t[k], acc);
+                    }
+                    if (c0 < na) {  // na % 8 == 4
+                        float t[4];
+                        tmem_ld4(trow + c0, t);
+                        tmem_wait_ld();
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) acc = fmaf(ea[(c0 + k) * RT + m], t[k], acc);
+                    }
+                    const float val = shift + r_lg2(acc);
+                    const int s = s0 + sl;
+                    if (st.type == 1) {
+                        act[st.buf_out + s * RT + m] = val;
+                    } else {
+                        const int col = __ldg(p.root_map + s);
+                        racc[col * RT + m] = r_lse2(racc[col * RT + m], val);
+                    }
+                }
+                fence_before();
+                __syncthreads();
+            }
+        }
+        // ---------------- outputs -------------------------------------------
+        if (tid < RT) {
+            const int64_t srow = base + tid;
+            if (srow < p.n) {
+                int best = -1;
+                float bv = -CUDART_INF_F;
+                for (int c = 0; c < p.C; ++c) {
+                    const float v = racc[c * RT + tid] * 0.6931471805599453f;
+                    p.out[srow * p.C + c] = v;
+                    if (!(v != v) && (best < 0 || v > bv)) {
+                        best = c;
+                        bv = v;
+                    }
+                }
+                if (p.argmax) p.argmax[srow] = best;
+            }
+        }
+        __syncthreads();
+    }
+    fence_before();
+    __syncthreads();
+    if (warp == 0)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
+                     "r"(TMEM_COLS));
+}
+
+// xT[f][s] = x[s][f] for s < n (zero for n <= s < rows_pad)
+__global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64_t ld, int F,
+                                   float *__restrict__ xT, int64_t ldT, int64_t rows_pad) {
+    __shared__ float t[32][33];
+    const int64_t s0 = (int64_t)blockIdx.y * 32, f0 = (int64_t)blockIdx.x * 32;
+    const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
+    for (int k = ty; k < 32; k += 8) {
+        const int64_t s = s0 + k, f = f0 + tx;
+        t[k][tx] = (s < n && f < F) ? __ldg(x + s * ld + f) : 0.f;
+    }
+    __syncthreads();
+    for (int k = ty; k < 32; k += 8) {
+        const int64_t f = f0 + k, s = s0 + tx;
+        if (f < F && s < rows_pad) xT[f * ldT + s] = t[tx][k];
+    }
+}
+
+size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup) {
+    size_t off = 128 + (size_t)smem_floats * 4 + (size_t)C * RT * 4 + (size_t)max_na * RT * 4 +
+                 2 * RT * 4;
+    off = (off + 1023) & ~(size_t)1023;
+    off += 2 * (size_t)RT * max_kpad * 2;
+    off = (off + 1023) & ~(size_t)1023;
+    off += 2 * (size_t)max_ngroup * max_kpad * 2;
+    return off + 1024;  // alignment slack for the dynamic base
+}
+
+cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st) {
+    auto fn = marg ? rat_eval_kernel<true> : rat_eval_kernel<false>;
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    fn<<<grid, RTH, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
+                             int64_t rows_pad, cudaStream_t st) {
+    dim3 grid((unsigned)((F + 31) / 32), (unsigned)((rows_pad + 31) / 32));
+    transpose_x_kernel<<<grid, dim3(32, 8), 0, st>>>(x, n, ld, F, xT, ldT, rows_pad);
+    return cudaGetLastError();
+}
+
+}  // namespace spnb

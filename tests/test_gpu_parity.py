@@ -216,3 +216,47 @@ def test_tiny_discrete_exact():
         x = np.array(list(itertools.product(*[range(-1, k + 1) for k in doms])), np.float32)
         _parity(g, x)
         _parity(g, nan_mask(x, 0.3, seed), marginal=True)
+
+
+# ----------------------------------------------------------------- layered tensor-core path (a5)
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 12, 5), (24, 1, 1, 4, 4, 2),
+                                   (128, 3, 2, 20, 40, 10)])
+def test_layered_rat_small_matches_oracle(shape):
+    F, D, R, S, I, C = shape
+    g = rat_spn(11, F=F, D=D, R=R, S=S, I=I, C=C)
+    x, _ = ancestral_sample(g, 1000, 12)
+    err, P = _parity(g, x, layered_path=2, tc_precision=2)
+    assert P.info()["path"] == 1
+    _parity(g, nan_mask(x, 0.2, 13), marginal=True, layered_path=2, tc_precision=2)
+
+
+def test_layered_matches_generic_path():
+    g = rat_spn(21, F=96, D=3, R=3, S=8, I=8, C=4)
+    x, _ = ancestral_sample(g, 2000, 22)
+    a, am_a, Pa = _run(g, x, layered_path=2, tc_precision=2)
+    b, am_b, Pb = _run(g, x, layered_path=1)
+    assert Pa.info()["path"] == 1 and Pb.info()["path"] == 0
+    _cmp(a, b.astype(np.float64), tol=1e-5)
+
+
+def test_c4_layered_full_graph_sampled():
+    """Config 4 graph (518,730 nodes) on the layered path; oracle on a sample."""
+    from spn_inputs import config_graph
+    g = config_graph("C4")
+    x, _ = ancestral_sample(g, 3000, 4002)
+    for prec in (2, 1):
+        out, am, P = _run(g, x, layered_path=2, tc_precision=prec)
+        assert P.info()["path"] == 1
+        idx = np.random.default_rng(0).choice(len(x), 300, replace=False)
+        ref, am_ref = oracle_eval(g, x[idx])
+        _cmp(out[idx], ref)
+        _cmp_argmax(am[idx], ref, am_ref)
+
+
+def test_layered_ragged_and_chunked():
+    g = rat_spn(31, F=64, D=2, R=2, S=8, I=8, C=3)
+    x, _ = ancestral_sample(g, 70_001, 32)     # > one 65,536-sample chunk, ragged tail
+    out, am, P = _run(g, x, layered_path=2)
+    idx = np.concatenate([np.arange(0, 50), np.arange(65_500, 65_600), np.arange(69_950, 70_001)])
+    ref, _ = oracle_eval(g, x[idx])
+    _cmp(out[idx], ref)

@@ -239,3 +239,32 @@ def test_codegen_multi_root_shared_and_leaf_roots():
     x[:, 2] = np.random.default_rng(2).integers(-1, 4, size=100)
     _check_program(g, x, False)
     _check_program(g, nan_mask(x, 0.3, 1), True)
+
+
+# ------------------------------------------------------------------ layered (RAT-SPN) plan
+def test_layered_detection_accepts_rat_rejects_others():
+    from spn_inputs import rat_spn
+    ok, why = spnb.build_layered(spnb.Graph(rat_spn(3, F=32, D=2, R=2, S=4, I=8, C=3)))
+    assert ok is not None, why
+    for g in (speaker_spn(2001), toy_spn(), tiny_discrete_spn(1)):
+        p, why = spnb.build_layered(spnb.Graph(g))
+        assert p is None and why
+
+
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 12, 5), (24, 1, 1, 4, 4, 2)])
+def test_layered_plan_matches_oracle(shape):
+    from spn_inputs import rat_spn
+    from tests.layered_emulator import emulate_layered
+    F, D, R, S, I, C = shape
+    g = rat_spn(7, F=F, D=D, R=R, S=S, I=I, C=C)
+    plan, why = spnb.build_layered(spnb.Graph(g))
+    assert plan is not None, why
+    x, _ = ancestral_sample(g, 200, 3)
+    for marg, xx in ((False, x), (True, nan_mask(x, 0.2, 4))):
+        em = emulate_layered(plan, xx, g.n_roots, marginal=marg)
+        ref, _ = oracle_eval(g, xx, marginal=marg)
+        err = np.abs(em - ref) / np.maximum(1.0, np.abs(ref))
+        assert err.max() < 1e-5, err.max()
+        # single f16 pass: weight rounding only (2^-12 relative per weight)
+        em1 = emulate_layered(plan, xx, g.n_roots, marginal=marg, prec=1)
+        assert (np.abs(em1 - ref) / np.maximum(1.0, np.abs(ref))).max() < 5e-3

@@ -27,7 +27,8 @@ NVCC_FLAGS = ARCH + ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
 CXX_FLAGS = ["-O2", "-std=c++17", "-fPIC", "-Wall", "-I", CSRC, "-I", INC,
              "-I", "/usr/local/cuda/include"]
 
-CU_SOURCES = ["dag_eval_k1.cu", "dag_eval_k2.cu", "dag_eval_k4.cu", "rat_eval.cu"]
+CU_SOURCES = ["dag_eval_k1.cu", "dag_eval_k2.cu", "dag_eval_k4.cu", "dag_eval_k8.cu",
+              "rat_eval.cu"]
 CXX_SOURCES = ["prepare.cpp", "layered.cpp", "api.cpp"]
 HEADERS = ["program.h", "dag_eval.cuh", "prepare.h", "layered.h"]
 

@@ -22,6 +22,8 @@ namespace spnb {
 cudaError_t dag_eval_launch_k1(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
 cudaError_t dag_eval_launch_k2(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
 cudaError_t dag_eval_launch_k4(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
+cudaError_t dag_eval_launch_k8(const KParams &, bool, bool, int, int, size_t, cudaStream_t);
+int dag_eval_occupancy_k8(bool, bool, int, size_t);
 int dag_eval_occupancy_k1(bool, bool, int, size_t);
 int dag_eval_occupancy_k2(bool, bool, int, size_t);
 int dag_eval_occupancy_k4(bool, bool, int, size_t);
@@ -40,8 +42,11 @@ struct RParams {
     int32_t *argmax;
     int32_t prec;
     int32_t smem_floats, max_kpad, max_ngroup, max_na;
+    int32_t max_vars;
+    int32_t first_leaf;
 };
-size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup);
+size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
+                      int max_vars);
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st);
@@ -101,6 +106,7 @@ struct DevicePlan {
     int64_t chunk = 0;
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
+    int32_t max_vars = 0, first_leaf = 0;
     spn_plan_stats stats;
 };
 
@@ -118,6 +124,7 @@ int launch_kernel(const KParams &p, int K, bool marg, bool xs, int grid, int blo
                   cudaStream_t st) {
     cudaError_t e;
     switch (K) {
+        case 8: e = dag_eval_launch_k8(p, marg, xs, grid, block, smem, st); break;
         case 4: e = dag_eval_launch_k4(p, marg, xs, grid, block, smem, st); break;
         case 2: e = dag_eval_launch_k2(p, marg, xs, grid, block, smem, st); break;
         case 1: e = dag_eval_launch_k1(p, marg, xs, grid, block, smem, st); break;
@@ -129,6 +136,7 @@ int launch_kernel(const KParams &p, int K, bool marg, bool xs, int grid, int blo
 
 int occupancy(int K, bool marg, bool xs, int block, size_t smem) {
     switch (K) {
+        case 8: return dag_eval_occupancy_k8(marg, xs, block, smem);
         case 4: return dag_eval_occupancy_k4(marg, xs, block, smem);
         case 2: return dag_eval_occupancy_k2(marg, xs, block, smem);
         case 1: return dag_eval_occupancy_k1(marg, xs, block, smem);
@@ -214,6 +222,8 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         rp.max_kpad = P.max_kpad;
         rp.max_ngroup = P.max_ngroup;
         rp.max_na = P.max_na;
+        rp.max_vars = P.max_vars;
+        rp.first_leaf = P.first_leaf;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
@@ -332,9 +342,12 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     P->max_kpad = lp.max_kpad;
     P->max_ngroup = lp.max_ngroup;
     P->max_na = lp.max_na;
-    // transposed-feature scratch: chunks of up to 64k samples (or ~256 MB)
+    P->max_vars = lp.max_vars;
+    P->first_leaf = lp.first_leaf;
+    // transposed-feature scratch: chunks small enough (<= ~48 MB) that the
+    // tile slices re-read by every repetition stay resident in L2
     int64_t chunk = 65536;
-    while (chunk > 1024 && (int64_t)g.F * chunk * 4 > ((int64_t)256 << 20)) chunk /= 2;
+    while (chunk > 1024 && (int64_t)g.F * chunk * 4 > ((int64_t)48 << 20)) chunk /= 2;
     P->chunk = chunk;
     int rc;
     std::vector<uint8_t> w8(lp.wimg.size() * 2);
@@ -368,6 +381,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     }
     s.n_tasks = (int64_t)lp.steps.size();
     s.fma_per_sample = lp.fma_per_sample;
+    s.mufu_per_sample = lp.mufu_per_sample;
     s.tc_flops_per_sample = lp.tc_flops_per_sample * (P->prec == 3 ? 3 : 1);
     s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)lp.C + 4;
     s.path = 1;
@@ -483,7 +497,8 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         detect_layered(g, lp);
         size_t lsmem = 0;
         if (lp.ok) {
-            lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup);
+            lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup,
+                                   lp.max_vars);
             if (lsmem > (size_t)smem_optin) {
                 lp.ok = false;
                 lp.why = "activations do not fit in shared memory";
@@ -494,8 +509,9 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, t0, out_plan);
     }
     int K = opt.samples_per_thread ? opt.samples_per_thread : 4;
-    if (K != 1 && K != 2 && K != 4) return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2 or 4");
-    const int max_block = K == 4 ? 384 : 512;
+    if (K != 1 && K != 2 && K != 4 && K != 8)
+        return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
+    const int max_block = K == 8 ? 256 : (K == 4 ? 384 : 512);
     int block = opt.block_threads ? opt.block_threads : max_block;
     if (block % 32 || block < 32 || block > max_block)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 within the kernel bound");
@@ -504,10 +520,11 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     const int tpw = WT + 4;
     const size_t xtile = (size_t)g.F * tpw * 4;
     // stage features in shared memory when a few warps' tiles fit comfortably
-    bool xs = xtile * std::min(nwarps, 8) <= (size_t)smem_optin * 3 / 4;
+    bool xs = xtile * 4 <= (size_t)smem_optin * 3 / 4;
 
     CodegenConfig cfg;
     cfg.K = K;
+    cfg.maxd = K == 8 ? 10 : MAXD;
     cfg.x_in_smem = xs;
     cfg.tpw = tpw;
     cfg.max_task_ops = opt.max_task_nodes > 0 ? opt.max_task_nodes : -1;
@@ -536,8 +553,8 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
             break;
         }
         if (iter > 40) return set_err(SPN_E_UNSUPPORTED, "cannot fit the plan into shared memory");
-        if (xs && nwarps > 8 && !opt.block_threads) {
-            nwarps -= 2;
+        if (xs && nwarps > 4 && !opt.block_threads) {
+            nwarps -= (nwarps > 8 ? 2 : 1);
             block = nwarps * 32;
             continue;
         }
@@ -676,10 +693,12 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
                       int64_t *n_tables, void *edges, int64_t *n_edges, int64_t *slots) {
     if (!valid_graph_handle(graph) || !n_records || !n_tasks || !n_tables || !n_edges)
         return set_err(SPN_E_ARG, "bad arguments");
-    if (samples_per_thread != 1 && samples_per_thread != 2 && samples_per_thread != 4)
-        return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2 or 4");
+    if (samples_per_thread != 1 && samples_per_thread != 2 && samples_per_thread != 4 &&
+        samples_per_thread != 8)
+        return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
     CodegenConfig cfg;
     cfg.K = samples_per_thread;
+    cfg.maxd = samples_per_thread == 8 ? 10 : MAXD;
     cfg.x_in_smem = x_in_smem != 0;
     cfg.tpw = 32 * cfg.K + 4;
     cfg.max_task_ops = max_task_ops;

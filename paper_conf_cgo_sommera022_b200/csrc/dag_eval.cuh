@@ -75,6 +75,21 @@ struct SIO<4> {
     }
 };
 template <>
+struct SIO<8> {
+    static __device__ __forceinline__ void ld(uint32_t a, float (&v)[8]) {
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]) : "r"(a));
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7]) : "r"(a + 16));
+    }
+    static __device__ __forceinline__ void st(uint32_t a, const float (&v)[8]) {
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};"
+                     :: "r"(a), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]) : "memory");
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};"
+                     :: "r"(a + 16), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]) : "memory");
+    }
+};
+template <>
 struct SIO<2> {
     static __device__ __forceinline__ void ld(uint32_t a, float (&v)[2]) {
         asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v[0]), "=f"(v[1]) : "r"(a));
@@ -104,6 +119,19 @@ struct GIO<4> {
     }
     static __device__ __forceinline__ void st(float *p, const float (&v)[4]) {
         *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+};
+template <>
+struct GIO<8> {
+    static __device__ __forceinline__ void ld(const float *p, float (&v)[8]) {
+        const float4 t = *reinterpret_cast<const float4 *>(p);
+        const float4 u = *reinterpret_cast<const float4 *>(p + 4);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+        v[4] = u.x; v[5] = u.y; v[6] = u.z; v[7] = u.w;
+    }
+    static __device__ __forceinline__ void st(float *p, const float (&v)[8]) {
+        *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+        *reinterpret_cast<float4 *>(p + 4) = make_float4(v[4], v[5], v[6], v[7]);
     }
 };
 template <>
@@ -162,8 +190,8 @@ __device__ __forceinline__ void lds4(uint32_t a, uint32_t &x, uint32_t &y, uint3
 
 // Leaf product: acc = C + sum_i leaf_i over the parameter records at pp
 // (ng Gaussian then nd discrete).  Returns the address after the last one.
-template <int S, bool ACC, int K, bool MARG, bool XS>
-__device__ __forceinline__ uint32_t h_lprod(float (&r)[MAXD][K], uint32_t ng, float C,
+template <int S, bool ACC, int D, int K, bool MARG, bool XS>
+__device__ __forceinline__ uint32_t h_lprod(float (&r)[D][K], uint32_t ng, float C,
                                             uint32_t nd, uint32_t pp,
                                             const Env<K, MARG, XS> &e) {
     float acc[K];
@@ -255,8 +283,8 @@ __device__ __forceinline__ float lse_vals(const float (&v)[N], float bias) {
     return (hi + bias) + lg2a(s);
 }
 
-template <int S, int N, int K>
-__device__ __forceinline__ void h_lse(float (&r)[MAXD][K], float bias) {
+template <int S, int N, int D, int K>
+__device__ __forceinline__ void h_lse(float (&r)[D][K], float bias) {
     FOR_K {
         if constexpr (N == 1) {
             r[S - 1][j] += bias;
@@ -291,8 +319,8 @@ __device__ __forceinline__ void gauss_acc(float (&acc)[K], uint32_t pp, const En
 }
 
 // Fused weighted sum over KC Gaussian leaf products (SLPk record).
-template <int S, int KC, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_slp(float (&r)[MAXD][K], uint32_t counts, float bias,
+template <int S, int KC, int D, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_slp(float (&r)[D][K], uint32_t counts, float bias,
                                       const float (&Cs)[4], uint32_t pp,
                                       const Env<K, MARG, XS> &e) {
     float v[KC][K];
@@ -314,8 +342,8 @@ __device__ __forceinline__ void h_slp(float (&r)[MAXD][K], uint32_t counts, floa
 }
 
 // Straight-line product of exactly N Gaussian leaves (parameter records at pp).
-template <int S, bool ACC, int N, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_gprod(float (&r)[MAXD][K], float C, uint32_t pp,
+template <int S, bool ACC, int N, int D, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_gprod(float (&r)[D][K], float C, uint32_t pp,
                                         const Env<K, MARG, XS> &e) {
     uint32_t f[N], ya[N], zb[N], wc[N];
 #pragma unroll
@@ -412,8 +440,8 @@ struct ArgState {
     }
 };
 
-template <int S, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_out(float (&r)[MAXD][K], uint32_t root,
+template <int S, int D, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_out(float (&r)[D][K], uint32_t root,
                                       const Env<K, MARG, XS> &e, ArgState<K> &am) {
     FOR_K {
         const float v = r[S - 1][j] * 0.6931471805599453f;
@@ -428,10 +456,11 @@ __device__ __forceinline__ void h_out(float (&r)[MAXD][K], uint32_t root,
 
 // ---------------------------------------------------------------------------
 // Valid stack depths per op (sp = depth before the op).
-__host__ __device__ constexpr bool op_valid(int op, int sp) {
+__host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
+    if (sp > D) return false;
     return (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
             (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4))
-               ? (sp >= 0 && sp < MAXD)
+               ? (sp >= 0 && sp < D)
            : (op == OP_LACC || op == OP_LSE1 || op == OP_STS || op == OP_STG || op == OP_OUT ||
               (op >= OP_GACC1 && op <= OP_GACC4))
                ? (sp >= 1)
@@ -448,7 +477,7 @@ __host__ __device__ constexpr bool op_valid(int op, int sp) {
 // combinations end the task.
 #define SPN_CASE(O, S)                                                           \
     case O * NSP + S:                                                            \
-        if constexpr (op_valid(O, S)) {                                          \
+        if constexpr (op_valid(O, S, D)) {                                          \
             SPN_BODY_##O(S)                                                      \
         } else {                                                                 \
             return;                                                              \
@@ -462,7 +491,7 @@ __host__ __device__ constexpr bool op_valid(int op, int sp) {
 #define SPN_NEXT(NEWPC)                                                          \
     pc = (NEWPC);                                                                \
     lds4(pc, cx, cy, cz, cw);
-#define SPN_SS(S) (S < MAXD ? S : 0)
+#define SPN_SS(S) (S < D ? S : 0)
 #define SPN_BODY_1(S)                                                            \
     {                                                                            \
         const uint32_t ng = cx >> CASE_BITS, nd = cz, pp = pc + 16;              \
@@ -582,10 +611,10 @@ __host__ __device__ constexpr bool op_valid(int op, int sp) {
 // thread's K samples.  All case labels 0..511 exist, so the dispatch is one
 // unchecked jump-table lookup (build with nvcc -jtd 10).  Each case loads the
 // next record right after reading its own operands (see SPN_NEXT).
-template <int K, bool MARG, bool XS>
+template <int K, bool MARG, bool XS, int D>
 __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &e,
                                          ArgState<K> &am) {
-    float r[MAXD][K];
+    float r[D][K];
     uint32_t pc = prog;
     uint32_t cx, cy, cz, cw;
     lds4(pc, cx, cy, cz, cw);
@@ -652,8 +681,8 @@ __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__r
     asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
 }
 
-template <int K, bool MARG, bool XS>
-__global__ void __launch_bounds__(K == 4 ? 384 : 512) dag_eval_kernel(const KParams p) {
+template <int K, bool MARG, bool XS, int D>
+__global__ void __launch_bounds__(K == 8 ? 256 : (K == 4 ? 384 : 512)) dag_eval_kernel(const KParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     constexpr int WT = 32 * K;
     Rec *prog_s = reinterpret_cast<Rec *>(smem_raw);
@@ -714,7 +743,7 @@ __global__ void __launch_bounds__(K == 4 ? 384 : 512) dag_eval_kernel(const KPar
             const int64_t base = wt * WT;
             ArgState<K> am;
             tile_begin(base, am);
-            run_task<K, MARG, XS>(prog_a, e, am);
+            run_task<K, MARG, XS, D>(prog_a, e, am);
             tile_end(base, am);
         }
     } else {
@@ -731,7 +760,7 @@ __global__ void __launch_bounds__(K == 4 ? 384 : 512) dag_eval_kernel(const KPar
                 for (int64_t i = threadIdx.x; i < len + 2; i += blockDim.x)
                     prog_s[i] = i < len ? p.prog[b + i] : make_end();
                 __syncthreads();
-                if (active) run_task<K, MARG, XS>(prog_a, e, am);
+                if (active) run_task<K, MARG, XS, D>(prog_a, e, am);
             }
             if (active) tile_end(base, am);
         }
@@ -740,10 +769,10 @@ __global__ void __launch_bounds__(K == 4 ? 384 : 512) dag_eval_kernel(const KPar
 
 // ---------------------------------------------------------------------------
 // Host-side helpers, instantiated per K in dag_eval_k{1,2,4}.cu.
-template <int K, bool MARG, bool XS>
+template <int K, bool MARG, bool XS, int D>
 cudaError_t dag_eval_launch_t(const KParams &p, int grid, int block, size_t smem,
                               cudaStream_t st) {
-    auto fn = dag_eval_kernel<K, MARG, XS>;
+    auto fn = dag_eval_kernel<K, MARG, XS, D>;
     // the attribute persists per function: set it only when a larger size is needed
     static size_t configured = 0;
     if (smem > configured) {
@@ -756,9 +785,9 @@ cudaError_t dag_eval_launch_t(const KParams &p, int grid, int block, size_t smem
     return cudaGetLastError();
 }
 
-template <int K, bool MARG, bool XS>
+template <int K, bool MARG, bool XS, int D>
 int dag_eval_occupancy_t(int block, size_t smem) {
-    auto fn = dag_eval_kernel<K, MARG, XS>;
+    auto fn = dag_eval_kernel<K, MARG, XS, D>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
         cudaSuccess)
         return 0;
@@ -768,19 +797,26 @@ int dag_eval_occupancy_t(int block, size_t smem) {
     return nb;
 }
 
+// maximum register-stack depth per samples-per-thread variant (registers:
+// D x K stack values per thread)
+template <int K>
+constexpr int stack_depth() { return K == 8 ? 10 : MAXD; }
+
 #define SPNB_INSTANTIATE_K(K)                                                             \
     cudaError_t dag_eval_launch_k##K(const KParams &p, bool marg, bool xs, int grid,       \
                                      int block, size_t smem, cudaStream_t st) {            \
-        if (marg) return xs ? dag_eval_launch_t<K, true, true>(p, grid, block, smem, st)  \
-                            : dag_eval_launch_t<K, true, false>(p, grid, block, smem, st); \
-        return xs ? dag_eval_launch_t<K, false, true>(p, grid, block, smem, st)           \
-                  : dag_eval_launch_t<K, false, false>(p, grid, block, smem, st);         \
+        constexpr int D = stack_depth<K>();                                               \
+        if (marg) return xs ? dag_eval_launch_t<K, true, true, D>(p, grid, block, smem, st)  \
+                            : dag_eval_launch_t<K, true, false, D>(p, grid, block, smem, st); \
+        return xs ? dag_eval_launch_t<K, false, true, D>(p, grid, block, smem, st)           \
+                  : dag_eval_launch_t<K, false, false, D>(p, grid, block, smem, st);         \
     }                                                                                     \
     int dag_eval_occupancy_k##K(bool marg, bool xs, int block, size_t smem) {             \
-        if (marg) return xs ? dag_eval_occupancy_t<K, true, true>(block, smem)            \
-                            : dag_eval_occupancy_t<K, true, false>(block, smem);          \
-        return xs ? dag_eval_occupancy_t<K, false, true>(block, smem)                     \
-                  : dag_eval_occupancy_t<K, false, false>(block, smem);                   \
+        constexpr int D = stack_depth<K>();                                               \
+        if (marg) return xs ? dag_eval_occupancy_t<K, true, true, D>(block, smem)            \
+                            : dag_eval_occupancy_t<K, true, false, D>(block, smem);          \
+        return xs ? dag_eval_occupancy_t<K, false, true, D>(block, smem)                     \
+                  : dag_eval_occupancy_t<K, false, false, D>(block, smem);                   \
     }
 
 }  // namespace spnb

@@ -433,7 +433,17 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
     // root values must be emitted in root-index order: remap via root_order
     plan.root_map = root_order;
     plan.smem_floats = buf_peak;
+    int32_t next = -1;
+    for (int32_t i = (int32_t)plan.steps.size() - 1; i >= 0; --i) {
+        LStep &st = plan.steps[i];
+        if (st.type == 0) {
+            st.rep = next;
+            next = i;
+        }
+    }
+    plan.first_leaf = next;
     for (auto &st : plan.steps) {
+        if (st.type == 0) plan.max_vars = std::max(plan.max_vars, st.n_vars);
         plan.max_kpad = std::max(plan.max_kpad, st.k_pad);
         plan.max_ngroup = std::max(plan.max_ngroup, st.n_group);
         plan.max_na = std::max(plan.max_na, st.na);

@@ -38,7 +38,7 @@ struct LStep {
     int64_t cst_off;     // LEAF: float C[n_out]
     int64_t w_off;       // SUM/ROOT: byte offset of the f16 weight images
     int64_t w_group_bytes;  // bytes per (group, part) image
-    int32_t rep;         // repetition (ROOT)
+    int32_t rep;         // LEAF: index of the next LEAF step in the schedule (-1: none)
     int32_t pad_;
 };
 
@@ -51,7 +51,8 @@ struct LayeredPlan {
     std::vector<float> fparams;  // leaf (a,b) pairs and C constants
     std::vector<uint16_t> wimg;  // f16 weight images (hi then lo per group)
     int32_t smem_floats = 0;     // activation buffers
-    int32_t max_kpad = 0, max_ngroup = 0, max_na = 0;
+    int32_t max_kpad = 0, max_ngroup = 0, max_na = 0, max_vars = 0;
+    int32_t first_leaf = -1;
     std::vector<int32_t> root_map;  // root-region value index -> output column
     int64_t tc_flops_per_sample = 0;  // one precision pass
     int64_t fma_per_sample = 0;

@@ -559,7 +559,7 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
     for (int64_t u = 0; u < c.n; ++u) {
         if (is_leaf(c.kind[u])) continue;
         int32_t nd = compute_need(u);
-        while (nd > MAXD) {
+        while (nd > cfg.maxd) {
             // materialise the non-stored inner child with the largest need
             int64_t best = -1;
             int32_t bn = 0;
@@ -593,7 +593,7 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
     bool overflow = false;
     auto rec_of = [&](uint32_t op, int sp, uint32_t arg, uint32_t y = 0, uint32_t z = 0,
                       uint32_t w = 0) {
-        if (sp > MAXD || sp < 0 || arg > ARG_MAX) {
+        if (sp > cfg.maxd || sp < 0 || arg > ARG_MAX) {
             overflow = true;
             return;
         }
@@ -766,7 +766,7 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
         prog.push_back(make_rec(OP_END, 0, 0));
     }
     out.task_off.push_back((int64_t)prog.size());
-    if (overflow || max_sp > MAXD)
+    if (overflow || max_sp > cfg.maxd)
         return fail(msg, SPN_E_UNSUPPORTED, "register stack overflow (depth %lld)", max_sp);
     out.max_stack = max_sp;
     for (int32_t t = 0; t < T; ++t)

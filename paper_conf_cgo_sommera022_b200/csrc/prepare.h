@@ -25,6 +25,7 @@ struct CodegenConfig {
     int64_t max_task_ops = -1; // partition cap (LoSPN ops); <= 0: single task
     int64_t smem_slot_cap = 0; // shared-memory slots available per warp
     int lse_max = 4;           // largest stack LSE fan-in
+    int maxd = MAXD;           // register-stack depth of the kernel variant
 };
 
 struct PlanProgram {

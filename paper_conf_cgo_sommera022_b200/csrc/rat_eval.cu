@@ -46,6 +46,8 @@ struct RParams {
     int32_t *argmax;
     int32_t prec;       // 1: single f16 pass; 3: hi/lo split
     int32_t smem_floats, max_kpad, max_ngroup, max_na;
+    int32_t max_vars;   // largest leaf region (staged x rows)
+    int32_t first_leaf; // index of the first LEAF step
 };
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
@@ -145,28 +147,43 @@ __device__ __forceinline__ void fence_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// TMA bulk copy global -> shared, completion counted on an mbarrier (tx bytes)
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes,
+                                         uint32_t mbar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            dst),
+        "l"(src), "r"(bytes), "r"(mbar)
+        : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t mbar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(bytes)
+                 : "memory");
+}
+
 // element (row, k) of a K-major no-swizzle f16 operand image with `rows` rows
 __device__ __forceinline__ uint32_t img_off(int row, int k, int rows) {
     return (uint32_t)((k >> 3) * (rows * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
 }
 
+// LEAF step: the region's feature rows xs[v][m] (128 samples) are in shared
+// memory (staged by a bulk copy).  Thread unit = (sample pair, 4 distributions).
 template <bool MARG>
-__device__ void leaf_step(const LStep &st, const RParams &p, float *act, int64_t base, int tid) {
+__device__ void leaf_step(const LStep &st, const RParams &p, float *act, const float *xs,
+                          int tid) {
     const int I = st.n_out, V = st.n_vars;
     const int nq = I >> 2;
     const int units = (RT / 2) * nq;
     const float2 *ab = reinterpret_cast<const float2 *>(p.fparams + st.par_off);
     const float *cv = p.fparams + st.w_off;
-    const int32_t *vars = p.vars + st.vars_off;
     for (int u = tid; u < units; u += RTH) {
         const int m = (u % (RT / 2)) * 2, q = u / (RT / 2);
         const float4 cst = *reinterpret_cast<const float4 *>(p.fparams + st.cst_off + 4 * q);
         float a0[4] = {cst.x, cst.y, cst.z, cst.w};
         float a1[4] = {cst.x, cst.y, cst.z, cst.w};
-#pragma unroll 2
+#pragma unroll 4
         for (int v = 0; v < V; ++v) {
-            const int f = __ldg(vars + v);
-            const float2 xx = __ldg(reinterpret_cast<const float2 *>(p.xT + (int64_t)f * p.ldT + base + m));
+            const float2 xx = *reinterpret_cast<const float2 *>(xs + v * RT + m);
             const float4 p01 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q));
             const float4 p23 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q + 2));
             const float aa[4] = {p01.x, p01.z, p23.x, p23.z};
@@ -203,9 +220,9 @@ template <bool MARG>
 __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    // ---- shared-memory carve-up (offsets mirrored by rat_smem_bytes) ----
-    uint64_t *mbar = reinterpret_cast<uint64_t *>(smem);
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 8);
+    // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1 w, 2/3 x
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 64);
     size_t off = 128;
     float *act = reinterpret_cast<float *>(smem + off);
     off += (size_t)p.smem_floats * 4;
@@ -216,15 +233,17 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     float *sa = reinterpret_cast<float *>(smem + off);
     float *sb = sa + RT;
     off += 2 * RT * 4;
+    float *xsb = reinterpret_cast<float *>(smem + off);  // [2][max_vars][RT]
+    off += 2 * (size_t)p.max_vars * RT * 4;
     off = (off + 1023) & ~(size_t)1023;
     uint8_t *aimg = smem + off;  // [2][RT x kpad] f16 (hi, lo)
     const size_t aimg_part = (size_t)RT * p.max_kpad * 2;
     off += 2 * aimg_part;
     off = (off + 1023) & ~(size_t)1023;
     uint8_t *wsm = smem + off;   // [2][n_group x kpad] f16 (hi, lo)
-    const size_t w_part_max = (size_t)p.max_ngroup * p.max_kpad * 2;
 
-    const uint32_t mbar_a = r_smem(mbar);
+    const uint32_t bar_mma = r_smem(bars), bar_w = r_smem(bars + 1);
+    const uint32_t bar_x0 = r_smem(bars + 2);
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                          r_smem(tmem_slot)),
@@ -232,16 +251,40 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     if (tid == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mbar_a), "r"(1));
+        for (int i = 0; i < 4; ++i)
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(r_smem(bars + i)), "r"(1));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     fence_before();
     __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
-    uint32_t phase = 0;
+    uint32_t ph_mma = 0, ph_w = 0, ph_x[2] = {0, 0};
+    int xbuf = 0;  // buffer of the next leaf step
+
+    // x rows of a leaf step for the tile at `base` -> buffer b (one thread)
+    auto issue_x = [&](int step, int64_t base, int b) {
+        const LStep &ls = p.steps[step];
+        const uint32_t dst = r_smem(xsb + (size_t)b * p.max_vars * RT);
+        const uint32_t bar = bar_x0 + 8 * b;
+        mbar_expect_tx(bar, (uint32_t)ls.n_vars * RT * 4);
+        for (int v = 0; v < ls.n_vars; ++v) {
+            const int f = __ldg(p.vars + ls.vars_off + v);
+            bulk_g2s(dst + v * RT * 4, p.xT + (int64_t)f * p.ldT + base, RT * 4, bar);
+        }
+    };
+    auto issue_w = [&](const LStep &ws, int g) {
+        const size_t gb = (size_t)ws.w_group_bytes;
+        const uint8_t *src = p.wimg + ws.w_off + 2 * gb * g;
+        mbar_expect_tx(bar_w, (uint32_t)(gb * (p.prec == 3 ? 2 : 1)));
+        bulk_g2s(r_smem(wsm), src, (uint32_t)gb, bar_w);
+        if (p.prec == 3)
+            bulk_g2s(r_smem(wsm) + (uint32_t)((size_t)p.max_ngroup * p.max_kpad * 2), src + gb,
+                     (uint32_t)gb, bar_w);
+    };
 
     const int64_t n_tiles = (p.n + RT - 1) / RT;
+    if (tid == 0 && (int64_t)blockIdx.x < n_tiles) issue_x(p.first_leaf, (int64_t)blockIdx.x * RT, 0);
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const int64_t base = tile * RT;
         for (int i = tid; i < p.C * RT; i += RTH) racc[i] = -CUDART_INF_F;
@@ -249,11 +292,21 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
         for (int si = 0; si < p.n_steps; ++si) {
             const LStep &st = p.steps[si];
             if (st.type == 0) {
-                leaf_step<MARG>(st, p, act, base, tid);
+                const int b = xbuf;
+                mbar_wait(bar_x0 + 8 * b, ph_x[b]);
+                ph_x[b] ^= 1;
+                if (tid == 0) {  // prefetch the next leaf step's rows (maybe next tile)
+                    if (st.rep >= 0) issue_x(st.rep, base, b ^ 1);
+                    else if (tile + gridDim.x < n_tiles)
+                        issue_x(p.first_leaf, base + (int64_t)gridDim.x * RT, b ^ 1);
+                }
+                xbuf ^= 1;
+                leaf_step<MARG>(st, p, act, xsb + (size_t)b * p.max_vars * RT, tid);
                 __syncthreads();
                 continue;
             }
             // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
+            if (tid == 0) issue_w(st, 0);
             const int na = st.na, nb = st.nb, kpad = st.k_pad;
             if (tid < RT) {
                 const int m = tid;
@@ -287,18 +340,11 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             const uint32_t idesc = (1u << 4) | ((uint32_t)(st.n_group >> 3) << 17) |
                                    ((uint32_t)(RT >> 4) << 24);
             const uint32_t a_hi = r_smem(aimg), a_lo = a_hi + (uint32_t)aimg_part;
-            const uint32_t w_hi = r_smem(wsm), w_lo = w_hi + (uint32_t)w_part_max;
-            const size_t gbytes = (size_t)st.w_group_bytes;
+            const uint32_t w_hi = r_smem(wsm),
+                           w_lo = w_hi + (uint32_t)((size_t)p.max_ngroup * p.max_kpad * 2);
             for (int g = 0; g < st.n_groups; ++g) {
-                const uint4 *src = reinterpret_cast<const uint4 *>(p.wimg + st.w_off + 2 * gbytes * g);
-                const int nvec = (int)(gbytes / 16);
-                uint4 *dhi = reinterpret_cast<uint4 *>(wsm);
-                uint4 *dlo = reinterpret_cast<uint4 *>(wsm + w_part_max);
-                for (int i = tid; i < nvec; i += RTH) dhi[i] = __ldg(src + i);
-                if (p.prec == 3)
-                    for (int i = tid; i < nvec; i += RTH) dlo[i] = __ldg(src + nvec + i);
-                fence_async_smem();
-                __syncthreads();
+                mbar_wait(bar_w, ph_w);
+                ph_w ^= 1;
                 if (tid == 0) {
                     fence_after();
                     for (int kk = 0; kk < kpad / 16; ++kk) {
@@ -312,12 +358,15 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                                      umma_desc(w_lo + kb, lbo_b, 128), idesc, 1);
                         }
                     }
-                    umma_commit(mbar_a);
+                    umma_commit(bar_mma);
                 }
                 __syncwarp();
-                mbar_wait(mbar_a, phase);
-                phase ^= 1;
+                mbar_wait(bar_mma, ph_mma);
+                ph_mma ^= 1;
                 fence_after();
+                // the MMA has consumed the weights: fetch the next group's now,
+                // overlapping the copy with this group's epilogue
+                if (tid == 0 && g + 1 < st.n_groups) issue_w(st, g + 1);
                 // epilogue: warp quarter q reads TMEM lanes 32q..32q+31 (= samples)
                 const int qd = warp & 3, half = warp >> 2;
                 const int m = qd * 32 + lane;
@@ -400,9 +449,10 @@ __global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64
     }
 }
 
-size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup) {
+size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
+                      int max_vars) {
     size_t off = 128 + (size_t)smem_floats * 4 + (size_t)C * RT * 4 + (size_t)max_na * RT * 4 +
-                 2 * RT * 4;
+                 2 * RT * 4 + 2 * (size_t)max_vars * RT * 4;
     off = (off + 1023) & ~(size_t)1023;
     off += 2 * (size_t)RT * max_kpad * 2;
     off = (off + 1023) & ~(size_t)1023;

@@ -176,6 +176,7 @@ def test_codegen_speaker_tree():
     p = _check_program(g, x, False)
     assert len(p["task_off"]) == 2 and p["n_gslots"] == 0 and p["n_sslots"] == 0
     _check_program(g, nan_mask(x, 0.2, 3), True)
+    _check_program(g, x, False, K=8)
 
 
 @pytest.mark.parametrize("cap", [30, 150, 700])

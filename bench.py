@@ -41,6 +41,34 @@ def _peaks():
     return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
+def samples_per_rank(cfg: str, world: int) -> tuple[int, str]:
+    """C5 is a strong-scaling config (10M samples split over the GPUs,
+    BASELINE.json configs[4]); the others are weak (a full batch per GPU)."""
+    from spn_inputs import CONFIGS
+    n = CONFIGS[cfg]["n_samples"]
+    if cfg == "C5":
+        return n // world, "strong"
+    return n, "weak"
+
+
+def device_uniform(n: int, F: int, seed: int, start: int, dev, chunk: int = 65536):
+    """Counter-based U[0,1) features generated on the GPU, one generator per
+    65,536-sample chunk (shard independent; the RAT-SPN throughput recipe)."""
+    import torch
+    x = torch.empty((n, F), dtype=torch.float32, device=dev)
+    pos = start
+    while pos < start + n:
+        c = pos // chunk
+        gen = torch.Generator(device=dev)
+        gen.manual_seed(seed * 1_000_003 + c)
+        blk = torch.rand((chunk, F), generator=gen, device=dev, dtype=torch.float32)
+        a = pos - c * chunk
+        b = min(chunk, start + n - c * chunk)
+        x[pos - start:pos - start + (b - a)] = blk[a:b]
+        pos += b - a
+    return x
+
+
 def make_workload(cfg: str, rank: int, marginal: bool):
     """Seeded graph + this rank's input batch (host numpy)."""
     from spn_inputs import (CONFIGS, config_graph, ancestral_sample, add_outliers, nan_mask,
@@ -122,10 +150,14 @@ def cpu_baseline(g, x, marginal, target_s=12.0):
     """The oracle as it stands, timed on this host's cores on a bounded
     sample (~target_s seconds)."""
     from oracle import oracle_eval, num_threads
-    n0 = min(len(x), 2000)
-    t = time.perf_counter()
-    oracle_eval(g, x[:n0], marginal=marginal)
-    dt = time.perf_counter() - t
+    n0 = min(len(x), 16)
+    while True:
+        t = time.perf_counter()
+        oracle_eval(g, x[:n0], marginal=marginal)
+        dt = time.perf_counter() - t
+        if dt > 0.5 or n0 >= len(x):
+            break
+        n0 = min(len(x), n0 * 8)
     n = int(min(len(x), max(n0, n0 * target_s / max(dt, 1e-6))))
     t = time.perf_counter()
     oracle_eval(g, x[:n], marginal=marginal)
@@ -202,14 +234,24 @@ def run_ours(args):
         dist.barrier()
     import paper_conf_cgo_sommera022_b200 as spnb
 
-    g, x, n = make_workload(args.config, rank, args.marginal)
+    n_rank, scaling = samples_per_rank(args.config, world)
+    if args.config in ("C4", "C5"):
+        from spn_inputs import CONFIGS, config_graph
+        g = config_graph(args.config)
+        n = n_rank
+        xd = device_uniform(n, g.n_features, CONFIGS[args.config]["data_seed"], rank * n, dev)
+        x = xd[:min(n, 262_144)].cpu().numpy()   # host copy of a bounded subset (e2e, oracle)
+    else:
+        g, x, n = make_workload(args.config, rank, args.marginal)
+        xd = None
     G = spnb.Graph(g)
     t0 = time.perf_counter()
     P = spnb.Plan(G, device=local, samples_per_thread=args.K, block_threads=args.block,
                   tc_precision=args.tc_precision)
     prep_s = time.perf_counter() - t0
     info = P.info()
-    xd = torch.from_numpy(x).to(dev)
+    if xd is None:
+        xd = torch.from_numpy(x).to(dev)
     R = g.n_roots
     want_am = R > 1
     out = torch.empty((n, R), dtype=torch.float32, device=dev)
@@ -252,11 +294,12 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     tot_ms = float(t.item())
     value = n * world * args.steps / (tot_ms / 1e3)
+    n_e2e = x.shape[0]
 
     # ---- end to end through the public host-buffer API (H2D + D2H inside) ----
     xh = torch.from_numpy(x).pin_memory()
-    oh = torch.empty((n, R), dtype=torch.float32).pin_memory()
-    amh = torch.empty((n,), dtype=torch.int32).pin_memory() if want_am else None
+    oh = torch.empty((n_e2e, R), dtype=torch.float32).pin_memory()
+    amh = torch.empty((n_e2e,), dtype=torch.int32).pin_memory() if want_am else None
     P.infer_host(xh, marginal=args.marginal, out=oh, argmax=amh, want_argmax=want_am)
     e2e_steps = max(1, min(args.steps, 10))
     if world > 1:
@@ -268,7 +311,7 @@ def run_ours(args):
     te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_val = n * world / float(te.item())
+    e2e_val = n_e2e * world / float(te.item())
 
     if rank == 0:
         peaks, src = _peaks()
@@ -310,8 +353,10 @@ def run_ours(args):
         cpu = cpu_baseline(g, x, args.marginal) if world == 1 or True else None
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-                "dtype": "f32", "data": "synthetic (seeded ancestral samples)",
+                "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
+                "dtype": "f32", "data": ("synthetic (seeded ancestral samples)"
+                                         if args.config not in ("C4", "C5") else
+                                         "synthetic (counter-based U[0,1) per 65,536-sample chunk)"),
                 "config": _config_dict(args, g, n) | {
                     "plan": {k: info[k] for k in ("path", "n_nodes", "n_tasks", "n_records",
                                                   "block_threads", "samples_per_thread",
@@ -322,7 +367,8 @@ def run_ours(args):
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
                 "e2e": {"value": e2e_val, "unit": UNIT,
                         "h2d_bytes_per_step": int(x.nbytes),
-                        "d2h_bytes_per_step": int(n * R * 4 + (n * 4 if want_am else 0)),
+                        "d2h_bytes_per_step": int(n_e2e * R * 4 + (n_e2e * 4 if want_am else 0)),
+                        "samples_per_step": int(n_e2e),
                         "timing": "wall clock around the synchronous host-buffer call"},
                 "gpu_launches": args.steps,
                 "step_ms": {"min": min(times), "median": statistics.median(times),

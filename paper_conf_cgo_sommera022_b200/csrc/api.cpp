@@ -44,9 +44,10 @@ struct RParams {
     int32_t smem_floats, max_kpad, max_ngroup, max_na;
     int32_t max_vars;
     int32_t first_leaf;
+    int32_t max_leaf_params;
 };
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
-                      int max_vars);
+                      int max_vars, int max_leaf_params);
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st);
@@ -106,7 +107,7 @@ struct DevicePlan {
     int64_t chunk = 0;
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
-    int32_t max_vars = 0, first_leaf = 0;
+    int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0;
     spn_plan_stats stats;
 };
 
@@ -224,6 +225,7 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         rp.max_na = P.max_na;
         rp.max_vars = P.max_vars;
         rp.first_leaf = P.first_leaf;
+        rp.max_leaf_params = P.max_leaf_params;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
@@ -344,10 +346,12 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     P->max_na = lp.max_na;
     P->max_vars = lp.max_vars;
     P->first_leaf = lp.first_leaf;
+    P->max_leaf_params = lp.max_leaf_params;
     // transposed-feature scratch: chunks small enough (<= ~48 MB) that the
     // tile slices re-read by every repetition stay resident in L2
-    int64_t chunk = 65536;
-    while (chunk > 1024 && (int64_t)g.F * chunk * 4 > ((int64_t)48 << 20)) chunk /= 2;
+    // (a multiple of one full wave of 128-sample tiles: 148 SMs x 128)
+    const int64_t wave = (int64_t)sms * 128;
+    int64_t chunk = std::max<int64_t>(1, (((int64_t)48 << 20) / ((int64_t)g.F * 4)) / wave) * wave;
     P->chunk = chunk;
     int rc;
     std::vector<uint8_t> w8(lp.wimg.size() * 2);
@@ -498,7 +502,7 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         size_t lsmem = 0;
         if (lp.ok) {
             lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup,
-                                   lp.max_vars);
+                                   lp.max_vars, lp.max_leaf_params);
             if (lsmem > (size_t)smem_optin) {
                 lp.ok = false;
                 lp.why = "activations do not fit in shared memory";

@@ -276,7 +276,8 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
             return fail("internal sum region with several partitions");
     for (auto &reg : regions) {
         if (reg.nodes.size() > 64) return fail("region with more than 64 values");
-        if (reg.leaf && reg.nodes.size() % 4) return fail("leaf region size must be a multiple of 4");
+        if (reg.leaf && (reg.nodes.size() % 8 || reg.nodes.size() > 64))
+            return fail("leaf region size must be a multiple of 8 (<= 64)");
         if (!reg.leaf && reg.nodes.size() < 1) return fail("empty region");
     }
     for (auto &P : parts) {
@@ -364,12 +365,11 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
             st.n_vars = V;
             st.vars_off = (int64_t)plan.vars.size();
             plan.vars.insert(plan.vars.end(), reg.vars.begin(), reg.vars.end());
-            // params [v][i'] float2 (a, b); i' = half * Ih + k for dist i = half * Ih + k
+            // staged parameter block (16-byte aligned, one bulk copy):
+            //   ab[v][i] = (a, b) float2, then C[i] (padded to a multiple of 4)
             while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
             st.par_off = (int64_t)plan.fparams.size();
-            const int32_t Ih = (I + 1) / 2;
-            std::vector<float> ab((size_t)V * 2 * Ih * 2, 0.f);
-            std::vector<float> cv((size_t)V * 2 * Ih, 0.f);
+            std::vector<float> ab((size_t)V * I * 2, 0.f);
             std::vector<double> Cs(I, 0.0);
             for (int32_t i = 0; i < I; ++i) {
                 const int64_t u = reg.nodes[i];
@@ -383,20 +383,17 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
                                                 reg.vars.begin());
                     const double *pp = g.params.data() + g.param_begin[o];
                     const double a = 1.0 / (pp[1] * std::sqrt(2.0 * M_LN2));
-                    const double cc = -std::log2(pp[1] * std::sqrt(2.0 * M_PI));
-                    Cs[i] += cc;
-                    cv[(size_t)v * 2 * Ih + i] = (float)cc;
-                    const size_t idx = ((size_t)v * 2 * Ih + (size_t)i) * 2;
+                    Cs[i] += -std::log2(pp[1] * std::sqrt(2.0 * M_PI));
+                    const size_t idx = ((size_t)v * I + (size_t)i) * 2;
                     ab[idx] = (float)a;
                     ab[idx + 1] = (float)(a * pp[0]);
                 }
             }
             plan.fparams.insert(plan.fparams.end(), ab.begin(), ab.end());
-            while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
             st.cst_off = (int64_t)plan.fparams.size();
-            for (int32_t i = 0; i < 2 * Ih; ++i) plan.fparams.push_back(i < I ? (float)Cs[i] : 0.f);
-            st.w_off = (int64_t)plan.fparams.size();  // LEAF: per-(v,i) c (marginal)
-            plan.fparams.insert(plan.fparams.end(), cv.begin(), cv.end());
+            for (int32_t i = 0; i < I; ++i) plan.fparams.push_back((float)Cs[i]);
+            while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
+            st.w_off = (int64_t)plan.fparams.size() - st.par_off;  // LEAF: block size (floats)
             st.buf_out = top0;
             buf_top = top0 + I * TILE;
             buf_peak = std::max(buf_peak, buf_top);
@@ -443,7 +440,10 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
     }
     plan.first_leaf = next;
     for (auto &st : plan.steps) {
-        if (st.type == 0) plan.max_vars = std::max(plan.max_vars, st.n_vars);
+        if (st.type == 0) {
+            plan.max_vars = std::max(plan.max_vars, st.n_vars);
+            plan.max_leaf_params = std::max<int32_t>(plan.max_leaf_params, (int32_t)st.w_off);
+        }
         plan.max_kpad = std::max(plan.max_kpad, st.k_pad);
         plan.max_ngroup = std::max(plan.max_ngroup, st.n_group);
         plan.max_na = std::max(plan.max_na, st.na);

@@ -34,9 +34,9 @@ struct LStep {
     int32_t n_group;     // N columns per group (multiple of 16)
     int32_t n_vars;      // LEAF: variables of the region
     int64_t vars_off;    // LEAF: int32 offset into vars[]
-    int64_t par_off;     // LEAF: float2 (a, b) [n_vars][n_out]; C at cst_off
-    int64_t cst_off;     // LEAF: float C[n_out]
-    int64_t w_off;       // SUM/ROOT: byte offset of the f16 weight images
+    int64_t par_off;     // LEAF: float offset of the staged block: (a, b)[n_vars][n_out], C[n_out]
+    int64_t cst_off;     // LEAF: float offset of C[n_out] (inside the block)
+    int64_t w_off;       // SUM/ROOT: byte offset of the f16 weight images; LEAF: block floats
     int64_t w_group_bytes;  // bytes per (group, part) image
     int32_t rep;         // LEAF: index of the next LEAF step in the schedule (-1: none)
     int32_t pad_;
@@ -52,6 +52,7 @@ struct LayeredPlan {
     std::vector<uint16_t> wimg;  // f16 weight images (hi then lo per group)
     int32_t smem_floats = 0;     // activation buffers
     int32_t max_kpad = 0, max_ngroup = 0, max_na = 0, max_vars = 0;
+    int32_t max_leaf_params = 0;    // floats of the largest staged leaf parameter block
     int32_t first_leaf = -1;
     std::vector<int32_t> root_map;  // root-region value index -> output column
     int64_t tc_flops_per_sample = 0;  // one precision pass

@@ -48,6 +48,7 @@ struct RParams {
     int32_t smem_floats, max_kpad, max_ngroup, max_na;
     int32_t max_vars;   // largest leaf region (staged x rows)
     int32_t first_leaf; // index of the first LEAF step
+    int32_t max_leaf_params;  // floats of the largest staged leaf parameter block
 };
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
@@ -166,53 +167,70 @@ __device__ __forceinline__ uint32_t img_off(int row, int k, int rows) {
     return (uint32_t)((k >> 3) * (rows * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
 }
 
-// LEAF step: the region's feature rows xs[v][m] (128 samples) are in shared
-// memory (staged by a bulk copy).  Thread unit = (sample pair, 4 distributions).
-template <bool MARG>
-__device__ void leaf_step(const LStep &st, const RParams &p, float *act, const float *xs,
-                          int tid) {
+// LEAF step: the region's feature rows xs[v][m] (128 samples) and its
+// parameter block ab[v][i] = (a, b), C[i] are in shared memory (one bulk-copy
+// stage).  256 threads = 32 sample quads x 8 distribution groups of DPT =
+// I/8 distributions; per variable a thread does 1 LDS.128 (x) + DPT LDS.64
+// (broadcast) for 8 DPT FFMA.
+template <int DPT, bool MARG>
+__device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const float *xs,
+                                            const float *prm, int tid) {
     const int I = st.n_out, V = st.n_vars;
-    const int nq = I >> 2;
-    const int units = (RT / 2) * nq;
-    const float2 *ab = reinterpret_cast<const float2 *>(p.fparams + st.par_off);
-    const float *cv = p.fparams + st.w_off;
-    for (int u = tid; u < units; u += RTH) {
-        const int m = (u % (RT / 2)) * 2, q = u / (RT / 2);
-        const float4 cst = *reinterpret_cast<const float4 *>(p.fparams + st.cst_off + 4 * q);
-        float a0[4] = {cst.x, cst.y, cst.z, cst.w};
-        float a1[4] = {cst.x, cst.y, cst.z, cst.w};
-#pragma unroll 4
-        for (int v = 0; v < V; ++v) {
-            const float2 xx = *reinterpret_cast<const float2 *>(xs + v * RT + m);
-            const float4 p01 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q));
-            const float4 p23 = __ldg(reinterpret_cast<const float4 *>(ab + (int64_t)v * I + 4 * q + 2));
-            const float aa[4] = {p01.x, p01.z, p23.x, p23.z};
-            const float bb[4] = {p01.y, p01.w, p23.y, p23.w};
-            if constexpr (MARG) {
-                const float4 c4 = __ldg(reinterpret_cast<const float4 *>(cv + (int64_t)v * I + 4 * q));
-                const float cc[4] = {c4.x, c4.y, c4.z, c4.w};
-                const bool n0 = xx.x != xx.x, n1 = xx.y != xx.y;
+    const int mq = (tid & 31) * 4;           // 4 samples
+    const int d0 = (tid >> 5) * DPT;         // first distribution
+    const float2 *ab = reinterpret_cast<const float2 *>(prm);
+    const float *C = prm + 2 * V * I;
+    float acc[DPT][4];
+#pragma unroll
+    for (int d = 0; d < DPT; ++d) {
+        const float cd = C[d0 + d];
+        acc[d][0] = cd; acc[d][1] = cd; acc[d][2] = cd; acc[d][3] = cd;
+    }
+    // log2 N = c - t^2 with c = log2(a) + K0 (used only to cancel a NaN leaf)
+    const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi)
+#pragma unroll 2
+    for (int v = 0; v < V; ++v) {
+        const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + mq);
+        const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
+        bool anynan = false;
+        if constexpr (MARG) anynan = (xv[0] != xv[0]) | (xv[1] != xv[1]) | (xv[2] != xv[2]) | (xv[3] != xv[3]);
+#pragma unroll
+        for (int d = 0; d < DPT; ++d) {
+            const float2 q = ab[v * I + d0 + d];
+            if (MARG && anynan) {
+                const float cc = r_lg2(q.x) + K0;
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
-                    const float t0 = fmaf(aa[k], xx.x, -bb[k]);
-                    const float t1 = fmaf(aa[k], xx.y, -bb[k]);
-                    a0[k] = fmaf(-(n0 ? cc[k] : t0), n0 ? 1.f : t0, a0[k]);
-                    a1[k] = fmaf(-(n1 ? cc[k] : t1), n1 ? 1.f : t1, a1[k]);
+                    const bool nan = xv[k] != xv[k];
+                    const float t = fmaf(q.x, xv[k], -q.y);
+                    acc[d][k] = fmaf(-(nan ? cc : t), nan ? 1.f : t, acc[d][k]);
                 }
             } else {
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
-                    const float t0 = fmaf(aa[k], xx.x, -bb[k]);
-                    const float t1 = fmaf(aa[k], xx.y, -bb[k]);
-                    a0[k] = fmaf(-t0, t0, a0[k]);
-                    a1[k] = fmaf(-t1, t1, a1[k]);
+                    const float t = fmaf(q.x, xv[k], -q.y);
+                    acc[d][k] = fmaf(-t, t, acc[d][k]);
                 }
             }
         }
+    }
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
-            *reinterpret_cast<float2 *>(act + st.buf_out + (4 * q + k) * RT + m) =
-                make_float2(a0[k], a1[k]);
+    for (int d = 0; d < DPT; ++d)
+        *reinterpret_cast<float4 *>(act + st.buf_out + (d0 + d) * RT + mq) =
+            make_float4(acc[d][0], acc[d][1], acc[d][2], acc[d][3]);
+}
+
+template <bool MARG>
+__device__ void leaf_step(const LStep &st, float *act, const float *xs, const float *prm, int tid) {
+    switch (st.n_out >> 3) {
+        case 1: leaf_step_t<1, MARG>(st, act, xs, prm, tid); break;
+        case 2: leaf_step_t<2, MARG>(st, act, xs, prm, tid); break;
+        case 3: leaf_step_t<3, MARG>(st, act, xs, prm, tid); break;
+        case 4: leaf_step_t<4, MARG>(st, act, xs, prm, tid); break;
+        case 5: leaf_step_t<5, MARG>(st, act, xs, prm, tid); break;
+        case 6: leaf_step_t<6, MARG>(st, act, xs, prm, tid); break;
+        case 7: leaf_step_t<7, MARG>(st, act, xs, prm, tid); break;
+        case 8: leaf_step_t<8, MARG>(st, act, xs, prm, tid); break;
     }
 }
 
@@ -233,8 +251,10 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     float *sa = reinterpret_cast<float *>(smem + off);
     float *sb = sa + RT;
     off += 2 * RT * 4;
-    float *xsb = reinterpret_cast<float *>(smem + off);  // [2][max_vars][RT]
-    off += 2 * (size_t)p.max_vars * RT * 4;
+    // leaf staging, 2 buffers of [max_vars][RT] x rows + [max_leaf_params] params
+    const size_t stage_floats = (size_t)p.max_vars * RT + (size_t)p.max_leaf_params;
+    float *xsb = reinterpret_cast<float *>(smem + off);
+    off += 2 * stage_floats * 4;
     off = (off + 1023) & ~(size_t)1023;
     uint8_t *aimg = smem + off;  // [2][RT x kpad] f16 (hi, lo)
     const size_t aimg_part = (size_t)RT * p.max_kpad * 2;
@@ -265,9 +285,11 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     // x rows of a leaf step for the tile at `base` -> buffer b (one thread)
     auto issue_x = [&](int step, int64_t base, int b) {
         const LStep &ls = p.steps[step];
-        const uint32_t dst = r_smem(xsb + (size_t)b * p.max_vars * RT);
+        const uint32_t dst = r_smem(xsb + (size_t)b * stage_floats);
         const uint32_t bar = bar_x0 + 8 * b;
-        mbar_expect_tx(bar, (uint32_t)ls.n_vars * RT * 4);
+        const uint32_t pbytes = (uint32_t)ls.w_off * 4;
+        mbar_expect_tx(bar, (uint32_t)ls.n_vars * RT * 4 + pbytes);
+        bulk_g2s(dst + (uint32_t)p.max_vars * RT * 4, p.fparams + ls.par_off, pbytes, bar);
         for (int v = 0; v < ls.n_vars; ++v) {
             const int f = __ldg(p.vars + ls.vars_off + v);
             bulk_g2s(dst + v * RT * 4, p.xT + (int64_t)f * p.ldT + base, RT * 4, bar);
@@ -301,7 +323,10 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                         issue_x(p.first_leaf, base + (int64_t)gridDim.x * RT, b ^ 1);
                 }
                 xbuf ^= 1;
-                leaf_step<MARG>(st, p, act, xsb + (size_t)b * p.max_vars * RT, tid);
+                {
+                    const float *stg = xsb + (size_t)b * stage_floats;
+                    leaf_step<MARG>(st, act, stg, stg + (size_t)p.max_vars * RT, tid);
+                }
                 __syncthreads();
                 continue;
             }
@@ -450,9 +475,9 @@ __global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64
 }
 
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
-                      int max_vars) {
+                      int max_vars, int max_leaf_params) {
     size_t off = 128 + (size_t)smem_floats * 4 + (size_t)C * RT * 4 + (size_t)max_na * RT * 4 +
-                 2 * RT * 4 + 2 * (size_t)max_vars * RT * 4;
+                 2 * RT * 4 + 2 * ((size_t)max_vars * RT + (size_t)max_leaf_params) * 4;
     off = (off + 1023) & ~(size_t)1023;
     off += 2 * (size_t)RT * max_kpad * 2;
     off = (off + 1023) & ~(size_t)1023;

@@ -30,7 +30,8 @@ def emulate_layered(plan: dict, x: np.ndarray, n_roots: int, marginal: bool = Fa
             if t == 0:
                 I, V = int(st["n_out"]), int(st["n_vars"])
                 ab = fp[int(st["par_off"]):int(st["par_off"]) + V * I * 2].reshape(V, I, 2)
-                cv = fp[int(st["w_off"]):int(st["w_off"]) + V * I].reshape(V, I)
+                # per-(v, i) c = log2(a) + 0.5 log2(ln2/pi) (= -log2(sigma sqrt(2 pi)))
+                cv = np.log2(ab[:, :, 0]) + 0.5 * np.log2(np.log(2.0) / np.pi)
                 acc = np.tile(fp[int(st["cst_off"]):int(st["cst_off"]) + I][:, None], (1, N))
                 for v in range(V):
                     xv = xd[:, int(vars_[int(st["vars_off"]) + v])]

@@ -252,7 +252,7 @@ def test_layered_detection_accepts_rat_rejects_others():
         assert p is None and why
 
 
-@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 12, 5), (24, 1, 1, 4, 4, 2)])
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (24, 1, 1, 4, 8, 2)])
 def test_layered_plan_matches_oracle(shape):
     from spn_inputs import rat_spn
     from tests.layered_emulator import emulate_layered

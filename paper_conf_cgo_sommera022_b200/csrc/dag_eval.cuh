@@ -341,16 +341,19 @@ __device__ __forceinline__ void h_slp(float (&r)[D][K], uint32_t counts, float b
     }
 }
 
-// Straight-line product of exactly N Gaussian leaves (parameter records at pp).
+// Straight-line product of exactly N Gaussian leaves.  The header carries the
+// leaves' feature offsets (16 bits each, fo), so the feature loads are issued
+// together with the parameter loads (records at pp: {-, a, b, c}).
 template <int S, bool ACC, int N, int D, int K, bool MARG, bool XS>
-__device__ __forceinline__ void h_gprod(float (&r)[D][K], float C, uint32_t pp,
-                                        const Env<K, MARG, XS> &e) {
+__device__ __forceinline__ void h_gprod(float (&r)[D][K], float C, uint32_t fo01, uint32_t fo23,
+                                        uint32_t pp, const Env<K, MARG, XS> &e) {
+    const uint32_t fo[4] = {fo01 & 0xffffu, fo01 >> 16, fo23 & 0xffffu, fo23 >> 16};
+    float xv[N][K];
+#pragma unroll
+    for (int i = 0; i < N; ++i) e.loadx(fo[i], xv[i]);
     uint32_t f[N], ya[N], zb[N], wc[N];
 #pragma unroll
     for (int i = 0; i < N; ++i) lds4(pp + 16 * i, f[i], ya[i], zb[i], wc[i]);
-    float xv[N][K];
-#pragma unroll
-    for (int i = 0; i < N; ++i) e.loadx(f[i], xv[i]);
     float acc[K];
     if constexpr (ACC) {
         FOR_K acc[j] = r[S - 1][j] + C;
@@ -568,9 +571,9 @@ __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
 #define SPN_GPROD_BODY(S, ACC, N)                                                \
     {                                                                            \
         const float C = __uint_as_float(cy);                                     \
-        const uint32_t pp = pc + 16;                                             \
+        const uint32_t fo01 = cz, fo23 = cw, pp = pc + 16;                       \
         SPN_NEXT(pc + 16 * (N + 1))                                              \
-        h_gprod<S, ACC, N>(r, C, pp, e);                                         \
+        h_gprod<S, ACC, N>(r, C, fo01, fo23, pp, e);                             \
     }
 #define SPN_BODY_15(S) SPN_GPROD_BODY(SPN_SS(S), false, 1)
 #define SPN_BODY_16(S) SPN_GPROD_BODY(SPN_SS(S), false, 2)

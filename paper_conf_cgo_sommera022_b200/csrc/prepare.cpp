@@ -616,8 +616,19 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             }
         }
         if (!acc) max_sp = std::max<int64_t>(max_sp, sp + 1);
-        if (nd == 0 && ng >= 1 && ng <= 4)  // straight-line variants
-            rec_of((acc ? OP_GACC1 : OP_GPUSH1) + ng - 1, acc ? sp + 1 : sp, 0, fbits((float)C));
+        bool packable = nd == 0 && ng >= 1 && ng <= 4;
+        uint32_t fo[4] = {0, 0, 0, 0};
+        if (packable) {
+            int k = 0;
+            for (int64_t u : lv) {
+                const uint32_t f = feat_arg(leaf[u].f);
+                if (f > 0xffffu) packable = false;
+                fo[k++] = f;
+            }
+        }
+        if (packable)  // straight-line variants, feature offsets in the header
+            rec_of((acc ? OP_GACC1 : OP_GPUSH1) + ng - 1, acc ? sp + 1 : sp, 0, fbits((float)C),
+                   fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16));
         else
             rec_of(acc ? OP_LACC : OP_LPUSH, acc ? sp + 1 : sp, ng, fbits((float)C), nd);
         for (int pass = 0; pass < 2; ++pass)

@@ -15,7 +15,9 @@
 //
 //   LPUSH  ng | C, nd        r[sp]   = C + sum of ng Gaussian + nd discrete leaves
 //   LACC   ng | C, nd        r[sp-1] += (same)          (leaf children of a product)
-//   GPUSHn / GACCn  | C      same for exactly n <= 4 Gaussian leaves (no loop)
+//   GPUSHn / GACCn  | C, f0|f1<<16, f2|f3<<16   same for exactly n <= 4 Gaussian
+//                            leaves (no loop); the 16-bit feature offsets of the
+//                            leaves ride in the header so x loads issue at once
 //   SLPk  counts | bias, C0, C1   r[sp] = LSE_c(C_c + sum of n_c Gaussian leaves) + bias
 //       for k = 2..4 children (n_c in 1..7 packed 3 bits each in arg); for k >= 3
 //       a record {C2, C3} follows, then the children's parameter records.

@@ -45,9 +45,10 @@ struct RParams {
     int32_t max_vars;
     int32_t first_leaf;
     int32_t max_leaf_params;
+    int32_t wbufs;
 };
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
-                      int max_vars, int max_leaf_params);
+                      int max_vars, int max_leaf_params, int prec, int wbufs);
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st);
@@ -107,7 +108,7 @@ struct DevicePlan {
     int64_t chunk = 0;
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
-    int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0;
+    int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
     spn_plan_stats stats;
 };
 
@@ -226,6 +227,7 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         rp.max_vars = P.max_vars;
         rp.first_leaf = P.first_leaf;
         rp.max_leaf_params = P.max_leaf_params;
+        rp.wbufs = P.wbufs;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
@@ -326,8 +328,8 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
 bool valid_graph_handle(const spn_handle *h) { return h && h->magic == H_GRAPH && h->graph; }
 
 int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare_options &opt,
-                    int dev, int sms, size_t smem, std::chrono::steady_clock::time_point t0,
-                    spn_handle **out_plan) {
+                    int dev, int sms, size_t smem, int wbufs,
+                    std::chrono::steady_clock::time_point t0, spn_handle **out_plan) {
     DevicePlan *P = new (std::nothrow) DevicePlan();
     if (!P) return set_err(SPN_E_OOM, "plan");
     P->device = dev;
@@ -347,6 +349,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     P->max_vars = lp.max_vars;
     P->first_leaf = lp.first_leaf;
     P->max_leaf_params = lp.max_leaf_params;
+    P->wbufs = wbufs;
     // transposed-feature scratch: chunks small enough (<= ~48 MB) that the
     // tile slices re-read by every repetition stay resident in L2
     // (a multiple of one full wave of 128-sample tiles: 148 SMs x 128)
@@ -498,19 +501,27 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     // ---- layered (RAT-SPN) tensor-core path ----
     if (opt.layered_path != 1) {
         LayeredPlan lp;
-        detect_layered(g, lp);
         size_t lsmem = 0;
-        if (lp.ok) {
+        int wbufs = 0;
+        const int prec = opt.tc_precision == 1 ? 1 : 3;
+        // prefer double-buffered weight groups (N <= 240, else N <= 120 per
+        // group), then serial groups
+        for (int attempt = 0; attempt < 3 && wbufs == 0; ++attempt) {
+            const int n_cap = attempt == 1 ? 120 : 240;
+            const int wb = attempt == 2 ? 1 : 2;
+            detect_layered(g, lp, n_cap);
+            if (!lp.ok) break;
             lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup,
-                                   lp.max_vars, lp.max_leaf_params);
-            if (lsmem > (size_t)smem_optin) {
-                lp.ok = false;
-                lp.why = "activations do not fit in shared memory";
-            }
+                                   lp.max_vars, lp.max_leaf_params, prec, wb);
+            if (lsmem <= (size_t)smem_optin) wbufs = wb;
+        }
+        if (lp.ok && wbufs == 0) {
+            lp.ok = false;
+            lp.why = "activations do not fit in shared memory";
         }
         if (!lp.ok && opt.layered_path == 2)
             return set_err(SPN_E_UNSUPPORTED, "layered path not applicable: " + lp.why);
-        if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, t0, out_plan);
+        if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, wbufs, t0, out_plan);
     }
     int K = opt.samples_per_thread ? opt.samples_per_thread : 4;
     if (K != 1 && K != 2 && K != 4 && K != 8)

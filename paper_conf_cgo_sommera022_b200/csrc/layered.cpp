@@ -94,7 +94,7 @@ struct Partition {
 
 }  // namespace
 
-void detect_layered(const GraphData &g, LayeredPlan &plan) {
+void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
     plan = LayeredPlan();
     CGraph c;
     canonicalise(g, c);
@@ -304,7 +304,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan) {
         st.nb = nb;
         st.n_out = S;
         st.k_pad = (nb + 15) / 16 * 16;
-        st.s_per_group = std::max(1, std::min(S, 240 / na));
+        st.s_per_group = std::max(1, std::min(S, n_cap / na));
         st.n_groups = (S + st.s_per_group - 1) / st.s_per_group;
         st.n_group = (st.s_per_group * na + 15) / 16 * 16;
         st.w_group_bytes = (int64_t)st.n_group * st.k_pad * 2;

@@ -62,6 +62,7 @@ struct LayeredPlan {
 };
 
 // Detects the structure; on success fills plan (ok = true).
-void detect_layered(const GraphData &g, LayeredPlan &plan);
+// n_cap: largest N (columns) of one MMA group (<= 240).
+void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap = 240);
 
 }  // namespace spnb

@@ -49,11 +49,12 @@ struct RParams {
     int32_t max_vars;   // largest leaf region (staged x rows)
     int32_t first_leaf; // index of the first LEAF step
     int32_t max_leaf_params;  // floats of the largest staged leaf parameter block
+    int32_t wbufs;      // 2: double-buffered weight groups + TMEM ping-pong; 1: serial
 };
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
 constexpr int RTH = 256;  // threads per CTA
-constexpr uint32_t TMEM_COLS = 256;
+constexpr uint32_t TMEM_BUF = 256;  // columns per accumulator buffer
 
 __device__ __forceinline__ float r_ex2(float x) {
     float y;
@@ -239,7 +240,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1 w, 2/3 x
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1/2 w, 3/4 x
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 64);
     size_t off = 128;
     float *act = reinterpret_cast<float *>(smem + off);
@@ -260,18 +261,21 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     const size_t aimg_part = (size_t)RT * p.max_kpad * 2;
     off += 2 * aimg_part;
     off = (off + 1023) & ~(size_t)1023;
-    uint8_t *wsm = smem + off;   // [2][n_group x kpad] f16 (hi, lo)
+    uint8_t *wsm = smem + off;   // [wbufs][prec==3 ? 2 : 1][n_group x kpad] f16
+    const size_t w_part = (size_t)p.max_ngroup * p.max_kpad * 2;
+    const size_t w_buf = w_part * (p.prec == 3 ? 2 : 1);
+    const uint32_t tmem_cols = p.wbufs == 2 ? 2 * TMEM_BUF : TMEM_BUF;
 
-    const uint32_t bar_mma = r_smem(bars), bar_w = r_smem(bars + 1);
-    const uint32_t bar_x0 = r_smem(bars + 2);
+    const uint32_t bar_mma = r_smem(bars), bar_w0 = r_smem(bars + 1);
+    const uint32_t bar_x0 = r_smem(bars + 3);
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                          r_smem(tmem_slot)),
-                     "r"(TMEM_COLS));
+                     "r"(tmem_cols));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     if (tid == 0) {
-        for (int i = 0; i < 4; ++i)
+        for (int i = 0; i < 5; ++i)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(r_smem(bars + i)), "r"(1));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -279,45 +283,50 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
-    uint32_t ph_mma = 0, ph_w = 0, ph_x[2] = {0, 0};
+    uint32_t ph_mma = 0, ph_w[2] = {0, 0}, ph_x[2] = {0, 0};
     int xbuf = 0;  // buffer of the next leaf step
 
-    // x rows of a leaf step for the tile at `base` -> buffer b (one thread)
+    // x rows + parameter block of a leaf step for the tile at `base` -> buffer
+    // b; issued by the lanes of warp 0 (one bulk copy per lane)
     auto issue_x = [&](int step, int64_t base, int b) {
         const LStep &ls = p.steps[step];
+        const int nv = ls.n_vars;
         const uint32_t dst = r_smem(xsb + (size_t)b * stage_floats);
         const uint32_t bar = bar_x0 + 8 * b;
         const uint32_t pbytes = (uint32_t)ls.w_off * 4;
-        mbar_expect_tx(bar, (uint32_t)ls.n_vars * RT * 4 + pbytes);
-        bulk_g2s(dst + (uint32_t)p.max_vars * RT * 4, p.fparams + ls.par_off, pbytes, bar);
-        for (int v = 0; v < ls.n_vars; ++v) {
+        if (lane == 0) {
+            mbar_expect_tx(bar, (uint32_t)nv * RT * 4 + pbytes);
+            bulk_g2s(dst + (uint32_t)p.max_vars * RT * 4, p.fparams + ls.par_off, pbytes, bar);
+        }
+        __syncwarp();
+        for (int v = lane; v < nv; v += 32) {
             const int f = __ldg(p.vars + ls.vars_off + v);
             bulk_g2s(dst + v * RT * 4, p.xT + (int64_t)f * p.ldT + base, RT * 4, bar);
         }
     };
-    auto issue_w = [&](const LStep &ws, int g) {
+    auto issue_w = [&](const LStep &ws, int g, int b) {  // one thread
         const size_t gb = (size_t)ws.w_group_bytes;
         const uint8_t *src = p.wimg + ws.w_off + 2 * gb * g;
-        mbar_expect_tx(bar_w, (uint32_t)(gb * (p.prec == 3 ? 2 : 1)));
-        bulk_g2s(r_smem(wsm), src, (uint32_t)gb, bar_w);
-        if (p.prec == 3)
-            bulk_g2s(r_smem(wsm) + (uint32_t)((size_t)p.max_ngroup * p.max_kpad * 2), src + gb,
-                     (uint32_t)gb, bar_w);
+        const uint32_t bar = bar_w0 + 8 * b;
+        const uint32_t dst = r_smem(wsm) + (uint32_t)(b * w_buf);
+        mbar_expect_tx(bar, (uint32_t)(gb * (p.prec == 3 ? 2 : 1)));
+        bulk_g2s(dst, src, (uint32_t)gb, bar);
+        if (p.prec == 3) bulk_g2s(dst + (uint32_t)w_part, src + gb, (uint32_t)gb, bar);
     };
 
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    if (tid == 0 && (int64_t)blockIdx.x < n_tiles) issue_x(p.first_leaf, (int64_t)blockIdx.x * RT, 0);
+    if (warp == 0 && (int64_t)blockIdx.x < n_tiles) issue_x(p.first_leaf, (int64_t)blockIdx.x * RT, 0);
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const int64_t base = tile * RT;
         for (int i = tid; i < p.C * RT; i += RTH) racc[i] = -CUDART_INF_F;
         __syncthreads();
         for (int si = 0; si < p.n_steps; ++si) {
-            const LStep &st = p.steps[si];
+            const LStep st = p.steps[si];  // by value: fields live in registers
             if (st.type == 0) {
                 const int b = xbuf;
                 mbar_wait(bar_x0 + 8 * b, ph_x[b]);
                 ph_x[b] ^= 1;
-                if (tid == 0) {  // prefetch the next leaf step's rows (maybe next tile)
+                if (warp == 0) {  // prefetch the next leaf step's rows (maybe next tile)
                     if (st.rep >= 0) issue_x(st.rep, base, b ^ 1);
                     else if (tile + gridDim.x < n_tiles)
                         issue_x(p.first_leaf, base + (int64_t)gridDim.x * RT, b ^ 1);
@@ -331,7 +340,11 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 continue;
             }
             // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
-            if (tid == 0) issue_w(st, 0);
+            const int G = st.n_groups;
+            if (tid == 0) {
+                issue_w(st, 0, 0);
+                if (p.wbufs == 2 && G > 1) issue_w(st, 1, 1);
+            }
             const int na = st.na, nb = st.nb, kpad = st.k_pad;
             if (tid < RT) {
                 const int m = tid;
@@ -365,34 +378,9 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             const uint32_t idesc = (1u << 4) | ((uint32_t)(st.n_group >> 3) << 17) |
                                    ((uint32_t)(RT >> 4) << 24);
             const uint32_t a_hi = r_smem(aimg), a_lo = a_hi + (uint32_t)aimg_part;
-            const uint32_t w_hi = r_smem(wsm),
-                           w_lo = w_hi + (uint32_t)((size_t)p.max_ngroup * p.max_kpad * 2);
-            for (int g = 0; g < st.n_groups; ++g) {
-                mbar_wait(bar_w, ph_w);
-                ph_w ^= 1;
-                if (tid == 0) {
-                    fence_after();
-                    for (int kk = 0; kk < kpad / 16; ++kk) {
-                        const uint32_t ka = kk * 2 * lbo_a, kb = kk * 2 * lbo_b;
-                        umma_f16(tmem, umma_desc(a_hi + ka, lbo_a, 128), umma_desc(w_hi + kb, lbo_b, 128),
-                                 idesc, kk > 0);
-                        if (p.prec == 3) {
-                            umma_f16(tmem, umma_desc(a_lo + ka, lbo_a, 128),
-                                     umma_desc(w_hi + kb, lbo_b, 128), idesc, 1);
-                            umma_f16(tmem, umma_desc(a_hi + ka, lbo_a, 128),
-                                     umma_desc(w_lo + kb, lbo_b, 128), idesc, 1);
-                        }
-                    }
-                    umma_commit(bar_mma);
-                }
-                __syncwarp();
-                mbar_wait(bar_mma, ph_mma);
-                ph_mma ^= 1;
-                fence_after();
-                // the MMA has consumed the weights: fetch the next group's now,
-                // overlapping the copy with this group's epilogue
-                if (tid == 0 && g + 1 < st.n_groups) issue_w(st, g + 1);
-                // epilogue: warp quarter q reads TMEM lanes 32q..32q+31 (= samples)
+            // epilogue of group g from TMEM buffer tb: warp quarter q reads
+            // lanes 32q..32q+31 (= samples); the two warp halves split the sums
+            auto epilogue = [&](int g, uint32_t tb) {
                 const int qd = warp & 3, half = warp >> 2;
                 const int m = qd * 32 + lane;
                 const int s0 = g * st.s_per_group;
@@ -402,7 +390,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 const float shift = sa[m] + sb[m];
                 for (int sl = sl0; sl < sl1; ++sl) {
                     float acc = 0.f;
-                    const uint32_t trow = tmem + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
+                    const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
                     int c0 = 0;
                     for (; c0 + 8 <= na; c0 += 8) {
                         float t[8];
@@ -427,6 +415,43 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                         racc[col * RT + m] = r_lse2(racc[col * RT + m], val);
                     }
                 }
+            };
+            for (int g = 0; g < G; ++g) {
+                const int wb = p.wbufs == 2 ? (g & 1) : 0;
+                const uint32_t tb = p.wbufs == 2 ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
+                mbar_wait(bar_w0 + 8 * wb, ph_w[wb]);
+                ph_w[wb] ^= 1;
+                if (tid == 0) {
+                    fence_after();
+                    const uint32_t w_hi = r_smem(wsm) + (uint32_t)(wb * w_buf);
+                    const uint32_t w_lo = w_hi + (uint32_t)w_part;
+                    for (int kk = 0; kk < kpad / 16; ++kk) {
+                        const uint32_t ka = kk * 2 * lbo_a, kb = kk * 2 * lbo_b;
+                        umma_f16(tmem + tb, umma_desc(a_hi + ka, lbo_a, 128),
+                                 umma_desc(w_hi + kb, lbo_b, 128), idesc, kk > 0);
+                        if (p.prec == 3) {
+                            umma_f16(tmem + tb, umma_desc(a_lo + ka, lbo_a, 128),
+                                     umma_desc(w_hi + kb, lbo_b, 128), idesc, 1);
+                            umma_f16(tmem + tb, umma_desc(a_hi + ka, lbo_a, 128),
+                                     umma_desc(w_lo + kb, lbo_b, 128), idesc, 1);
+                        }
+                    }
+                    umma_commit(bar_mma);
+                }
+                __syncwarp();
+                // overlap: the previous group's epilogue runs under this MMA
+                if (p.wbufs == 2 && g > 0) epilogue(g - 1, (uint32_t)((g - 1) & 1) * TMEM_BUF);
+                mbar_wait(bar_mma, ph_mma);
+                ph_mma ^= 1;
+                fence_after();
+                // the MMA has consumed weight buffer wb: refill it
+                if (tid == 0 && g + p.wbufs < G) issue_w(st, g + p.wbufs, wb);
+                if (p.wbufs == 1) epilogue(g, 0u);
+                fence_before();
+                __syncthreads();
+            }
+            if (p.wbufs == 2) {
+                epilogue(G - 1, (uint32_t)((G - 1) & 1) * TMEM_BUF);
                 fence_before();
                 __syncthreads();
             }
@@ -454,7 +479,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     __syncthreads();
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
-                     "r"(TMEM_COLS));
+                     "r"(tmem_cols));
 }
 
 // xT[f][s] = x[s][f] for s < n (zero for n <= s < rows_pad)
@@ -475,13 +500,13 @@ __global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64
 }
 
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
-                      int max_vars, int max_leaf_params) {
+                      int max_vars, int max_leaf_params, int prec, int wbufs) {
     size_t off = 128 + (size_t)smem_floats * 4 + (size_t)C * RT * 4 + (size_t)max_na * RT * 4 +
                  2 * RT * 4 + 2 * ((size_t)max_vars * RT + (size_t)max_leaf_params) * 4;
     off = (off + 1023) & ~(size_t)1023;
     off += 2 * (size_t)RT * max_kpad * 2;
     off = (off + 1023) & ~(size_t)1023;
-    off += 2 * (size_t)max_ngroup * max_kpad * 2;
+    off += (size_t)wbufs * (prec == 3 ? 2 : 1) * (size_t)max_ngroup * max_kpad * 2;
     return off + 1024;  // alignment slack for the dynamic base
 }
 

@@ -341,6 +341,45 @@ __device__ __forceinline__ void h_slp(float (&r)[D][K], uint32_t counts, float b
     }
 }
 
+// Straight-line fused sum over KC children of 2 Gaussian leaves each.
+template <int S, int KC, int D, int K, bool MARG, bool XS>
+__device__ __forceinline__ void h_slpu(float (&r)[D][K], float bias, const float (&Cs)[4],
+                                       const uint32_t (&fo)[6], uint32_t pp,
+                                       const Env<K, MARG, XS> &e) {
+    constexpr int NL = 2 * KC;
+    float xv[NL][K];
+#pragma unroll
+    for (int i = 0; i < NL; ++i) e.loadx(fo[i], xv[i]);
+    uint32_t f[NL], ya[NL], zb[NL], wc[NL];
+#pragma unroll
+    for (int i = 0; i < NL; ++i) lds4(pp + 16 * i, f[i], ya[i], zb[i], wc[i]);
+    float v[KC][K];
+#pragma unroll
+    for (int c = 0; c < KC; ++c) {
+        FOR_K v[c][j] = Cs[c];
+#pragma unroll
+        for (int l = 0; l < 2; ++l) {
+            const int i = 2 * c + l;
+            const float a = __uint_as_float(ya[i]), b = __uint_as_float(zb[i]);
+            FOR_K {
+                const float t = fmaf(a, xv[i][j], -b);
+                if constexpr (MARG) {
+                    const bool nan = xv[i][j] != xv[i][j];
+                    v[c][j] = fmaf(-(nan ? __uint_as_float(wc[i]) : t), nan ? 1.f : t, v[c][j]);
+                } else {
+                    v[c][j] = fmaf(-t, t, v[c][j]);
+                }
+            }
+        }
+    }
+    FOR_K {
+        float w[KC];
+#pragma unroll
+        for (int c = 0; c < KC; ++c) w[c] = v[c][j];
+        r[S][j] = lse_vals<KC>(w, bias);
+    }
+}
+
 // Straight-line product of exactly N Gaussian leaves.  The header carries the
 // leaves' feature offsets (16 bits each, fo), so the feature loads are issued
 // together with the parameter loads (records at pp: {-, a, b, c}).
@@ -462,7 +501,8 @@ __device__ __forceinline__ void h_out(float (&r)[D][K], uint32_t root,
 __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
     if (sp > D) return false;
     return (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
-            (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4))
+            (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4) ||
+            op == OP_SLPU2 || op == OP_SLPU3)
                ? (sp >= 0 && sp < D)
            : (op == OP_LACC || op == OP_LSE1 || op == OP_STS || op == OP_STG || op == OP_OUT ||
               (op >= OP_GACC1 && op <= OP_GACC4))
@@ -608,7 +648,34 @@ __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
 #define SPN_BODY_23(S) SPN_SLP_BODY(S, 2)
 #define SPN_BODY_24(S) SPN_SLP_BODY(S, 3)
 #define SPN_BODY_25(S) SPN_SLP_BODY(S, 4)
-#define SPN_UNUSED_CASES case 442: case 443: case 444: case 445: case 446: case 447: case 448: case 449: case 450: case 451: case 452: case 453: case 454: case 455: case 456: case 457: case 458: case 459: case 460: case 461: case 462: case 463: case 464: case 465: case 466: case 467: case 468: case 469: case 470: case 471: case 472: case 473: case 474: case 475: case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
+#define SPN_SLPU_BODY(S, KC)                                                     \
+    {                                                                            \
+        const float bias = __uint_as_float(cy);                                  \
+        float Cs[4];                                                             \
+        Cs[0] = __uint_as_float(cz);                                             \
+        Cs[1] = __uint_as_float(cw);                                             \
+        uint32_t ex, ey, ez, ew;                                                 \
+        lds4(pc + 16, ex, ey, ez, ew);                                           \
+        uint32_t fo[6];                                                          \
+        if (KC == 2) {                                                           \
+            fo[0] = ex & 0xffffu; fo[1] = ex >> 16;                              \
+            fo[2] = ey & 0xffffu; fo[3] = ey >> 16;                              \
+            fo[4] = 0; fo[5] = 0;                                                \
+            Cs[2] = 0.f;                                                         \
+        } else {                                                                 \
+            Cs[2] = __uint_as_float(ex);                                         \
+            fo[0] = ey & 0xffffu; fo[1] = ey >> 16;                              \
+            fo[2] = ez & 0xffffu; fo[3] = ez >> 16;                              \
+            fo[4] = ew & 0xffffu; fo[5] = ew >> 16;                              \
+        }                                                                        \
+        Cs[3] = 0.f;                                                             \
+        const uint32_t pp = pc + 32;                                             \
+        SPN_NEXT(pp + 16 * 2 * KC)                                               \
+        h_slpu<SPN_SS(S), KC>(r, bias, Cs, fo, pp, e);                           \
+    }
+#define SPN_BODY_26(S) SPN_SLPU_BODY(S, 2)
+#define SPN_BODY_27(S) SPN_SLPU_BODY(S, 3)
+#define SPN_UNUSED_CASES case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
 
 // Run one task's program (shared memory at byte address prog) for this
 // thread's K samples.  All case labels 0..511 exist, so the dispatch is one
@@ -649,6 +716,8 @@ __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &
             SPN_ALL_SP(SPN_CASE, 23)
             SPN_ALL_SP(SPN_CASE, 24)
             SPN_ALL_SP(SPN_CASE, 25)
+            SPN_ALL_SP(SPN_CASE, 26)
+            SPN_ALL_SP(SPN_CASE, 27)
             SPN_UNUSED_CASES
             default:
                 __builtin_unreachable();

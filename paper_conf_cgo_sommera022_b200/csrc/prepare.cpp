@@ -723,8 +723,26 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
                 lv.insert(lv.end(), cl.begin(), cl.end());
             }
             max_sp = std::max<int64_t>(max_sp, sp + 1);
-            rec_of(OP_SLP2 + (uint32_t)(n - 2), sp, counts, fbits((float)bias), Cb[0], Cb[1]);
-            if (n >= 3) prog.push_back(Rec{Cb[2], Cb[3], 0, 0});
+            // straight-line form for children of exactly 2 leaves (n = 2, 3)
+            bool uni = (n == 2 || n == 3) && counts == (n == 2 ? 0x12u : 0x92u);
+            uint32_t fo[6] = {0, 0, 0, 0, 0, 0};
+            if (uni) {
+                for (size_t k = 0; k < lv.size(); ++k) {
+                    fo[k] = feat_arg(leaf[lv[k]].f);
+                    if (fo[k] > 0xffffu) uni = false;
+                }
+            }
+            if (uni && n == 2) {
+                rec_of(OP_SLPU2, sp, 0, fbits((float)bias), Cb[0], Cb[1]);
+                prog.push_back(Rec{fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16), 0, 0});
+            } else if (uni) {
+                rec_of(OP_SLPU3, sp, 0, fbits((float)bias), Cb[0], Cb[1]);
+                prog.push_back(Rec{Cb[2], fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16),
+                                   fo[4] | (fo[5] << 16)});
+            } else {
+                rec_of(OP_SLP2 + (uint32_t)(n - 2), sp, counts, fbits((float)bias), Cb[0], Cb[1]);
+                if (n >= 3) prog.push_back(Rec{Cb[2], Cb[3], 0, 0});
+            }
             for (int64_t l : lv) prog.push_back(Rec{feat_arg(leaf[l].f), leaf[l].y, leaf[l].z, leaf[l].w});
             return;
         }
@@ -799,6 +817,10 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             i += cs / NSP - OP_GPUSH1 + 1;
         else if (cs / NSP >= OP_GACC1 && cs / NSP <= OP_GACC4)
             i += cs / NSP - OP_GACC1 + 1;
+        else if (cs / NSP == OP_SLPU2 && cs < OP_COUNT * NSP)
+            i += 1 + 4;
+        else if (cs / NSP == OP_SLPU3 && cs < OP_COUNT * NSP)
+            i += 1 + 6;
         else if (cs / NSP >= OP_SLP2 && cs / NSP <= OP_SLP4 && cs < OP_COUNT * NSP) {
             const uint32_t cnt = prog[i].x >> CASE_BITS;
             i += (cs / NSP >= OP_SLP3 ? 1 : 0) + (cnt & 7u) + ((cnt >> 3) & 7u) +

@@ -21,6 +21,10 @@
 //   SLPk  counts | bias, C0, C1   r[sp] = LSE_c(C_c + sum of n_c Gaussian leaves) + bias
 //       for k = 2..4 children (n_c in 1..7 packed 3 bits each in arg); for k >= 3
 //       a record {C2, C3} follows, then the children's parameter records.
+//   SLPU2 | bias, C0, C1  + {f0|f1<<16, f2|f3<<16, -, -} + 4 leaf records
+//   SLPU3 | bias, C0, C1  + {C2, f0|f1<<16, f2|f3<<16, f4|f5<<16} + 6 leaf records
+//       straight-line forms of the dominant SLP shapes (children of 2 leaves),
+//       with the leaves' feature offsets up front so all loads issue at once.
 //       followed by ng Gaussian parameter records {f, a, b, c} and nd discrete
 //       records {f, table, lo, K}.  Gaussian: c - (a*x_f - b)^2 = log2 N(x; mu, s)
 //       with a = 1/(s sqrt(2 ln2)), b = a mu, c = -log2(s sqrt(2 pi)); the c's
@@ -68,7 +72,9 @@ enum Op : uint32_t {
     OP_SLP2 = 23,   // fused weighted sum of 2..4 Gaussian leaf products
     OP_SLP3 = 24,
     OP_SLP4 = 25,
-    OP_COUNT = 26
+    OP_SLPU2 = 26,  // straight-line SLP: 2 children x 2 Gaussian leaves
+    OP_SLPU3 = 27,  // straight-line SLP: 3 children x 2 Gaussian leaves
+    OP_COUNT = 28
 };
 
 constexpr int MAXD = 16;              // register stack depth

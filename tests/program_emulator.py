@@ -15,7 +15,7 @@ NSP = 17
 OPS = ["END", "LPUSH", "LACC", "ADD", "LSE1", "LSE2", "LSE3", "LSE4",
        "LDS", "LDG", "STS", "STG", "GLSE", "OUT", "NOP",
        "GPUSH1", "GPUSH2", "GPUSH3", "GPUSH4", "GACC1", "GACC2", "GACC3", "GACC4",
-       "SLP2", "SLP3", "SLP4"]
+       "SLP2", "SLP3", "SLP4", "SLPU2", "SLPU3"]
 SLOT_GLOBAL = 0x80000000
 SLOT_NONE = 0xFFFFFFFF
 
@@ -69,11 +69,19 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
             if op == "END":
                 break
             if op.startswith("SLP"):
-                k = int(op[3])
-                Cs = [_f32(r["z"]), _f32(r["w"])]
-                if k >= 3:
-                    Cs += [_f32(rec[pc]["x"]), _f32(rec[pc]["y"])]
-                    pc += 1
+                if op.startswith("SLPU"):
+                    k = int(op[4])
+                    Cs = [_f32(r["z"]), _f32(r["w"])]
+                    if k == 3:
+                        Cs.append(_f32(rec[pc]["x"]))
+                    pc += 1                   # feature-offset record (offsets repeat below)
+                    arg = 2 | (2 << 3) | ((2 << 6) if k == 3 else 0)
+                else:
+                    k = int(op[3])
+                    Cs = [_f32(r["z"]), _f32(r["w"])]
+                    if k >= 3:
+                        Cs += [_f32(rec[pc]["x"]), _f32(rec[pc]["y"])]
+                        pc += 1
                 vals = []
                 for ci in range(k):
                     acc = np.full(N, Cs[ci])

@@ -754,7 +754,7 @@ __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__r
 }
 
 template <int K, bool MARG, bool XS, int D>
-__global__ void __launch_bounds__(K == 8 ? 256 : (K == 4 ? 384 : 512)) dag_eval_kernel(const KParams p) {
+__global__ void __launch_bounds__(K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 512))) dag_eval_kernel(const KParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     constexpr int WT = 32 * K;
     Rec *prog_s = reinterpret_cast<Rec *>(smem_raw);
@@ -872,7 +872,7 @@ int dag_eval_occupancy_t(int block, size_t smem) {
 // maximum register-stack depth per samples-per-thread variant (registers:
 // D x K stack values per thread)
 template <int K>
-constexpr int stack_depth() { return K == 8 ? 10 : MAXD; }
+constexpr int stack_depth() { return (K == 8 || K == 2) ? 10 : MAXD; }
 
 #define SPNB_INSTANTIATE_K(K)                                                             \
     cudaError_t dag_eval_launch_k##K(const KParams &p, bool marg, bool xs, int grid,       \

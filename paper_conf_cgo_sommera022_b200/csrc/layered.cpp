@@ -305,6 +305,8 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
         st.n_out = S;
         st.k_pad = (nb + 15) / 16 * 16;
         st.s_per_group = std::max(1, std::min(S, n_cap / na));
+        // an even number of sums per group balances the two epilogue warp halves
+        if (st.s_per_group > 1 && st.s_per_group < S && (st.s_per_group & 1)) st.s_per_group -= 1;
         st.n_groups = (S + st.s_per_group - 1) / st.s_per_group;
         st.n_group = (st.s_per_group * na + 15) / 16 * 16;
         st.w_group_bytes = (int64_t)st.n_group * st.k_pad * 2;

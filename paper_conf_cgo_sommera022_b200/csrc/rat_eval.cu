@@ -283,7 +283,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
-    uint32_t ph_mma = 0, ph_w[2] = {0, 0}, ph_x[2] = {0, 0};
+    uint32_t ph_mma = 0, ph_w = 0, ph_x = 0;  // phase parity bits (bit b: buffer b)
     int xbuf = 0;  // buffer of the next leaf step
 
     // x rows + parameter block of a leaf step for the tile at `base` -> buffer
@@ -324,8 +324,8 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             const LStep st = p.steps[si];  // by value: fields live in registers
             if (st.type == 0) {
                 const int b = xbuf;
-                mbar_wait(bar_x0 + 8 * b, ph_x[b]);
-                ph_x[b] ^= 1;
+                mbar_wait(bar_x0 + 8 * b, (ph_x >> b) & 1u);
+                ph_x ^= 1u << b;
                 if (warp == 0) {  // prefetch the next leaf step's rows (maybe next tile)
                     if (st.rep >= 0) issue_x(st.rep, base, b ^ 1);
                     else if (tile + gridDim.x < n_tiles)
@@ -419,8 +419,8 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             for (int g = 0; g < G; ++g) {
                 const int wb = p.wbufs == 2 ? (g & 1) : 0;
                 const uint32_t tb = p.wbufs == 2 ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
-                mbar_wait(bar_w0 + 8 * wb, ph_w[wb]);
-                ph_w[wb] ^= 1;
+                mbar_wait(bar_w0 + 8 * wb, (ph_w >> wb) & 1u);
+                ph_w ^= 1u << wb;
                 if (tid == 0) {
                     fence_after();
                     const uint32_t w_hi = r_smem(wsm) + (uint32_t)(wb * w_buf);

@@ -523,10 +523,14 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
             return set_err(SPN_E_UNSUPPORTED, "layered path not applicable: " + lp.why);
         if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, wbufs, t0, out_plan);
     }
-    int K = opt.samples_per_thread ? opt.samples_per_thread : 4;
+    // auto: K = 2 samples/thread with up to 24 warps when 16+ warps' feature
+    // tiles fit in shared memory (more warps hide the interpreter's latency),
+    // else K = 4 (measured on C2: K2x24 warps 0.733 ms vs K4x12 0.776 ms)
+    int K = opt.samples_per_thread ? opt.samples_per_thread
+                                   : ((size_t)g.F * 68 * 4 * 16 <= (size_t)170 * 1024 ? 2 : 4);
     if (K != 1 && K != 2 && K != 4 && K != 8)
         return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
-    const int max_block = K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 512));
+    const int max_block = K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 1024));
     int block = opt.block_threads ? opt.block_threads : max_block;
     if (block % 32 || block < 32 || block > max_block)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 within the kernel bound");
@@ -539,7 +543,7 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
 
     CodegenConfig cfg;
     cfg.K = K;
-    cfg.maxd = (K == 8 || K == 2) ? 10 : MAXD;
+    cfg.maxd = K == 4 ? MAXD : 10;
     cfg.x_in_smem = xs;
     cfg.tpw = tpw;
     cfg.max_task_ops = opt.max_task_nodes > 0 ? opt.max_task_nodes : -1;
@@ -713,7 +717,7 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
         return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
     CodegenConfig cfg;
     cfg.K = samples_per_thread;
-    cfg.maxd = (samples_per_thread == 8 || samples_per_thread == 2) ? 10 : MAXD;
+    cfg.maxd = samples_per_thread == 4 ? MAXD : 10;
     cfg.x_in_smem = x_in_smem != 0;
     cfg.tpw = 32 * cfg.K + 4;
     cfg.max_task_ops = max_task_ops;

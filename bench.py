@@ -350,7 +350,8 @@ def run_ours(args):
                                "dtype": "f16 (hi/lo split)" if args.tc_precision != 1 else "f16",
                                "peak_source": f"bf16_tflops ({src}); f16 dense rate = bf16"},
                     "hbm": hbm_part}
-        cpu = cpu_baseline(g, x, args.marginal) if world == 1 or True else None
+        # the oracle baseline is timed on rank 0 at N = 1 only (contract)
+        cpu = cpu_baseline(g, x, args.marginal) if world == 1 else None
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
                 "higher_is_better": True, "scaling": scaling, "vs_baseline": None,

@@ -41,11 +41,13 @@ def _nvcc():
 
 
 def _digest(paths, extra):
+    """Content hash of the sources/headers and the flags.  Absolute paths are
+    left out so a tree copied elsewhere (the GPU box) reuses its objects."""
     h = hashlib.sha256()
     for p in paths:
         with open(p, "rb") as f:
             h.update(f.read())
-    h.update(" ".join(extra).encode())
+    h.update(" ".join(a for a in extra if not os.path.isabs(a)).encode())
     return h.hexdigest()[:16]
 
 

@@ -3,6 +3,8 @@
 // launches and the host-buffer end-to-end pipeline.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -46,6 +48,7 @@ struct RParams {
     int32_t first_leaf;
     int32_t max_leaf_params;
     int32_t wbufs;
+    unsigned long long *prof;
 };
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
                       int max_vars, int max_leaf_params, int prec, int wbufs);
@@ -109,6 +112,7 @@ struct DevicePlan {
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
     int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
+    unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
     spn_plan_stats stats;
 };
 
@@ -162,6 +166,17 @@ void free_plan(DevicePlan *p) {
     cudaFree(p->d_wimg);
     cudaFree(p->d_root_map);
     cudaFree(p->d_xT);
+    if (p->d_prof) {
+        unsigned long long h[8];
+        if (cudaMemcpy(h, p->d_prof, sizeof(h), cudaMemcpyDeviceToHost) == cudaSuccess) {
+            const char *names[8] = {"leaf_wait", "leaf_compute", "leaf_barrier", "sum_phase1",
+                                    "w_wait", "mma_issue+epilogue", "mma_wait", "other"};
+            fprintf(stderr, "[spnb profile] cycles summed over CTAs:");
+            for (int k = 0; k < 8; ++k) fprintf(stderr, " %s=%llu", names[k], h[k]);
+            fprintf(stderr, "\n");
+        }
+        cudaFree(p->d_prof);
+    }
     for (int i = 0; i < 2; ++i) {
         if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
         cudaFree(p->hx[i]);
@@ -228,6 +243,7 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         rp.first_leaf = P.first_leaf;
         rp.max_leaf_params = P.max_leaf_params;
         rp.wbufs = P.wbufs;
+        rp.prof = P.d_prof;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
@@ -365,6 +381,8 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         free_plan(P);
         return rc;
     }
+    if (getenv("SPNB_PROFILE") && cudaMalloc(&P->d_prof, 8 * sizeof(unsigned long long)) == cudaSuccess)
+        cudaMemset(P->d_prof, 0, 8 * sizeof(unsigned long long));
     cudaError_t e = cudaMalloc(&P->d_xT, (size_t)g.F * chunk * 4);
     if (e != cudaSuccess) {
         free_plan(P);
@@ -530,7 +548,7 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
                                    : ((size_t)g.F * 68 * 4 * 16 <= (size_t)170 * 1024 ? 2 : 4);
     if (K != 1 && K != 2 && K != 4 && K != 8)
         return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
-    const int max_block = K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 1024));
+    const int max_block = K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 512));
     int block = opt.block_threads ? opt.block_threads : max_block;
     if (block % 32 || block < 32 || block > max_block)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 within the kernel bound");
@@ -543,7 +561,7 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
 
     CodegenConfig cfg;
     cfg.K = K;
-    cfg.maxd = K == 4 ? MAXD : 10;
+    cfg.maxd = (K == 8 || K == 2) ? 10 : MAXD;
     cfg.x_in_smem = xs;
     cfg.tpw = tpw;
     cfg.max_task_ops = opt.max_task_nodes > 0 ? opt.max_task_nodes : -1;
@@ -717,7 +735,7 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
         return set_err(SPN_E_ARG, "samples_per_thread must be 1, 2, 4 or 8");
     CodegenConfig cfg;
     cfg.K = samples_per_thread;
-    cfg.maxd = samples_per_thread == 4 ? MAXD : 10;
+    cfg.maxd = (samples_per_thread == 8 || samples_per_thread == 2) ? 10 : MAXD;
     cfg.x_in_smem = x_in_smem != 0;
     cfg.tpw = 32 * cfg.K + 4;
     cfg.max_task_ops = max_task_ops;

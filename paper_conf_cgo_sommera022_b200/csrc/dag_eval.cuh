@@ -341,19 +341,15 @@ __device__ __forceinline__ void h_slp(float (&r)[D][K], uint32_t counts, float b
     }
 }
 
-// Straight-line fused sum over KC children of 2 Gaussian leaves each, times
-// nt (0..2) tail leaves, pushed (ACC = false) or accumulated into r[S-1].
-template <int S, int KC, bool ACC, int D, int K, bool MARG, bool XS>
+// Straight-line fused sum over KC children of 2 Gaussian leaves each.
+template <int S, int KC, int D, int K, bool MARG, bool XS>
 __device__ __forceinline__ void h_slpu(float (&r)[D][K], float bias, const float (&Cs)[4],
-                                       const uint32_t (&fo)[8], uint32_t nt, uint32_t pp,
+                                       const uint32_t (&fo)[6], uint32_t pp,
                                        const Env<K, MARG, XS> &e) {
     constexpr int NL = 2 * KC;
     float xv[NL][K];
 #pragma unroll
     for (int i = 0; i < NL; ++i) e.loadx(fo[i], xv[i]);
-    float xt[2][K];
-    if (nt > 0) e.loadx(fo[6], xt[0]);
-    if (nt > 1) e.loadx(fo[7], xt[1]);
     uint32_t f[NL], ya[NL], zb[NL], wc[NL];
 #pragma unroll
     for (int i = 0; i < NL; ++i) lds4(pp + 16 * i, f[i], ya[i], zb[i], wc[i]);
@@ -376,34 +372,11 @@ __device__ __forceinline__ void h_slpu(float (&r)[D][K], float bias, const float
             }
         }
     }
-    float res[K];
     FOR_K {
         float w[KC];
 #pragma unroll
         for (int c = 0; c < KC; ++c) w[c] = v[c][j];
-        res[j] = lse_vals<KC>(w, bias);
-    }
-#pragma unroll
-    for (int l = 0; l < 2; ++l) {
-        if (nt > (uint32_t)l) {
-            uint32_t tf, ta, tb, tc;
-            lds4(pp + 16 * (NL + l), tf, ta, tb, tc);
-            const float a = __uint_as_float(ta), b = __uint_as_float(tb);
-            FOR_K {
-                const float t = fmaf(a, xt[l][j], -b);
-                if constexpr (MARG) {
-                    const bool nan = xt[l][j] != xt[l][j];
-                    res[j] = fmaf(-(nan ? __uint_as_float(tc) : t), nan ? 1.f : t, res[j]);
-                } else {
-                    res[j] = fmaf(-t, t, res[j]);
-                }
-            }
-        }
-    }
-    if constexpr (ACC) {
-        FOR_K r[S - 1][j] += res[j];
-    } else {
-        FOR_K r[S][j] = res[j];
+        r[S][j] = lse_vals<KC>(w, bias);
     }
 }
 
@@ -526,13 +499,13 @@ __device__ __forceinline__ void h_out(float (&r)[D][K], uint32_t root,
 // ---------------------------------------------------------------------------
 // Valid stack depths per op (sp = depth before the op).
 __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
-    return (sp > D) ? false
-           : (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
-              (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4) ||
-              op == OP_SLPU2 || op == OP_SLPU3)
+    if (sp > D) return false;
+    return (op == OP_LPUSH || op == OP_LDS || op == OP_LDG || op == OP_GLSE ||
+            (op >= OP_GPUSH1 && op <= OP_GPUSH4) || (op >= OP_SLP2 && op <= OP_SLP4) ||
+            op == OP_SLPU2 || op == OP_SLPU3)
                ? (sp >= 0 && sp < D)
            : (op == OP_LACC || op == OP_LSE1 || op == OP_STS || op == OP_STG || op == OP_OUT ||
-              (op >= OP_GACC1 && op <= OP_GACC4) || op == OP_SLPU2A || op == OP_SLPU3A)
+              (op >= OP_GACC1 && op <= OP_GACC4))
                ? (sp >= 1)
            : (op == OP_ADD || op == OP_LSE2) ? (sp >= 2)
            : (op == OP_LSE3) ? (sp >= 3)
@@ -675,45 +648,34 @@ __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
 #define SPN_BODY_23(S) SPN_SLP_BODY(S, 2)
 #define SPN_BODY_24(S) SPN_SLP_BODY(S, 3)
 #define SPN_BODY_25(S) SPN_SLP_BODY(S, 4)
-#define SPN_SLPU_BODY(S, KC, ACC)                                                \
+#define SPN_SLPU_BODY(S, KC)                                                     \
     {                                                                            \
         const float bias = __uint_as_float(cy);                                  \
-        const uint32_t nt = cx >> CASE_BITS;                                     \
         float Cs[4];                                                             \
         Cs[0] = __uint_as_float(cz);                                             \
         Cs[1] = __uint_as_float(cw);                                             \
-        Cs[3] = 0.f;                                                             \
         uint32_t ex, ey, ez, ew;                                                 \
         lds4(pc + 16, ex, ey, ez, ew);                                           \
-        uint32_t fo[8];                                                          \
-        uint32_t pp = pc + 32;                                                   \
+        uint32_t fo[6];                                                          \
         if (KC == 2) {                                                           \
             fo[0] = ex & 0xffffu; fo[1] = ex >> 16;                              \
             fo[2] = ey & 0xffffu; fo[3] = ey >> 16;                              \
             fo[4] = 0; fo[5] = 0;                                                \
-            fo[6] = ez; fo[7] = ew;                                              \
             Cs[2] = 0.f;                                                         \
         } else {                                                                 \
             Cs[2] = __uint_as_float(ex);                                         \
             fo[0] = ey & 0xffffu; fo[1] = ey >> 16;                              \
             fo[2] = ez & 0xffffu; fo[3] = ez >> 16;                              \
             fo[4] = ew & 0xffffu; fo[5] = ew >> 16;                              \
-            fo[6] = 0; fo[7] = 0;                                                \
-            if (nt) {                                                            \
-                uint32_t t0, t1, t2, t3;                                         \
-                lds4(pp, t0, t1, t2, t3);                                        \
-                fo[6] = t0; fo[7] = t1;                                          \
-                pp += 16;                                                        \
-            }                                                                    \
         }                                                                        \
-        SPN_NEXT(pp + 16 * (2 * KC + nt))                                        \
-        h_slpu<S, KC, ACC>(r, bias, Cs, fo, nt, pp, e);                          \
+        Cs[3] = 0.f;                                                             \
+        const uint32_t pp = pc + 32;                                             \
+        SPN_NEXT(pp + 16 * 2 * KC)                                               \
+        h_slpu<SPN_SS(S), KC>(r, bias, Cs, fo, pp, e);                           \
     }
-#define SPN_BODY_26(S) SPN_SLPU_BODY(SPN_SS(S), 2, false)
-#define SPN_BODY_27(S) SPN_SLPU_BODY(SPN_SS(S), 3, false)
-#define SPN_BODY_28(S) SPN_SLPU_BODY(S, 2, true)
-#define SPN_BODY_29(S) SPN_SLPU_BODY(S, 3, true)
-#define SPN_UNUSED_CASES case 510: case 511: return;
+#define SPN_BODY_26(S) SPN_SLPU_BODY(S, 2)
+#define SPN_BODY_27(S) SPN_SLPU_BODY(S, 3)
+#define SPN_UNUSED_CASES case 476: case 477: case 478: case 479: case 480: case 481: case 482: case 483: case 484: case 485: case 486: case 487: case 488: case 489: case 490: case 491: case 492: case 493: case 494: case 495: case 496: case 497: case 498: case 499: case 500: case 501: case 502: case 503: case 504: case 505: case 506: case 507: case 508: case 509: case 510: case 511: return;
 
 // Run one task's program (shared memory at byte address prog) for this
 // thread's K samples.  All case labels 0..511 exist, so the dispatch is one
@@ -756,8 +718,6 @@ __device__ __forceinline__ void run_task(uint32_t prog, const Env<K, MARG, XS> &
             SPN_ALL_SP(SPN_CASE, 25)
             SPN_ALL_SP(SPN_CASE, 26)
             SPN_ALL_SP(SPN_CASE, 27)
-            SPN_ALL_SP(SPN_CASE, 28)
-            SPN_ALL_SP(SPN_CASE, 29)
             SPN_UNUSED_CASES
             default:
                 __builtin_unreachable();
@@ -794,7 +754,7 @@ __device__ __forceinline__ void load_x_tile(float *xw, int tpw, const float *__r
 }
 
 template <int K, bool MARG, bool XS, int D>
-__global__ void __launch_bounds__(K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 1024))) dag_eval_kernel(const KParams p) {
+__global__ void __launch_bounds__(K == 8 ? 256 : (K == 4 ? 384 : (K == 2 ? 768 : 512))) dag_eval_kernel(const KParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     constexpr int WT = 32 * K;
     Rec *prog_s = reinterpret_cast<Rec *>(smem_raw);
@@ -912,7 +872,7 @@ int dag_eval_occupancy_t(int block, size_t smem) {
 // maximum register-stack depth per samples-per-thread variant (registers:
 // D x K stack values per thread)
 template <int K>
-constexpr int stack_depth() { return K == 4 ? MAXD : 10; }
+constexpr int stack_depth() { return (K == 8 || K == 2) ? 10 : MAXD; }
 
 #define SPNB_INSTANTIATE_K(K)                                                             \
     cudaError_t dag_eval_launch_k##K(const KParams &p, bool marg, bool xs, int grid,       \

@@ -643,56 +643,6 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
         fixes.push_back({(int64_t)prog.size(), u, 0});
         rec_of(OP_LDS, sp, 0, fbits((float)bias));
     };
-    // straight-line SLPU form of an SLP-eligible sum whose children all have
-    // exactly 2 Gaussian leaves; optional accumulate mode and <= 2 tail leaves
-    auto slpu_ok = [&](int64_t s, const std::vector<int64_t> &tail) -> bool {
-        if (!slp_ok(s)) return false;
-        const int64_t n = fan(s);
-        if (n != 2 && n != 3) return false;
-        if (tail.size() > 2) return false;
-        for (int64_t e = c.cb[s]; e < c.cb[s + 1]; ++e) {
-            const int64_t ch = c.ch[e];
-            if (c.kind[ch] != SPN_PRODUCT || fan(ch) != 2) return false;
-            for (int64_t f = c.cb[ch]; f < c.cb[ch + 1]; ++f)
-                if (feat_arg(leaf[c.ch[f]].f) > 0xffffu) return false;
-        }
-        for (int64_t l : tail)
-            if (!leaf[l].gauss || feat_arg(leaf[l].f) > 0xffffu) return false;
-        return true;
-    };
-    auto emit_slpu = [&](int64_t s, int sp, double bias, bool acc, const std::vector<int64_t> &tail) {
-        const int64_t n = fan(s);
-        uint32_t Cb[3] = {0, 0, 0};
-        std::vector<int64_t> lv;
-        int ci = 0;
-        for (int64_t e = c.cb[s]; e < c.cb[s + 1]; ++e, ++ci) {
-            const int64_t ch = c.ch[e];
-            double C = lw2(c.w[e]);
-            for (int64_t f = c.cb[ch]; f < c.cb[ch + 1]; ++f) {
-                C += leaf[c.ch[f]].c;
-                lv.push_back(c.ch[f]);
-            }
-            Cb[ci] = fbits((float)C);
-        }
-        double b = bias;
-        for (int64_t l : tail) b += leaf[l].c;
-        uint32_t fo[6] = {0, 0, 0, 0, 0, 0}, ft[2] = {0, 0};
-        for (size_t k = 0; k < lv.size(); ++k) fo[k] = feat_arg(leaf[lv[k]].f);
-        for (size_t k = 0; k < tail.size(); ++k) ft[k] = feat_arg(leaf[tail[k]].f);
-        const uint32_t nt = (uint32_t)tail.size();
-        if (!acc) max_sp = std::max<int64_t>(max_sp, sp + 1);
-        const uint32_t op = n == 2 ? (acc ? OP_SLPU2A : OP_SLPU2) : (acc ? OP_SLPU3A : OP_SLPU3);
-        rec_of(op, acc ? sp + 1 : sp, nt, fbits((float)b), Cb[0], Cb[1]);
-        if (n == 2) {
-            prog.push_back(Rec{fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16), ft[0], ft[1]});
-        } else {
-            prog.push_back(Rec{Cb[2], fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16),
-                               fo[4] | (fo[5] << 16)});
-            if (nt) prog.push_back(Rec{ft[0], ft[1], 0, 0});
-        }
-        for (int64_t l : lv) prog.push_back(Rec{feat_arg(leaf[l].f), leaf[l].y, leaf[l].z, leaf[l].w});
-        for (int64_t l : tail) prog.push_back(Rec{feat_arg(leaf[l].f), leaf[l].y, leaf[l].z, leaf[l].w});
-    };
     std::function<void(int64_t, int, double)> emit_value;
     auto emit_child = [&](int64_t ch, int sp, double bias) {
         if (!is_leaf(c.kind[ch]) && mat[ch]) emit_load(ch, sp, bias);
@@ -718,17 +668,8 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
                 emit_leaves(leaves, sp, false, bias);
                 return;
             }
-            // the last inner child (lowest need) fused with the leaves when it
-            // is an SLPU-shaped sum: SLPU (push) or SLPUA (accumulate) + tail
-            const int64_t lastc = inner.back().second;
-            const bool fuse = !mat[lastc] && slpu_ok(lastc, leaves);
             for (size_t i = 0; i < inner.size(); ++i) {
-                const bool is_last = i + 1 == inner.size();
-                if (is_last && fuse) {
-                    emit_slpu(lastc, i == 0 ? sp : sp, bias, i > 0, leaves);
-                    return;
-                }
-                const bool last_add = leaves.empty() && is_last;
+                const bool last_add = leaves.empty() && i + 1 == inner.size();
                 if (i == 0) {
                     emit_child(inner[i].second, sp, inner.size() == 1 && leaves.empty() ? bias : 0.0);
                 } else {
@@ -782,12 +723,26 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
                 lv.insert(lv.end(), cl.begin(), cl.end());
             }
             max_sp = std::max<int64_t>(max_sp, sp + 1);
-            if (slpu_ok(u, {})) {
-                emit_slpu(u, sp, bias, false, {});
-                return;
+            // straight-line form for children of exactly 2 leaves (n = 2, 3)
+            bool uni = (n == 2 || n == 3) && counts == (n == 2 ? 0x12u : 0x92u);
+            uint32_t fo[6] = {0, 0, 0, 0, 0, 0};
+            if (uni) {
+                for (size_t k = 0; k < lv.size(); ++k) {
+                    fo[k] = feat_arg(leaf[lv[k]].f);
+                    if (fo[k] > 0xffffu) uni = false;
+                }
             }
-            rec_of(OP_SLP2 + (uint32_t)(n - 2), sp, counts, fbits((float)bias), Cb[0], Cb[1]);
-            if (n >= 3) prog.push_back(Rec{Cb[2], Cb[3], 0, 0});
+            if (uni && n == 2) {
+                rec_of(OP_SLPU2, sp, 0, fbits((float)bias), Cb[0], Cb[1]);
+                prog.push_back(Rec{fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16), 0, 0});
+            } else if (uni) {
+                rec_of(OP_SLPU3, sp, 0, fbits((float)bias), Cb[0], Cb[1]);
+                prog.push_back(Rec{Cb[2], fo[0] | (fo[1] << 16), fo[2] | (fo[3] << 16),
+                                   fo[4] | (fo[5] << 16)});
+            } else {
+                rec_of(OP_SLP2 + (uint32_t)(n - 2), sp, counts, fbits((float)bias), Cb[0], Cb[1]);
+                if (n >= 3) prog.push_back(Rec{Cb[2], Cb[3], 0, 0});
+            }
             for (int64_t l : lv) prog.push_back(Rec{feat_arg(leaf[l].f), leaf[l].y, leaf[l].z, leaf[l].w});
             return;
         }
@@ -862,12 +817,10 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             i += cs / NSP - OP_GPUSH1 + 1;
         else if (cs / NSP >= OP_GACC1 && cs / NSP <= OP_GACC4)
             i += cs / NSP - OP_GACC1 + 1;
-        else if ((cs / NSP == OP_SLPU2 || cs / NSP == OP_SLPU2A) && cs < OP_COUNT * NSP)
-            i += 1 + 4 + (prog[i].x >> CASE_BITS);
-        else if ((cs / NSP == OP_SLPU3 || cs / NSP == OP_SLPU3A) && cs < OP_COUNT * NSP) {
-            const int64_t nt = prog[i].x >> CASE_BITS;
-            i += 1 + (nt ? 1 : 0) + 6 + nt;
-        }
+        else if (cs / NSP == OP_SLPU2 && cs < OP_COUNT * NSP)
+            i += 1 + 4;
+        else if (cs / NSP == OP_SLPU3 && cs < OP_COUNT * NSP)
+            i += 1 + 6;
         else if (cs / NSP >= OP_SLP2 && cs / NSP <= OP_SLP4 && cs < OP_COUNT * NSP) {
             const uint32_t cnt = prog[i].x >> CASE_BITS;
             i += (cs / NSP >= OP_SLP3 ? 1 : 0) + (cnt & 7u) + ((cnt >> 3) & 7u) +

@@ -25,12 +25,6 @@
 //   SLPU3 | bias, C0, C1  + {C2, f0|f1<<16, f2|f3<<16, f4|f5<<16} + 6 leaf records
 //       straight-line forms of the dominant SLP shapes (children of 2 leaves),
 //       with the leaves' feature offsets up front so all loads issue at once.
-//       arg = nt (0..2 "tail" leaves multiplying the sum: their -t^2 is added
-//       to the result, their constants are folded into bias); the tail's
-//       feature offsets are {z, w} of SLPU2's offset record, or a record
-//       {ft0, ft1, -, -} after SLPU3's; tail parameter records come last.
-//   SLPU2A / SLPU3A: the same, accumulated into r[sp-1] (a product of the
-//       value below on the stack and this sum)
 //       followed by ng Gaussian parameter records {f, a, b, c} and nd discrete
 //       records {f, table, lo, K}.  Gaussian: c - (a*x_f - b)^2 = log2 N(x; mu, s)
 //       with a = 1/(s sqrt(2 ln2)), b = a mu, c = -log2(s sqrt(2 pi)); the c's
@@ -80,9 +74,7 @@ enum Op : uint32_t {
     OP_SLP4 = 25,
     OP_SLPU2 = 26,  // straight-line SLP: 2 children x 2 Gaussian leaves
     OP_SLPU3 = 27,  // straight-line SLP: 3 children x 2 Gaussian leaves
-    OP_SLPU2A = 28, // ... accumulated into r[sp-1] (product of a stack value and the sum)
-    OP_SLPU3A = 29,
-    OP_COUNT = 30
+    OP_COUNT = 28
 };
 
 constexpr int MAXD = 16;              // register stack depth

@@ -50,6 +50,7 @@ struct RParams {
     int32_t first_leaf; // index of the first LEAF step
     int32_t max_leaf_params;  // floats of the largest staged leaf parameter block
     int32_t wbufs;      // 2: double-buffered weight groups + TMEM ping-pong; 1: serial
+    unsigned long long *prof;  // optional phase-cycle counters (thread 0 of each CTA)
 };
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
@@ -315,6 +316,16 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     };
 
     const int64_t n_tiles = (p.n + RT - 1) / RT;
+    // optional profiling: cycles per phase measured by thread 0
+    unsigned long long pc_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long t_mark = clock64();
+    auto prof_mark = [&](int k) {
+        if (p.prof && tid == 0) {
+            const unsigned long long t = clock64();
+            pc_acc[k] += t - t_mark;
+            t_mark = t;
+        }
+    };
     if (warp == 0 && (int64_t)blockIdx.x < n_tiles) issue_x(p.first_leaf, (int64_t)blockIdx.x * RT, 0);
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const int64_t base = tile * RT;
@@ -324,8 +335,10 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             const LStep st = p.steps[si];  // by value: fields live in registers
             if (st.type == 0) {
                 const int b = xbuf;
+                prof_mark(7);
                 mbar_wait(bar_x0 + 8 * b, (ph_x >> b) & 1u);
                 ph_x ^= 1u << b;
+                prof_mark(0);  // 0: waiting for the leaf rows
                 if (warp == 0) {  // prefetch the next leaf step's rows (maybe next tile)
                     if (st.rep >= 0) issue_x(st.rep, base, b ^ 1);
                     else if (tile + gridDim.x < n_tiles)
@@ -336,7 +349,9 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                     const float *stg = xsb + (size_t)b * stage_floats;
                     leaf_step<MARG>(st, act, stg, stg + (size_t)p.max_vars * RT, tid);
                 }
+                prof_mark(1);  // 1: leaf compute
                 __syncthreads();
+                prof_mark(2);  // 2: leaf barrier
                 continue;
             }
             // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
@@ -372,6 +387,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             }
             fence_async_smem();
             __syncthreads();
+            prof_mark(3);  // 3: sum phase 1 (+barrier)
             // ---------------- phase 2: per N-group MMA + epilogue -------------
             const uint32_t lbo_a = RT * 16;
             const uint32_t lbo_b = (uint32_t)st.n_group * 16;
@@ -389,23 +405,32 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 const int sl0 = half ? hcut : 0, sl1 = half ? ns : hcut;
                 const float shift = sa[m] + sb[m];
                 for (int sl = sl0; sl < sl1; ++sl) {
-                    float acc = 0.f;
+                    // TMEM loads in batches of up to 32 columns, one wait per batch
                     const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
-                    int c0 = 0;
-                    for (; c0 + 8 <= na; c0 += 8) {
-                        float t[8];
-                        tmem_ld8(trow + c0, t);
+                    float a4[4] = {0.f, 0.f, 0.f, 0.f};  // 4 independent FMA chains
+                    for (int cb = 0; cb < na; cb += 32) {
+                        float t[32];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const int c0 = cb + q * 8;
+                            if (c0 + 8 <= na) {
+                                float v8[8];
+                                tmem_ld8(trow + c0, v8);
+#pragma unroll
+                                for (int k = 0; k < 8; ++k) t[q * 8 + k] = v8[k];
+                            } else if (c0 < na) {
+                                float v4[4];
+                                tmem_ld4(trow + c0, v4);
+#pragma unroll
+                                for (int k = 0; k < 4; ++k) t[q * 8 + k] = v4[k];
+                            }
+                        }
                         tmem_wait_ld();
 #pragma unroll
-                        for (int k = 0; k < 8; ++k) acc = fmaf(ea[(c0 + k) * RT + m], t[k], acc);
+                        for (int i = 0; i < 32; ++i)
+                            if (cb + i < na) a4[i & 3] = fmaf(ea[(cb + i) * RT + m], t[i], a4[i & 3]);
                     }
-                    if (c0 < na) {  // na % 8 == 4
-                        float t[4];
-                        tmem_ld4(trow + c0, t);
-                        tmem_wait_ld();
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) acc = fmaf(ea[(c0 + k) * RT + m], t[k], acc);
-                    }
+                    const float acc = (a4[0] + a4[1]) + (a4[2] + a4[3]);
                     const float val = shift + r_lg2(acc);
                     const int s = s0 + sl;
                     if (st.type == 1) {
@@ -421,6 +446,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 const uint32_t tb = p.wbufs == 2 ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
                 mbar_wait(bar_w0 + 8 * wb, (ph_w >> wb) & 1u);
                 ph_w ^= 1u << wb;
+                prof_mark(4);  // 4: waiting for weights
                 if (tid == 0) {
                     fence_after();
                     const uint32_t w_hi = r_smem(wsm) + (uint32_t)(wb * w_buf);
@@ -441,9 +467,11 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 __syncwarp();
                 // overlap: the previous group's epilogue runs under this MMA
                 if (p.wbufs == 2 && g > 0) epilogue(g - 1, (uint32_t)((g - 1) & 1) * TMEM_BUF);
+                prof_mark(5);  // 5: MMA issue + overlapped epilogue
                 mbar_wait(bar_mma, ph_mma);
                 ph_mma ^= 1;
                 fence_after();
+                prof_mark(6);  // 6: waiting for the MMA
                 // the MMA has consumed weight buffer wb: refill it
                 if (tid == 0 && g + p.wbufs < G) issue_w(st, g + p.wbufs, wb);
                 if (p.wbufs == 1) epilogue(g, 0u);
@@ -475,6 +503,8 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
         }
         __syncthreads();
     }
+    if (p.prof && tid == 0)
+        for (int k = 0; k < 8; ++k) atomicAdd(p.prof + k, pc_acc[k]);
     fence_before();
     __syncthreads();
     if (warp == 0)

@@ -15,7 +15,7 @@ NSP = 17
 OPS = ["END", "LPUSH", "LACC", "ADD", "LSE1", "LSE2", "LSE3", "LSE4",
        "LDS", "LDG", "STS", "STG", "GLSE", "OUT", "NOP",
        "GPUSH1", "GPUSH2", "GPUSH3", "GPUSH4", "GACC1", "GACC2", "GACC3", "GACC4",
-       "SLP2", "SLP3", "SLP4", "SLPU2", "SLPU3", "SLPU2A", "SLPU3A"]
+       "SLP2", "SLP3", "SLP4", "SLPU2", "SLPU3"]
 SLOT_GLOBAL = 0x80000000
 SLOT_NONE = 0xFFFFFFFF
 
@@ -69,17 +69,12 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
             if op == "END":
                 break
             if op.startswith("SLP"):
-                nt, accm = 0, False
                 if op.startswith("SLPU"):
                     k = int(op[4])
-                    accm = op.endswith("A")
-                    nt = arg
                     Cs = [_f32(r["z"]), _f32(r["w"])]
                     if k == 3:
                         Cs.append(_f32(rec[pc]["x"]))
                     pc += 1                   # feature-offset record (offsets repeat below)
-                    if k == 3 and nt:
-                        pc += 1               # tail feature-offset record
                     arg = 2 | (2 << 3) | ((2 << 6) if k == 3 else 0)
                 else:
                     k = int(op[3])
@@ -98,18 +93,7 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
                         t = a * xv - b
                         acc = acc - (np.where(np.isnan(xv), c, t * t) if marginal else t * t)
                     vals.append(acc)
-                res = _lse(vals) + _f32(r["y"])
-                for _ in range(nt):
-                    q = rec[pc]
-                    pc += 1
-                    xv = xd[:, feat(int(q["x"]))]
-                    a, b, c = _f32(q["y"]), _f32(q["z"]), _f32(q["w"])
-                    t = a * xv - b
-                    res = res - (np.where(np.isnan(xv), c, t * t) if marginal else t * t)
-                if accm:
-                    stack[sp - 1] = stack[sp - 1] + res
-                else:
-                    stack[sp] = res
+                stack[sp] = _lse(vals) + _f32(r["y"])
                 continue
             if op[:5] in ("GPUSH", "GACC1", "GACC2", "GACC3", "GACC4"):
                 ng, nd = int(op[-1]), 0

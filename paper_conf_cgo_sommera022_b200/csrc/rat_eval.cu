@@ -396,39 +396,53 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             const uint32_t a_hi = r_smem(aimg), a_lo = a_hi + (uint32_t)aimg_part;
             // epilogue of group g from TMEM buffer tb: warp quarter q reads
             // lanes 32q..32q+31 (= samples); the two warp halves split the sums
+            // this thread's sample (TMEM lane quarter) and its ea values in
+            // registers, reused by every sum of every group of this step
+            const int qd = warp & 3, half = warp >> 2;
+            const int m_ep = qd * 32 + lane;
+            float ear[64];
+#pragma unroll
+            for (int i = 0; i < 64; ++i) ear[i] = i < na ? ea[i * RT + m_ep] : 0.f;
+            const float shift = sa[m_ep] + sb[m_ep];
             auto epilogue = [&](int g, uint32_t tb) {
-                const int qd = warp & 3, half = warp >> 2;
-                const int m = qd * 32 + lane;
+                const int m = m_ep;
                 const int s0 = g * st.s_per_group;
                 const int ns = min(st.s_per_group, st.n_out - s0);
                 const int hcut = (ns + 1) >> 1;
                 const int sl0 = half ? hcut : 0, sl1 = half ? ns : hcut;
-                const float shift = sa[m] + sb[m];
                 for (int sl = sl0; sl < sl1; ++sl) {
                     // TMEM loads in batches of up to 32 columns, one wait per batch
                     const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
                     float a4[4] = {0.f, 0.f, 0.f, 0.f};  // 4 independent FMA chains
-                    for (int cb = 0; cb < na; cb += 32) {
-                        float t[32];
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) {
-                            const int c0 = cb + q * 8;
-                            if (c0 + 8 <= na) {
-                                float v8[8];
-                                tmem_ld8(trow + c0, v8);
+                    for (int cb = 0; cb < 64; cb += 32) {
+                        if (cb < na) {
+                            float t[32];
 #pragma unroll
-                                for (int k = 0; k < 8; ++k) t[q * 8 + k] = v8[k];
-                            } else if (c0 < na) {
-                                float v4[4];
-                                tmem_ld4(trow + c0, v4);
+                            for (int q = 0; q < 4; ++q) {
+                                const int c0 = cb + q * 8;
+                                if (c0 + 8 <= na) {
+                                    float v8[8];
+                                    tmem_ld8(trow + c0, v8);
 #pragma unroll
-                                for (int k = 0; k < 4; ++k) t[q * 8 + k] = v4[k];
+                                    for (int k = 0; k < 8; ++k) t[q * 8 + k] = v8[k];
+                                } else if (c0 < na) {
+                                    float v4[4];
+                                    tmem_ld4(trow + c0, v4);
+#pragma unroll
+                                    for (int k = 0; k < 4; ++k) {
+                                        t[q * 8 + k] = v4[k];
+                                        t[q * 8 + 4 + k] = 0.f;
+                                    }
+                                } else {
+#pragma unroll
+                                    for (int k = 0; k < 8; ++k) t[q * 8 + k] = 0.f;
+                                }
                             }
-                        }
-                        tmem_wait_ld();
+                            tmem_wait_ld();
 #pragma unroll
-                        for (int i = 0; i < 32; ++i)
-                            if (cb + i < na) a4[i & 3] = fmaf(ea[(cb + i) * RT + m], t[i], a4[i & 3]);
+                            for (int i = 0; i < 32; ++i) a4[i & 3] = fmaf(ear[cb + i], t[i], a4[i & 3]);
+                        }
                     }
                     const float acc = (a4[0] + a4[1]) + (a4[2] + a4[3]);
                     const float val = shift + r_lg2(acc);

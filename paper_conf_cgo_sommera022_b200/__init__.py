@@ -75,7 +75,7 @@ def load_library(path: str | None = None):
     global _lib
     if _lib is not None:
         return _lib
-    path = path or _LIB_PATH
+    path = path or os.environ.get("SPNB_LIB") or _LIB_PATH  # SPNB_LIB: variant builds (experiments)
     if not os.path.exists(path):
         raise ImportError(f"libspnb.so not built ({path}); run __graft_entry__.build()")
     lib = ctypes.CDLL(path)

@@ -375,13 +375,22 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 float hi = -CUDART_INF_F;
                 for (int j = 0; j < nb; ++j) hi = r_maxnan(hi, VB[j * RT + m]);
                 const float hc = fmaxf(hi, -1e30f);
-                for (int j = 0; j < kpad; ++j) {
-                    const float e = j < nb ? r_ex2(VB[j * RT + m] - hc) : 0.f;
-                    const __half h = __float2half_rn(e);
-                    const __half l = __float2half_rn(e - __half2float(h));
-                    const uint32_t o = img_off(m, j, RT);
-                    *reinterpret_cast<__half *>(aimg + o) = h;
-                    *reinterpret_cast<__half *>(aimg + aimg_part + o) = l;
+                for (int j0 = 0; j0 < kpad; j0 += 8) {  // 8 k-values = one 16-byte row
+                    uint32_t hw[4], lw[4];
+#pragma unroll
+                    for (int k = 0; k < 8; k += 2) {
+                        const int j = j0 + k;
+                        const float e0 = j < nb ? r_ex2(VB[j * RT + m] - hc) : 0.f;
+                        const float e1 = j + 1 < nb ? r_ex2(VB[(j + 1) * RT + m] - hc) : 0.f;
+                        const __half h0 = __float2half_rn(e0), h1 = __float2half_rn(e1);
+                        const __half l0 = __float2half_rn(e0 - __half2float(h0));
+                        const __half l1 = __float2half_rn(e1 - __half2float(h1));
+                        hw[k >> 1] = (uint32_t)__half_as_ushort(h0) | ((uint32_t)__half_as_ushort(h1) << 16);
+                        lw[k >> 1] = (uint32_t)__half_as_ushort(l0) | ((uint32_t)__half_as_ushort(l1) << 16);
+                    }
+                    const uint32_t o = img_off(m, j0, RT);
+                    *reinterpret_cast<uint4 *>(aimg + o) = make_uint4(hw[0], hw[1], hw[2], hw[3]);
+                    *reinterpret_cast<uint4 *>(aimg + aimg_part + o) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
                 }
                 sb[m] = hi;
             }

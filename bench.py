@@ -215,6 +215,16 @@ def _config_dict(args, g, n):
             "parallelism": f"dp{args.gpus} (sample sharding)"}
 
 
+def launches_per_step(info: dict, n: int, want_am: bool) -> int:
+    """Kernels of this library launched by one inference call (see api.cpp)."""
+    if info["path"] == 2:   # one generated kernel per task (+ argmax if unfused)
+        return info["n_tasks"] + (1 if want_am and info["n_tasks"] > 1 else 0)
+    if info["path"] == 1:   # per transposed chunk: transpose + layered kernel
+        chunk = max(1, info["chunk_samples"])
+        return 2 * ((n + chunk - 1) // chunk)
+    return 1
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -327,7 +337,7 @@ def run_ours(args):
                 traffic = json.load(f).get("dram_bytes_per_launch")
         hbm_part = {"achieved": hbm, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                     "frac": hbm / peaks["hbm_gbs"]}
-        if info["path"] == 0:
+        if info["path"] in (0, 2):
             roof = {"bound": "alu", "pipe": "MUFU ex2/lg2 (16 op/clk/SM)",
                     "achieved": mufu / 1e9, "peak": mufu_peak / 1e9, "unit": "Gop/s",
                     "frac": mufu / mufu_peak, "traffic": traffic,
@@ -363,7 +373,8 @@ def run_ours(args):
                                                   "block_threads", "samples_per_thread",
                                                   "grid", "smem_bytes", "mufu_per_sample",
                                                   "fma_per_sample", "tc_flops_per_sample",
-                                                  "max_stack")},
+                                                  "max_stack", "kernel_regs", "ctas_per_sm",
+                                                  "mufu_exec_per_sample", "compile_ms")},
                     "prepare_s": prep_s},
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
                 "e2e": {"value": e2e_val, "unit": UNIT,
@@ -371,7 +382,7 @@ def run_ours(args):
                         "d2h_bytes_per_step": int(n_e2e * R * 4 + (n_e2e * 4 if want_am else 0)),
                         "samples_per_step": int(n_e2e),
                         "timing": "wall clock around the synchronous host-buffer call"},
-                "gpu_launches": args.steps,
+                "gpu_launches": args.steps * launches_per_step(info, n, want_am),
                 "step_ms": {"min": min(times), "median": statistics.median(times),
                             "max": max(times)}}
         print(json.dumps(line), flush=True)

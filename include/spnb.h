@@ -79,8 +79,17 @@ typedef struct spn_prepare_options {
                                    0 = auto (shared-memory budget), -1 = none  */
     int32_t tc_precision;       /* layered path: 0 auto (= 2), 1 f16 single
                                    pass, 2 f16 hi/lo split (3 MMAs, ~fp32)    */
-    int32_t ctas_per_sm;        /* 0 = auto                                    */
-    int32_t reserved[8];        /* must be zero                                */
+    int32_t ctas_per_sm;        /* 0 = auto; compiled path: the kernels'
+                                   __launch_bounds__ minimum CTAs per SM     */
+    int32_t compiled_path;      /* 0 auto, 1 off (interpreter), 2 force: one
+                                   straight-line kernel generated per SPN task
+                                   (PTX) and assembled for the device at
+                                   prepare time (the paper's per-SPN GPU
+                                   compilation, §IV-C).
+                                   Auto uses it for non-layered graphs unless
+                                   samples_per_thread / max_task_nodes are set
+                                   (interpreter knobs) or compilation fails  */
+    int32_t reserved[7];        /* must be zero                                */
 } spn_prepare_options;
 
 /* Statistics of a prepared plan (used by the benchmark's roofline). */
@@ -100,11 +109,19 @@ typedef struct spn_plan_stats {
                                    3/sum edge)                                */
     int64_t bytes_per_sample;   /* 4*n_features + 4*n_roots (+4 argmax)       */
     int64_t tc_flops_per_sample;/* layered path only                          */
-    int32_t path;               /* 0 generic interpreter, 1 layered RAT path  */
+    int32_t path;               /* 0 generic interpreter, 1 layered RAT path,
+                                   2 compiled (generated per-SPN kernels)    */
     int32_t block_threads, samples_per_thread, grid;
     int32_t smem_bytes;
     int32_t x_in_smem;
     double  prepare_ms;
+    /* compiled path (path 2) */
+    int32_t kernel_regs;        /* max registers per thread over the kernels  */
+    int32_t ctas_per_sm;        /* min resident CTAs per SM over the kernels  */
+    int64_t mufu_exec_per_sample; /* ex2 + lg2 the generated code executes    */
+    double  compile_ms;         /* PTX assembly wall time (tasks in parallel)  */
+    int64_t chunk_samples;      /* layered path: samples per transposed chunk
+                                   (one transpose + one layered launch each)  */
 } spn_plan_stats;
 
 /* Fill *opt with defaults (all auto). */
@@ -220,6 +237,24 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
                       void *records, int64_t *n_records, int64_t *task_off, int64_t *n_tasks,
                       float *tables, int64_t *n_tables, void *edges, int64_t *n_edges,
                       int64_t *slots);
+
+/*
+ * spn_codegen: run the compiled path's code generator (no GPU needed) and
+ *   return task `task`'s generated code: lang = 1 the PTX the library
+ *   assembles (entries <name>_j / <name>_m), lang = 0 the same IR printed as
+ *   plain C++ defining `<name>_host(x, n, ld, out, R, argmax, tab, marg)`,
+ *   which the CPU test-suite compiles to check the generator against the
+ *   oracle.  Sizes first (NULL buffers): *src_len (bytes incl. NUL),
+ *   *n_roots, *n_tables (floats), *n_tasks; then again with buffers.
+ *   name[64] receives the kernel base name; roots[] the output columns the
+ *   task writes; tables[] the discrete-leaf tables (log2) passed as `tab`.
+ *   compile = 1 additionally assembles the PTX with nvJitLink for
+ *   sm_<arch> (arch e.g. "100a"), returning SPN_E_UNSUPPORTED with the
+ *   assembler log in spn_last_error on failure.
+ */
+int spn_codegen(const spn_handle *graph, int32_t task, int32_t lang, char *src, int64_t *src_len,
+                char *name, int32_t *roots, int32_t *n_roots, float *tables, int64_t *n_tables,
+                int32_t *n_tasks, int32_t compile, const char *arch);
 
 /* Free a graph or a plan; NULL is a no-op.  The caller must synchronise
    outstanding work on the plan first. */

@@ -53,7 +53,8 @@ class _Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("samples_per_thread", ctypes.c_int32), ("layered_path", ctypes.c_int32),
                 ("max_task_nodes", ctypes.c_int64), ("tc_precision", ctypes.c_int32),
-                ("ctas_per_sm", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("ctas_per_sm", ctypes.c_int32), ("compiled_path", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
 
 
 class _Stats(ctypes.Structure):
@@ -64,7 +65,9 @@ class _Stats(ctypes.Structure):
         "tc_flops_per_sample")] + [
         (n, ctypes.c_int32) for n in ("path", "block_threads", "samples_per_thread", "grid",
                                       "smem_bytes", "x_in_smem")] + [
-        ("prepare_ms", ctypes.c_double)]
+        ("prepare_ms", ctypes.c_double), ("kernel_regs", ctypes.c_int32),
+        ("ctas_per_sm", ctypes.c_int32), ("mufu_exec_per_sample", ctypes.c_int64),
+        ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64)]
 
 
 _lib = None
@@ -94,9 +97,11 @@ def load_library(path: str | None = None):
     lib.spn_partition_graph.argtypes = [P, I64, P, P, P, P]
     lib.spn_build_program.argtypes = [P, I32, I32, I64, I64, P, P, P, P, P, P, P, P, P]
     lib.spn_build_layered.argtypes = [P, P, P, I64, P, P, P, P, P, P]
+    lib.spn_codegen.argtypes = [P, I32, I32, P, P, P, P, P, P, P, P, I32, ctypes.c_char_p]
     for name in ("spn_load_graph", "spn_prepare", "spn_infer_joint", "spn_infer_marginal",
                  "spn_infer_joint_host", "spn_infer_marginal_host", "spn_plan_info",
-                 "spn_partition_graph", "spn_build_program", "spn_build_layered"):
+                 "spn_partition_graph", "spn_build_program", "spn_build_layered",
+                 "spn_codegen"):
         getattr(lib, name).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -161,7 +166,8 @@ class Plan:
 
     def __init__(self, graph: Graph, device: int | None = None, block_threads: int = 0,
                  samples_per_thread: int = 0, max_task_nodes: int = 0,
-                 layered_path: int = 0, tc_precision: int = 0, ctas_per_sm: int = 0):
+                 layered_path: int = 0, tc_precision: int = 0, ctas_per_sm: int = 0,
+                 compiled_path: int = 0):
         lib = load_library()
         opt = _Options()
         lib.spn_default_options(ctypes.byref(opt))
@@ -175,6 +181,7 @@ class Plan:
         opt.layered_path = layered_path
         opt.tc_precision = tc_precision
         opt.ctas_per_sm = ctas_per_sm
+        opt.compiled_path = compiled_path
         h = ctypes.c_void_p()
         _check(lib.spn_prepare(graph.handle, ctypes.byref(opt), ctypes.byref(h)))
         self._h = h
@@ -302,3 +309,29 @@ def build_layered(graph: Graph):
                                  _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w), _ptr(rm)))
     return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
             "smem_floats": int(sizes[5])}, ""
+
+
+def codegen(graph: Graph, task: int = 0, lang: str = "cpp", compile: bool = False,
+            arch: str = "100a"):
+    """Host-only: the compiled path's generated code for one task
+    (``spn_codegen``): lang "ptx" (what the library assembles) or "cpp" (the
+    same IR as host C++, for CPU checks).  Returns dict(source, name, roots,
+    tables, n_tasks).  compile=True also assembles the PTX for sm_<arch>
+    with nvJitLink (raises SPNError on failure)."""
+    lg = {"cpp": 0, "ptx": 1}[lang]
+    lib = load_library()
+    sl, nt = ctypes.c_int64(), ctypes.c_int64()
+    nr, ntask = ctypes.c_int32(), ctypes.c_int32()
+    _check(lib.spn_codegen(graph.handle, int(task), lg, None, ctypes.byref(sl), None, None,
+                           ctypes.byref(nr), None, ctypes.byref(nt), ctypes.byref(ntask), 0,
+                           arch.encode()))
+    src = ctypes.create_string_buffer(sl.value)
+    name = ctypes.create_string_buffer(64)
+    roots = np.zeros(max(1, nr.value), dtype=np.int32)
+    tab = np.zeros(max(1, nt.value), dtype=np.float32)
+    _check(lib.spn_codegen(graph.handle, int(task), lg, src, ctypes.byref(sl), name, _ptr(roots),
+                           ctypes.byref(nr), _ptr(tab), ctypes.byref(nt), ctypes.byref(ntask),
+                           int(bool(compile)), arch.encode()))
+    return {"source": src.value.decode(), "name": name.value.decode(),
+            "roots": roots[:nr.value].copy(), "tables": tab[:nt.value].copy(),
+            "n_tasks": int(ntask.value)}

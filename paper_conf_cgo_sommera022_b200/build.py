@@ -28,9 +28,13 @@ CXX_FLAGS = ["-O2", "-std=c++17", "-fPIC", "-Wall", "-I", CSRC, "-I", INC,
              "-I", "/usr/local/cuda/include"]
 
 CU_SOURCES = ["dag_eval_k1.cu", "dag_eval_k2.cu", "dag_eval_k4.cu", "dag_eval_k8.cu",
-              "rat_eval.cu"]
-CXX_SOURCES = ["prepare.cpp", "layered.cpp", "api.cpp"]
-HEADERS = ["program.h", "dag_eval.cuh", "prepare.h", "layered.h"]
+              "rat_eval.cu", "argmax.cu"]
+CXX_SOURCES = ["prepare.cpp", "layered.cpp", "codegen.cpp", "jit.cpp", "api.cpp"]
+HEADERS = ["program.h", "dag_eval.cuh", "prepare.h", "layered.h", "codegen.h", "jit.h"]
+# headers each CUDA translation unit includes (so editing host-side headers does
+# not rebuild the slow interpreter objects)
+CU_DEPS = {"rat_eval.cu": ["layered.h", "prepare.h", "program.h"], "argmax.cu": []}
+CU_DEPS_DEFAULT = ["dag_eval.cuh", "program.h"]
 
 
 def _nvcc():
@@ -75,7 +79,8 @@ def build(verbose: bool = False, jobs: int = 0) -> str:
         for s in CU_SOURCES:
             src = os.path.join(CSRC, s)
             obj = os.path.join(BUILD, s + ".o")
-            key = _digest([src] + hdrs, NVCC_FLAGS)
+            deps = [os.path.join(CSRC, h) for h in CU_DEPS.get(s, CU_DEPS_DEFAULT)]
+            key = _digest([src] + deps, NVCC_FLAGS)
             futs.append(ex.submit(_compile, [nvcc] + NVCC_FLAGS, src, obj, key))
         for s in CXX_SOURCES:
             src = os.path.join(CSRC, s)

@@ -10,11 +10,15 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <atomic>
 #include <mutex>
+#include <thread>
 #include <new>
 #include <string>
 #include <vector>
 
+#include "codegen.h"
+#include "jit.h"
 #include "layered.h"
 #include "prepare.h"
 #include "program.h"
@@ -55,6 +59,7 @@ size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st);
+cudaError_t argmax_rows_launch(const float *out, int64_t n, int R, int32_t *argmax, cudaStream_t st);
 }  // namespace spnb
 
 using namespace spnb;
@@ -113,6 +118,12 @@ struct DevicePlan {
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
     int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
     unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
+    // compiled (per-SPN generated kernel) path
+    std::vector<JitKernel> jk;
+    std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM x waves
+    int jblock = 256;
+    bool jfused_argmax = false;
+    float *d_jtab = nullptr;
     spn_plan_stats stats;
 };
 
@@ -166,6 +177,8 @@ void free_plan(DevicePlan *p) {
     cudaFree(p->d_wimg);
     cudaFree(p->d_root_map);
     cudaFree(p->d_xT);
+    cudaFree(p->d_jtab);
+    for (auto &k : p->jk) jit_unload(k);
     if (p->d_prof) {
         unsigned long long h[8];
         if (cudaMemcpy(h, p->d_prof, sizeof(h), cudaMemcpyDeviceToHost) == cudaSuccess) {
@@ -222,6 +235,22 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
     if (!x || !out) return set_err(SPN_E_ARG, "null x/out");
     if (ld < P.F) return set_err(SPN_E_ARG, "ld < n_features");
     DeviceGuard dg(P.device);
+    if (P.path == 2) {
+        std::string msg;
+        const int32_t *tasks_am = P.jfused_argmax ? argmax : nullptr;
+        for (size_t t = 0; t < P.jk.size(); ++t) {
+            const int64_t need = (n + P.jblock - 1) / P.jblock;
+            const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, P.jgrid_max[t]));
+            const int rc = jit_launch(P.jk[t], marg, grid, P.jblock, (cudaStream_t)stream, x, n, ld,
+                                      out, P.R, (int *)tasks_am, P.d_jtab, msg);
+            if (rc != SPN_OK) return set_err(rc, msg);
+        }
+        if (argmax && !P.jfused_argmax) {
+            cudaError_t e = argmax_rows_launch(out, n, P.R, argmax, (cudaStream_t)stream);
+            if (e != cudaSuccess) return cuda_err(e, "argmax launch");
+        }
+        return SPN_OK;
+    }
     if (P.path == 1) {
         RParams rp;
         memset(&rp, 0, sizeof(rp));
@@ -410,11 +439,120 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     s.tc_flops_per_sample = lp.tc_flops_per_sample * (P->prec == 3 ? 3 : 1);
     s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)lp.C + 4;
     s.path = 1;
+    s.chunk_samples = chunk;
     s.block_threads = 256;
     s.samples_per_thread = 0;
     s.grid = P->grid_max;
     s.smem_bytes = (int32_t)smem;
     s.x_in_smem = 0;
+    s.prepare_ms =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    spn_handle *h = new (std::nothrow) spn_handle();
+    if (!h) {
+        free_plan(P);
+        return set_err(SPN_E_OOM, "handle");
+    }
+    h->magic = H_PLAN;
+    h->plan = P;
+    *out_plan = h;
+    return SPN_OK;
+}
+
+// Compiled path (kernel KS): generate one straight-line kernel per task
+// (codegen.cpp, emitted as PTX), assemble them for the device's architecture in
+// parallel threads, load them with the driver API.  Returns SPN_OK with
+// *out_plan set, or an error (the caller decides whether to fall back to
+// the interpreter).
+int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev, int sms,
+                     std::chrono::steady_clock::time_point t0, spn_handle **out_plan) {
+    JitOptions jo;
+    jo.block = opt.block_threads ? opt.block_threads : 256;
+    if (jo.block % 32 || jo.block < 32 || jo.block > 1024)
+        return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
+    // launch bound: 2 CTAs of 256 threads per SM by default (<= 128 registers;
+    // measured on C2: ptxas needs ~80, more CTAs hide the MUFU latency)
+    jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 512 / jo.block);
+    if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
+    JitProgram jp;
+    std::string msg;
+    int rc = generate_jit(g, jo, jp, msg);
+    if (rc != SPN_OK) return set_err(rc, msg);
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    if (major < 10) return set_err(SPN_E_UNSUPPORTED, "compiled path targets sm_100a (B200)");
+    const std::string arch = std::to_string(major * 10 + minor) + "a";
+    const auto tc0 = std::chrono::steady_clock::now();
+    const size_t T = jp.tasks.size();
+    // 2T assembly jobs (joint + marginal module per task) on all host cores
+    std::vector<std::vector<char>> cubins(2 * T);
+    std::vector<std::string> logs(2 * T);
+    std::vector<int> rcs(2 * T, SPN_OK);
+    {
+        const size_t J = 2 * T;
+        const size_t nthreads = std::max<size_t>(1, std::min<size_t>(J, std::thread::hardware_concurrency()));
+        std::atomic<size_t> next{0};
+        std::vector<std::thread> th;
+        for (size_t i = 0; i < nthreads; ++i)
+            th.emplace_back([&] {
+                for (size_t j; (j = next++) < J;)
+                    rcs[j] = jit_compile(jp.tasks[j / 2].ptx[j % 2], arch, cubins[j], logs[j]);
+            });
+        for (auto &x : th) x.join();
+    }
+    for (size_t j = 0; j < 2 * T; ++j)
+        if (rcs[j] != SPN_OK) return set_err(rcs[j], "compiled path: " + logs[j].substr(0, 2000));
+    const double compile_ms =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tc0).count();
+    DevicePlan *P = new (std::nothrow) DevicePlan();
+    if (!P) return set_err(SPN_E_OOM, "plan");
+    P->device = dev;
+    P->path = 2;
+    P->F = g.F;
+    P->R = (int32_t)g.roots.size();
+    P->sms = sms;
+    P->jblock = jo.block;
+    P->jfused_argmax = jp.fused_argmax;
+    P->block = jo.block;
+    int max_regs = 0, min_occ = 1 << 30;
+    for (size_t t = 0; t < T; ++t) {
+        P->jk.push_back(JitKernel());
+        JitKernel &k = P->jk.back();
+        for (int v = 0; v < 2; ++v)
+            if ((rc = jit_load(cubins[2 * t + v], jp.tasks[t].name, v, jo.block, k, msg)) != SPN_OK) {
+                free_plan(P);
+                return set_err(rc, msg);
+            }
+        const int occ = std::max(1, std::min(k.occupancy[0], k.occupancy[1]));
+        // grid-stride loop over samples: a few waves of resident CTAs
+        P->jgrid_max.push_back(sms * occ * 4);
+        max_regs = std::max({max_regs, k.regs[0], k.regs[1]});
+        min_occ = std::min(min_occ, occ);
+    }
+    if ((rc = upload(&P->d_jtab, jp.tables))) {
+        free_plan(P);
+        return rc;
+    }
+    spn_plan_stats &s = P->stats;
+    memset(&s, 0, sizeof(s));
+    s.n_nodes = jp.n_nodes;
+    s.n_leaves = jp.n_leaves;
+    s.n_sums = jp.n_sums;
+    s.n_products = jp.n_products;
+    s.n_sum_edges = jp.n_sum_edges;
+    s.n_tasks = (int64_t)T;
+    s.mufu_per_sample = jp.mufu_per_sample;
+    s.fma_per_sample = jp.fma_per_sample;
+    s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)g.roots.size();
+    s.path = 2;
+    s.block_threads = jo.block;
+    s.samples_per_thread = 1;
+    s.grid = P->jgrid_max.empty() ? 0 : P->jgrid_max[0];
+    s.x_in_smem = 0;
+    s.kernel_regs = max_regs;
+    s.ctas_per_sm = min_occ;
+    s.mufu_exec_per_sample = jp.mufu_exec_per_sample;
+    s.compile_ms = compile_ms;
     s.prepare_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     spn_handle *h = new (std::nothrow) spn_handle();
@@ -502,8 +640,10 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     spn_prepare_options opt;
     spn_default_options(&opt);
     if (opt_in) opt = *opt_in;
-    for (int i = 0; i < 8; ++i)
+    for (int i = 0; i < 7; ++i)
         if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
+    if (opt.compiled_path < 0 || opt.compiled_path > 2)
+        return set_err(SPN_E_ARG, "compiled_path must be 0 (auto), 1 (off) or 2 (force)");
     const auto t0 = std::chrono::steady_clock::now();
     const GraphData &g = *graph->graph;
 
@@ -540,6 +680,16 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         if (!lp.ok && opt.layered_path == 2)
             return set_err(SPN_E_UNSUPPORTED, "layered path not applicable: " + lp.why);
         if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, wbufs, t0, out_plan);
+    }
+    // ---- compiled path: one generated straight-line kernel per task ----
+    // auto: used unless the caller pins interpreter parameters
+    // (samples_per_thread / max_task_nodes) or a component is too large
+    if (opt.compiled_path == 2 ||
+        (opt.compiled_path == 0 && opt.samples_per_thread == 0 && opt.max_task_nodes == 0)) {
+        const int rc = prepare_compiled(g, opt, dev, sms, t0, out_plan);
+        if (rc == SPN_OK || opt.compiled_path == 2 || rc == SPN_E_ARG || rc == SPN_E_OOM) return rc;
+        // SPN_E_UNSUPPORTED / SPN_E_CUDA from the compiler or loader: the
+        // interpreter kernel (also sm_100a, not a CPU path) serves the graph
     }
     // auto: K = 2 samples/thread with up to 24 warps when 16+ warps' feature
     // tiles fit in shared memory (more warps hide the interpreter's latency),
@@ -790,6 +940,43 @@ int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, i
     if (fparams) memcpy(fparams, lp.fparams.data(), lp.fparams.size() * 4);
     if (wimg) memcpy(wimg, lp.wimg.data(), lp.wimg.size() * 2);
     if (root_map) memcpy(root_map, lp.root_map.data(), lp.root_map.size() * 4);
+    return SPN_OK;
+}
+
+int spn_codegen(const spn_handle *graph, int32_t task, int32_t lang, char *src, int64_t *src_len,
+                char *name, int32_t *roots, int32_t *n_roots, float *tables, int64_t *n_tables,
+                int32_t *n_tasks, int32_t compile, const char *arch) {
+    if (!valid_graph_handle(graph) || !src_len || !n_roots || !n_tables || !n_tasks)
+        return set_err(SPN_E_ARG, "bad arguments");
+    JitOptions jo;
+    JitProgram jp;
+    std::string msg;
+    int rc = generate_jit(*graph->graph, jo, jp, msg);
+    if (rc != SPN_OK) return set_err(rc, msg);
+    *n_tasks = (int32_t)jp.tasks.size();
+    if (task < 0 || task >= (int32_t)jp.tasks.size()) return set_err(SPN_E_ARG, "task out of range");
+    const JitTask &t = jp.tasks[task];
+    const std::string &text = lang == 1 ? t.source : t.cpp;
+    if (src) {
+        if (*src_len < (int64_t)text.size() + 1 || *n_roots < (int32_t)t.roots.size() ||
+            *n_tables < (int64_t)jp.tables.size() || !roots || !tables)
+            return set_err(SPN_E_ARG, "buffers too small");
+        memcpy(src, text.c_str(), text.size() + 1);
+        memcpy(roots, t.roots.data(), t.roots.size() * 4);
+        memcpy(tables, jp.tables.data(), jp.tables.size() * 4);
+        if (name) snprintf(name, 64, "%s", t.name.c_str());
+    }
+    *src_len = (int64_t)text.size() + 1;
+    *n_roots = (int32_t)t.roots.size();
+    *n_tables = (int64_t)jp.tables.size();
+    if (compile) {
+        std::vector<char> cubin;
+        std::string log;
+        for (int v = 0; v < 2; ++v) {
+            rc = jit_compile(t.ptx[v], arch ? arch : "100a", cubin, log);
+            if (rc != SPN_OK) return set_err(rc, log);
+        }
+    }
     return SPN_OK;
 }
 

@@ -260,3 +260,50 @@ def test_layered_ragged_and_chunked():
     idx = np.concatenate([np.arange(0, 50), np.arange(37_850, 37_950), np.arange(79_950, 80_001)])
     ref, _ = oracle_eval(g, x[idx])
     _cmp(out[idx], ref)
+
+
+# ----------------------------------------------------------------- compiled path (KS)
+def test_compiled_path_is_default_for_speaker_spn():
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 20_000, 41)
+    x = add_outliers(x, 0.01, 42)
+    err, P = _parity(g, x)
+    info = P.info()
+    assert info["path"] == 2 and info["n_tasks"] == 1, info
+    _parity(g, nan_mask(x, 0.2, 43), marginal=True)
+
+
+def test_compiled_matches_interpreter():
+    g = speaker_spn(2002)
+    x, _ = ancestral_sample(g, 10_000, 44)
+    a, _, Pa = _run(g, x, compiled_path=2)
+    b, _, Pb = _run(g, x, compiled_path=1)
+    assert Pa.info()["path"] == 2 and Pb.info()["path"] == 0
+    _cmp(a, b.astype(np.float64), tol=2e-6)
+
+
+def test_compiled_multi_task_argmax():
+    g = speaker_set(list(range(3001, 3009)))          # 8 components -> several tasks
+    x, _ = ancestral_sample(g, 5000, 45)
+    err, P = _parity(g, nan_mask(x, 0.2, 46), marginal=True, compiled_path=2)
+    assert P.info()["path"] == 2 and P.info()["n_tasks"] > 1
+
+
+def test_compiled_edge_values():
+    g = speaker_spn(2001)
+    x, _ = ancestral_sample(g, 512, 47)
+    x[0, 3] = np.inf
+    x[1, 5] = -np.inf
+    x[2, 7] = np.nan
+    x[3, :] = np.nan
+    x[4, 1] = 1e15
+    for marginal in (False, True):
+        _parity(g, x, marginal=marginal, compiled_path=2)
+
+
+@pytest.mark.parametrize("n", [1, 31, 255, 257, 100_003])
+def test_compiled_ragged(n):
+    g = toy_spn()
+    x = toy_data(n, seed=n)
+    _parity(g, x, compiled_path=2)
+    _parity(g, nan_mask(x, 0.3, n), marginal=True, compiled_path=2)

@@ -25,7 +25,8 @@ struct JitOptions {
     int block = 256;             // threads per CTA (launch bound)
     int min_blocks = 2;          // __launch_bounds__ min CTAs per SM (register cap)
     int64_t task_cap_nodes = 3000;  // pack connected components up to this size
-    int64_t max_task_nodes = 60000; // larger components: compiled path unsupported
+    int64_t max_task_nodes = 16000; // larger components: compiled path unsupported
+                                    // (ptxas time and register spills grow with size)
 };
 
 struct JitTask {

@@ -2,7 +2,7 @@
 # compiled path: GPU tests, bench lines C1/C2/C2m/C3m, ncu launch list + full capture of the generated kernel
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 O=gpurun_out; mkdir -p $O
-timeout 900 python -m pytest tests -m gpu -q -x --timeout 400 > $O/pytest_gpu.log 2>&1; echo "pytest=$?" >> $O/status.txt
+timeout 1500 python -m pytest tests -m gpu -q --timeout 600 --durations=15 > $O/pytest_gpu.log 2>&1; echo "pytest=$?" >> $O/status.txt
 for c in C2 C1; do
   timeout 600 python bench.py --config $c > $O/bench_$c.log 2>&1; echo "bench_$c=$?" >> $O/status.txt
 done

@@ -524,8 +524,10 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
                 return set_err(rc, msg);
             }
         const int occ = std::max(1, std::min(k.occupancy[0], k.occupancy[1]));
-        // grid-stride loop over samples: a few waves of resident CTAs
-        P->jgrid_max.push_back(sms * occ * 4);
+        // grid-stride loop over samples with exactly one wave of resident CTAs:
+        // every thread gets ceil or floor of n / threads samples (measured on
+        // C2: 4 waves left SMs idle for up to one extra iteration per CTA)
+        P->jgrid_max.push_back(sms * occ);
         max_regs = std::max({max_regs, k.regs[0], k.regs[1]});
         min_occ = std::min(min_occ, occ);
     }

@@ -88,7 +88,10 @@ typedef struct spn_prepare_options {
                                    compilation, §IV-C).
                                    Auto uses it for non-layered graphs unless
                                    samples_per_thread / max_task_nodes are set
-                                   (interpreter knobs) or compilation fails  */
+                                   (interpreter knobs), a task keeps more than
+                                   64 values live at once (register pressure:
+                                   region-graph cross products) or
+                                   compilation fails                          */
     int32_t reserved[7];        /* must be zero                                */
 } spn_prepare_options;
 

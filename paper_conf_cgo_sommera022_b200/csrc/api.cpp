@@ -477,6 +477,13 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     std::string msg;
     int rc = generate_jit(g, jo, jp, msg);
     if (rc != SPN_OK) return set_err(rc, msg);
+    if (opt.compiled_path == 0)
+        for (const JitTask &t : jp.tasks)
+            if (t.max_live > jo.max_live_auto)
+                return set_err(SPN_E_UNSUPPORTED, "compiled path: " + std::to_string(t.max_live) +
+                                                      " values live at once in " + t.name +
+                                                      " (auto limit " +
+                                                      std::to_string(jo.max_live_auto) + ")");
     int major = 0, minor = 0;
     cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
     cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);

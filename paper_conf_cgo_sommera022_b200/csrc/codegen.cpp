@@ -37,6 +37,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <numeric>
@@ -94,6 +95,7 @@ struct Ir {
     std::vector<Ins> ins;
     int32_t nreg = 0;
     bool marg = false;
+    size_t n_prologue = 0;  // leading instructions that load / prepare features
     std::vector<int32_t> argmax_roots;
 
     Opnd imm(double v) {
@@ -506,6 +508,33 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
     return s;
 }
 
+// Largest number of simultaneously live SSA values of the inner nodes when
+// the IR is executed in emission order (feature registers excluded: they are
+// few and ptxas rematerialises them).  A proxy for the register pressure
+// ptxas faces; straight-line code over region graphs (RAT-SPN cross
+// products) reaches hundreds, where assembly time explodes.
+int64_t ir_max_live(const Ir &ir) {
+    std::vector<int64_t> last(ir.nreg, -1);
+    std::vector<uint8_t> feat(ir.nreg, 0);
+    for (size_t k = 0; k < ir.ins.size(); ++k) {
+        const Ins &i = ir.ins[k];
+        for (const Opnd *o : {&i.a, &i.b, &i.c})
+            if (o->reg >= 0) last[o->reg] = (int64_t)k;
+        if (i.d >= 0 && k < ir.n_prologue) feat[i.d] = 1;
+    }
+    std::vector<int32_t> dies(ir.ins.size() + 1, 0);
+    for (int32_t r = 0; r < ir.nreg; ++r)
+        if (!feat[r] && last[r] >= 0) dies[last[r]]++;
+    int64_t live = 0, best = 0;
+    for (size_t k = 0; k < ir.ins.size(); ++k) {
+        const Ins &i = ir.ins[k];
+        live -= dies[k];
+        if (i.d >= 0 && !feat[i.d] && last[i.d] >= 0) ++live;
+        best = std::max(best, live);
+    }
+    return best;
+}
+
 }  // namespace
 
 int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std::string &msg) {
@@ -687,6 +716,7 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
                 }
                 if (use_d[f]) F.d = ir.marg ? ir.emit(I_SELNAN, R(F.x), ir.imm(0.0), R(xm)) : xm;
             }
+            ir.n_prologue = ir.ins.size();
             for (int64_t u : tnodes[t]) {
                 if (c.kind[u] == SPN_PRODUCT) tg.product(u);
                 else if (c.kind[u] == SPN_SUM) tg.sum(u);
@@ -707,6 +737,10 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
                 ir.ins.push_back(a);
             }
             const std::string suffix = marg ? "_m" : "_j";
+            jt.max_live = std::max(jt.max_live, ir_max_live(ir));
+            if (getenv("SPNB_JIT_VERBOSE"))
+                fprintf(stderr, "[spnb] task %d marg %d: %zu ins, max_live %lld\n", t, marg, ir.ins.size(),
+                        (long long)ir_max_live(ir));
             jt.ptx[marg] = ptx_head + emit_ptx_entry(ir, jt.name + suffix, opt.block, opt.min_blocks);
             cpp += emit_cpp(ir, jt.name + suffix + "_body");
         }

@@ -27,6 +27,9 @@ struct JitOptions {
     int64_t task_cap_nodes = 3000;  // pack connected components up to this size
     int64_t max_task_nodes = 16000; // larger components: compiled path unsupported
                                     // (ptxas time and register spills grow with size)
+    int64_t max_live_auto = 64;     // auto selection: larger ir_max_live stays on the
+                                    // interpreter (RAT-SPN cross products: hundreds of live
+                                    // values, ptxas takes minutes and the kernel spills)
 };
 
 struct JitTask {
@@ -38,6 +41,7 @@ struct JitTask {
     std::vector<int32_t> roots;  // output columns written by this task
     int64_t n_nodes = 0;         // canonical nodes evaluated (leaves included)
     int64_t n_features = 0;      // distinct features read
+    int64_t max_live = 0;        // ir_max_live: inner values live at once (register pressure proxy)
 };
 
 struct JitProgram {

@@ -33,27 +33,8 @@ int dag_eval_occupancy_k8(bool, bool, int, size_t);
 int dag_eval_occupancy_k1(bool, bool, int, size_t);
 int dag_eval_occupancy_k2(bool, bool, int, size_t);
 int dag_eval_occupancy_k4(bool, bool, int, size_t);
-struct RParams {
-    const LStep *steps;
-    int32_t n_steps;
-    int32_t C;
-    const int32_t *vars;
-    const float *fparams;
-    const uint8_t *wimg;
-    const int32_t *root_map;
-    const float *xT;
-    int64_t ldT;
-    int64_t n;
-    float *out;
-    int32_t *argmax;
-    int32_t prec;
-    int32_t smem_floats, max_kpad, max_ngroup, max_na;
-    int32_t max_vars;
-    int32_t first_leaf;
-    int32_t max_leaf_params;
-    int32_t wbufs;
-    unsigned long long *prof;
-};
+// RParams: layered.h
+
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,
                       int max_vars, int max_leaf_params, int prec, int wbufs);
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
@@ -117,11 +98,13 @@ struct DevicePlan {
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
     int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
+    int32_t tmem_overlap = 0;  // SPNB_TMEM_OVERLAP=1: epilogue under the next MMA (A/B)
     unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
     // compiled (per-SPN generated kernel) path
     std::vector<JitKernel> jk;
     std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM x waves
     int jblock = 256;
+    int jK = 1;  // samples per thread of the generated kernels
     bool jfused_argmax = false;
     float *d_jtab = nullptr;
     spn_plan_stats stats;
@@ -239,7 +222,7 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         std::string msg;
         const int32_t *tasks_am = P.jfused_argmax ? argmax : nullptr;
         for (size_t t = 0; t < P.jk.size(); ++t) {
-            const int64_t need = (n + P.jblock - 1) / P.jblock;
+            const int64_t need = (n + (int64_t)P.jblock * P.jK - 1) / ((int64_t)P.jblock * P.jK);
             const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, P.jgrid_max[t]));
             const int rc = jit_launch(P.jk[t], marg, grid, P.jblock, (cudaStream_t)stream, x, n, ld,
                                       out, P.R, (int *)tasks_am, P.d_jtab, msg);
@@ -272,6 +255,7 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         rp.first_leaf = P.first_leaf;
         rp.max_leaf_params = P.max_leaf_params;
         rp.wbufs = P.wbufs;
+        rp.overlap = P.tmem_overlap;
         rp.prof = P.d_prof;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
@@ -395,6 +379,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     P->first_leaf = lp.first_leaf;
     P->max_leaf_params = lp.max_leaf_params;
     P->wbufs = wbufs;
+    if (const char *ev = getenv("SPNB_TMEM_OVERLAP")) P->tmem_overlap = atoi(ev) != 0;
     // transposed-feature scratch: chunks small enough (<= ~48 MB) that the
     // tile slices re-read by every repetition stay resident in L2
     // (a multiple of one full wave of 128-sample tiles: 148 SMs x 128)
@@ -469,10 +454,12 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     jo.block = opt.block_threads ? opt.block_threads : 256;
     if (jo.block % 32 || jo.block < 32 || jo.block > 1024)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
-    // launch bound: 2 CTAs of 256 threads per SM by default (<= 128 registers;
-    // measured on C2: ptxas needs ~80, more CTAs hide the MUFU latency)
-    jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 512 / jo.block);
+    // launch bound: 3 CTAs of 256 threads per SM by default (<= 80 registers;
+    // measured on C2: 2.87e9 samples/s at 3 x 256 (80 regs, no spills) vs
+    // 2.83e9 at 2 x 256 (128 regs) and 2.56e9 at 6 x 128)
+    jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 768 / jo.block);
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
+    if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
     JitProgram jp;
     std::string msg;
     int rc = generate_jit(g, jo, jp, msg);
@@ -519,6 +506,7 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     P->R = (int32_t)g.roots.size();
     P->sms = sms;
     P->jblock = jo.block;
+    P->jK = jo.samples_per_thread;
     P->jfused_argmax = jp.fused_argmax;
     P->block = jo.block;
     int max_regs = 0, min_occ = 1 << 30;
@@ -555,7 +543,7 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)g.roots.size();
     s.path = 2;
     s.block_threads = jo.block;
-    s.samples_per_thread = 1;
+    s.samples_per_thread = jo.samples_per_thread;
     s.grid = P->jgrid_max.empty() ? 0 : P->jgrid_max[0];
     s.x_in_smem = 0;
     s.kernel_regs = max_regs;
@@ -673,7 +661,9 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         const int prec = opt.tc_precision == 1 ? 1 : 3;
         // prefer double-buffered weight groups (N <= 240, else N <= 120 per
         // group), then serial groups
-        for (int attempt = 0; attempt < 3 && wbufs == 0; ++attempt) {
+        int first_attempt = 0;  // SPNB_LAYERED_ATTEMPT: 1 = N<=120 groups, 2 = serial (A/B)
+        if (const char *ev = getenv("SPNB_LAYERED_ATTEMPT")) first_attempt = std::min(2, std::max(0, atoi(ev)));
+        for (int attempt = first_attempt; attempt < 3 && wbufs == 0; ++attempt) {
             const int n_cap = attempt == 1 ? 120 : 240;
             const int wb = attempt == 2 ? 1 : 2;
             detect_layered(g, lp, n_cap);
@@ -958,6 +948,8 @@ int spn_codegen(const spn_handle *graph, int32_t task, int32_t lang, char *src, 
     if (!valid_graph_handle(graph) || !src_len || !n_roots || !n_tables || !n_tasks)
         return set_err(SPN_E_ARG, "bad arguments");
     JitOptions jo;
+    if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
+    if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
     JitProgram jp;
     std::string msg;
     int rc = generate_jit(*graph->graph, jo, jp, msg);

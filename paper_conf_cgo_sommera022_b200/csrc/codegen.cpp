@@ -363,23 +363,32 @@ static inline float spnb_disc(float x, long long lo, long long K, const float *t
 
 // ---------------------------------------------------------------------------
 // PTX back end (sm_100a).
-std::string ptx_opnd(const Opnd &o) {
-    if (o.reg >= 0) return "%f" + std::to_string(o.reg);
+std::string ptx_opnd(const Opnd &o, const char *pf) {
+    if (o.reg >= 0) return pf + std::to_string(o.reg);
     char b[16];
     snprintf(b, sizeof(b), "0f%08X", fbits(o.imm));
     return b;
 }
 
-std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int min_blocks) {
+// Register-file prefix of sample slot j (K samples per thread interleave
+// instruction by instruction: K independent copies of the body for ILP and
+// K samples per instruction fetch).
+const char *kSlotPrefix[4] = {"%f", "%g", "%h", "%k"};
+
+std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int min_blocks,
+                           int K) {
     std::string body;
-    body.reserve(ir.ins.size() * 48);
+    body.reserve(ir.ins.size() * 48 * K);
     char b[4096];
     int np = 0, nr = 0, nd = 0;  // predicate / b32 / b64 temporaries
     for (const Ins &i : ir.ins) {
-        const std::string d = "%f" + std::to_string(i.d), a = ptx_opnd(i.a), bb = ptx_opnd(i.b),
-                          cc = ptx_opnd(i.c);
+      for (int j = 0; j < K; ++j) {
+        const char *pf = kSlotPrefix[j];
+        const std::string d = pf + std::to_string(i.d), a = ptx_opnd(i.a, pf), bb = ptx_opnd(i.b, pf),
+                          cc = ptx_opnd(i.c, pf);
+        const std::string xr = "%xr" + std::to_string(j), orow = "%orow" + std::to_string(j);
         switch (i.op) {
-            case I_LDX: snprintf(b, sizeof(b), "ld.global.nc.f32 %s, [%%xr+%lld];", d.c_str(), (long long)i.aux * 4); break;
+            case I_LDX: snprintf(b, sizeof(b), "ld.global.nc.f32 %s, [%s+%lld];", d.c_str(), xr.c_str(), (long long)i.aux * 4); break;
             case I_MOV: snprintf(b, sizeof(b), "mov.f32 %s, %s;", d.c_str(), a.c_str()); break;
             case I_FMA: snprintf(b, sizeof(b), "fma.rn.f32 %s, %s, %s, %s;", d.c_str(), a.c_str(), bb.c_str(), cc.c_str()); break;
             case I_ADD: snprintf(b, sizeof(b), "add.rn.f32 %s, %s, %s;", d.c_str(), a.c_str(), bb.c_str()); break;
@@ -398,7 +407,7 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
             }
             case I_SELINF: {
                 const int p = np++;
-                const std::string t = "%f" + std::to_string(ir.nreg + (int)(&i - ir.ins.data()));
+                const std::string t = pf + std::to_string(ir.nreg + (int)(&i - ir.ins.data()));
                 snprintf(b, sizeof(b), "abs.f32 %s, %s; setp.eq.f32 %%p%d, %s, 0f7F800000; selp.f32 %s, %s, %s, %%p%d;",
                          t.c_str(), a.c_str(), p, t.c_str(), d.c_str(), bb.c_str(), cc.c_str(), p);
                 break;
@@ -424,24 +433,26 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
                 break;
             }
             case I_OUT: {
-                const std::string t = "%f" + std::to_string(ir.nreg + (int)(&i - ir.ins.data()));
-                snprintf(b, sizeof(b), "mul.rn.f32 %s, %s, 0f3F317218; st.global.f32 [%%orow+%lld], %s;",
-                         t.c_str(), a.c_str(), (long long)i.aux * 4, t.c_str());
+                const std::string t = pf + std::to_string(ir.nreg + (int)(&i - ir.ins.data()));
+                snprintf(b, sizeof(b), "mul.rn.f32 %s, %s, 0f3F317218; @%%pv%d st.global.f32 [%s+%lld], %s;",
+                         t.c_str(), a.c_str(), j, orow.c_str(), (long long)i.aux * 4, t.c_str());
                 break;
             }
             case I_ARGMAX: {
                 // best / idx in registers; strict > keeps the lowest index on ties
-                std::string t = "setp.ne.s64 %pam, %amp, 0; @!%pam bra $Lskip_am; mov.f32 %fbest, 0fFF800000; mov.s32 %ridx, -1;";
+                std::string t = "setp.ne.s64 %pam, %amp, 0; and.pred %pam, %pam, %pv" + std::to_string(j) +
+                                "; @!%pam bra $Lskip_am" + std::to_string(j) +
+                                "; mov.f32 %fbest, 0fFF800000; mov.s32 %ridx, -1;";
                 for (int32_t r : ir.argmax_roots) {
                     char q[512];
                     snprintf(q, sizeof(q),
-                             " ld.global.f32 %%fw, [%%orow+%d]; setp.num.f32 %%pa, %%fw, %%fw; "
+                             " ld.global.f32 %%fw, [%s+%d]; setp.num.f32 %%pa, %%fw, %%fw; "
                              "setp.lt.s32 %%pb, %%ridx, 0; setp.gt.or.f32 %%pb, %%fw, %%fbest, %%pb; "
                              "and.pred %%pb, %%pb, %%pa; @%%pb mov.f32 %%fbest, %%fw; @%%pb mov.s32 %%ridx, %d;",
-                             r * 4, r);
+                             orow.c_str(), r * 4, r);
                     t += q;
                 }
-                t += " st.global.s32 [%amrow], %ridx; $Lskip_am:";
+                t += " st.global.s32 [%amrow" + std::to_string(j) + "], %ridx; $Lskip_am" + std::to_string(j) + ":";
                 body += "    " + t + "\n";
                 continue;
             }
@@ -449,6 +460,7 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
         body += "    ";
         body += b;
         body += '\n';
+      }
     }
     // temporaries beyond the SSA values: one per I_SELINF / I_OUT instruction slot
     const int nf = ir.nreg + (int)ir.ins.size() + 1;
@@ -464,12 +476,19 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
              "    .reg .pred %%pl, %%pam, %%pa, %%pb;\n"
              "    .reg .b32 %%r<%d>;\n"
              "    .reg .b64 %%rd<%d>;\n"
-             "    .reg .f32 %%f<%d>;\n"
              "    .reg .f32 %%fbest, %%fw;\n"
              "    .reg .s32 %%ridx, %%rtid, %%rcta, %%rncta, %%R;\n"
-             "    .reg .b64 %%x, %%n, %%gld, %%out, %%amp, %%tab, %%s, %%stride, %%xr, %%orow, %%amrow, %%t64;\n",
-             name.c_str(), block, min_blocks, np + 1, nr + 1, nd + 1, nf);
+             "    .reg .b64 %%x, %%n, %%gld, %%out, %%amp, %%tab, %%s, %%stride, %%t64, %%sj;\n",
+             name.c_str(), block, min_blocks, np + 1, nr + 1, nd + 1);
     s += b;
+    for (int j = 0; j < K; ++j) {
+        snprintf(b, sizeof(b),
+                 "    .reg .f32 %s<%d>;\n"
+                 "    .reg .pred %%pv%d;\n"
+                 "    .reg .b64 %%xr%d, %%orow%d, %%amrow%d;\n",
+                 kSlotPrefix[j], nf, j, j, j, j);
+        s += b;
+    }
     snprintf(b, sizeof(b),
              "    ld.param.u64 %%x, [p_x];\n"
              "    ld.param.u64 %%n, [p_n];\n"
@@ -487,18 +506,28 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
              "    mul.wide.u32 %%stride, %%rncta, %d;\n"
              "$Lloop:\n"
              "    setp.ge.s64 %%pl, %%s, %%n;\n"
-             "    @%%pl bra $Ldone;\n"
-             "    mul.lo.s64 %%t64, %%s, %%gld;\n"
-             "    shl.b64 %%t64, %%t64, 2;\n"
-             "    add.s64 %%xr, %%x, %%t64;\n"
-             "    cvt.s64.s32 %%t64, %%R;\n"
-             "    mul.lo.s64 %%t64, %%s, %%t64;\n"
-             "    shl.b64 %%t64, %%t64, 2;\n"
-             "    add.s64 %%orow, %%out, %%t64;\n"
-             "    shl.b64 %%t64, %%s, 2;\n"
-             "    add.s64 %%amrow, %%amp, %%t64;\n",
-             block, block);
+             "    @%%pl bra $Ldone;\n",
+             block * K, block * K);
     s += b;
+    for (int j = 0; j < K; ++j) {
+        // slot j: sample s + j*block; past the end it recomputes sample s
+        // (valid) and its stores are predicated off
+        snprintf(b, sizeof(b),
+                 "    add.s64 %%sj, %%s, %d;\n"
+                 "    setp.lt.s64 %%pv%d, %%sj, %%n;\n"
+                 "    selp.b64 %%sj, %%sj, %%s, %%pv%d;\n"
+                 "    mul.lo.s64 %%t64, %%sj, %%gld;\n"
+                 "    shl.b64 %%t64, %%t64, 2;\n"
+                 "    add.s64 %%xr%d, %%x, %%t64;\n"
+                 "    cvt.s64.s32 %%t64, %%R;\n"
+                 "    mul.lo.s64 %%t64, %%sj, %%t64;\n"
+                 "    shl.b64 %%t64, %%t64, 2;\n"
+                 "    add.s64 %%orow%d, %%out, %%t64;\n"
+                 "    shl.b64 %%t64, %%sj, 2;\n"
+                 "    add.s64 %%amrow%d, %%amp, %%t64;\n",
+                 j * block, j, j, j, j, j);
+        s += b;
+    }
     s += body;
     s += "    add.s64 %s, %s, %stride;\n"
          "    bra $Lloop;\n"
@@ -741,7 +770,8 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
             if (getenv("SPNB_JIT_VERBOSE"))
                 fprintf(stderr, "[spnb] task %d marg %d: %zu ins, max_live %lld\n", t, marg, ir.ins.size(),
                         (long long)ir_max_live(ir));
-            jt.ptx[marg] = ptx_head + emit_ptx_entry(ir, jt.name + suffix, opt.block, opt.min_blocks);
+            jt.ptx[marg] = ptx_head + emit_ptx_entry(ir, jt.name + suffix, opt.block, opt.min_blocks,
+                                                       opt.samples_per_thread);
             cpp += emit_cpp(ir, jt.name + suffix + "_body");
         }
         char b[1024];

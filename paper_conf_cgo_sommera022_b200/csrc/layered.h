@@ -65,4 +65,30 @@ struct LayeredPlan {
 // n_cap: largest N (columns) of one MMA group (<= 240).
 void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap = 240);
 
+// Kernel parameters of rat_eval_kernel (rat_eval.cu), filled by api.cpp.
+struct RParams {
+    const LStep *steps;
+    int32_t n_steps;
+    int32_t C;
+    const int32_t *vars;
+    const float *fparams;
+    const uint8_t *wimg;
+    const int32_t *root_map;
+    const float *xT;
+    int64_t ldT;
+    int64_t n;
+    float *out;
+    int32_t *argmax;
+    int32_t prec;       // 1: single f16 pass; 3: hi/lo split
+    int32_t smem_floats, max_kpad, max_ngroup, max_na;
+    int32_t max_vars;   // largest leaf region (staged x rows)
+    int32_t first_leaf; // index of the first LEAF step
+    int32_t max_leaf_params;  // floats of the largest staged leaf parameter block
+    int32_t wbufs;      // 2: double-buffered weight groups; 1: single buffer
+    int32_t overlap;    // 1 (with wbufs 2): epilogue of group g-1 under MMA g (TMEM
+                        // ping-pong); 0: MMA g, then its epilogue (measured on C4:
+                        // TMEM reads under a running MMA are ~4.6x slower, so 0 wins)
+    unsigned long long *prof;  // optional phase-cycle counters (thread 0 of each CTA)
+};
+
 }  // namespace spnb

@@ -31,27 +31,7 @@
 
 namespace spnb {
 
-struct RParams {
-    const LStep *steps;
-    int32_t n_steps;
-    int32_t C;
-    const int32_t *vars;
-    const float *fparams;
-    const uint8_t *wimg;
-    const int32_t *root_map;
-    const float *xT;
-    int64_t ldT;
-    int64_t n;
-    float *out;
-    int32_t *argmax;
-    int32_t prec;       // 1: single f16 pass; 3: hi/lo split
-    int32_t smem_floats, max_kpad, max_ngroup, max_na;
-    int32_t max_vars;   // largest leaf region (staged x rows)
-    int32_t first_leaf; // index of the first LEAF step
-    int32_t max_leaf_params;  // floats of the largest staged leaf parameter block
-    int32_t wbufs;      // 2: double-buffered weight groups + TMEM ping-pong; 1: serial
-    unsigned long long *prof;  // optional phase-cycle counters (thread 0 of each CTA)
-};
+
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
 constexpr int RTH = 256;  // threads per CTA
@@ -208,11 +188,16 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
                     acc[d][k] = fmaf(-(nan ? cc : t), nan ? 1.f : t, acc[d][k]);
                 }
             } else {
-#pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    const float t = fmaf(q.x, xv[k], -q.y);
-                    acc[d][k] = fmaf(-t, t, acc[d][k]);
-                }
+                // packed FP32 (FFMA2, sm_100): two samples per instruction, the
+                // parameters broadcast (.F32) and -b folded as an operand modifier
+                const float2 a2 = make_float2(q.x, q.x), nb2 = make_float2(-q.y, -q.y);
+                const float2 t01 = __ffma2_rn(make_float2(xv[0], xv[1]), a2, nb2);
+                const float2 t23 = __ffma2_rn(make_float2(xv[2], xv[3]), a2, nb2);
+                const float2 s01 = __ffma2_rn(make_float2(-t01.x, -t01.y), t01,
+                                              make_float2(acc[d][0], acc[d][1]));
+                const float2 s23 = __ffma2_rn(make_float2(-t23.x, -t23.y), t23,
+                                              make_float2(acc[d][2], acc[d][3]));
+                acc[d][0] = s01.x; acc[d][1] = s01.y; acc[d][2] = s23.x; acc[d][3] = s23.y;
             }
         }
     }
@@ -265,7 +250,8 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     uint8_t *wsm = smem + off;   // [wbufs][prec==3 ? 2 : 1][n_group x kpad] f16
     const size_t w_part = (size_t)p.max_ngroup * p.max_kpad * 2;
     const size_t w_buf = w_part * (p.prec == 3 ? 2 : 1);
-    const uint32_t tmem_cols = p.wbufs == 2 ? 2 * TMEM_BUF : TMEM_BUF;
+    const bool ovl = p.wbufs == 2 && p.overlap;
+    const uint32_t tmem_cols = ovl ? 2 * TMEM_BUF : TMEM_BUF;
 
     const uint32_t bar_mma = r_smem(bars), bar_w0 = r_smem(bars + 1);
     const uint32_t bar_x0 = r_smem(bars + 3);
@@ -449,8 +435,16 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                                 }
                             }
                             tmem_wait_ld();
+                            // packed FP32 (FFMA2): 2 x 2 independent chains
+                            float2 p01 = make_float2(a4[0], a4[1]), p23 = make_float2(a4[2], a4[3]);
 #pragma unroll
-                            for (int i = 0; i < 32; ++i) a4[i & 3] = fmaf(ear[cb + i], t[i], a4[i & 3]);
+                            for (int i = 0; i < 32; i += 4) {
+                                p01 = __ffma2_rn(make_float2(ear[cb + i], ear[cb + i + 1]),
+                                                 make_float2(t[i], t[i + 1]), p01);
+                                p23 = __ffma2_rn(make_float2(ear[cb + i + 2], ear[cb + i + 3]),
+                                                 make_float2(t[i + 2], t[i + 3]), p23);
+                            }
+                            a4[0] = p01.x; a4[1] = p01.y; a4[2] = p23.x; a4[3] = p23.y;
                         }
                     }
                     const float acc = (a4[0] + a4[1]) + (a4[2] + a4[3]);
@@ -466,7 +460,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             };
             for (int g = 0; g < G; ++g) {
                 const int wb = p.wbufs == 2 ? (g & 1) : 0;
-                const uint32_t tb = p.wbufs == 2 ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
+                const uint32_t tb = ovl ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
                 mbar_wait(bar_w0 + 8 * wb, (ph_w >> wb) & 1u);
                 ph_w ^= 1u << wb;
                 prof_mark(4);  // 4: waiting for weights
@@ -489,7 +483,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 }
                 __syncwarp();
                 // overlap: the previous group's epilogue runs under this MMA
-                if (p.wbufs == 2 && g > 0) epilogue(g - 1, (uint32_t)((g - 1) & 1) * TMEM_BUF);
+                if (ovl && g > 0) epilogue(g - 1, (uint32_t)((g - 1) & 1) * TMEM_BUF);
                 prof_mark(5);  // 5: MMA issue + overlapped epilogue
                 mbar_wait(bar_mma, ph_mma);
                 ph_mma ^= 1;
@@ -497,11 +491,11 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 prof_mark(6);  // 6: waiting for the MMA
                 // the MMA has consumed weight buffer wb: refill it
                 if (tid == 0 && g + p.wbufs < G) issue_w(st, g + p.wbufs, wb);
-                if (p.wbufs == 1) epilogue(g, 0u);
+                if (!ovl) epilogue(g, 0u);
                 fence_before();
                 __syncthreads();
             }
-            if (p.wbufs == 2) {
+            if (ovl) {
                 epilogue(G - 1, (uint32_t)((G - 1) & 1) * TMEM_BUF);
                 fence_before();
                 __syncthreads();

@@ -102,7 +102,8 @@ struct DevicePlan {
     unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
     // compiled (per-SPN generated kernel) path
     std::vector<JitKernel> jk;
-    std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM x waves
+    std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM (joint kernel)
+    std::vector<int32_t> jgrid_max_m;       // per task: SMs x CTAs/SM (marginal kernel)
     int jblock = 256;
     int jK = 1;  // samples per thread of the generated kernels
     bool jfused_argmax = false;
@@ -223,7 +224,8 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         const int32_t *tasks_am = P.jfused_argmax ? argmax : nullptr;
         for (size_t t = 0; t < P.jk.size(); ++t) {
             const int64_t need = (n + (int64_t)P.jblock * P.jK - 1) / ((int64_t)P.jblock * P.jK);
-            const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, P.jgrid_max[t]));
+            const int grid = (int)std::max<int64_t>(
+                1, std::min<int64_t>(need, marg ? P.jgrid_max_m[t] : P.jgrid_max[t]));
             const int rc = jit_launch(P.jk[t], marg, grid, P.jblock, (cudaStream_t)stream, x, n, ld,
                                       out, P.R, (int *)tasks_am, P.d_jtab, msg);
             if (rc != SPN_OK) return set_err(rc, msg);
@@ -513,16 +515,40 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     for (size_t t = 0; t < T; ++t) {
         P->jk.push_back(JitKernel());
         JitKernel &k = P->jk.back();
-        for (int v = 0; v < 2; ++v)
+        for (int v = 0; v < 2; ++v) {
             if ((rc = jit_load(cubins[2 * t + v], jp.tasks[t].name, v, jo.block, k, msg)) != SPN_OK) {
                 free_plan(P);
                 return set_err(rc, msg);
             }
+            // auto launch bounds: a variant that spills at min_blocks CTAs/SM
+            // is regenerated with one CTA/SM fewer (measured on C2: the
+            // marginal kernel spills 720 B at 3 x 256 threads, 80 registers,
+            // and runs 11% slower than at 2 x 256 without spills)
+            for (int mb = jo.min_blocks - 1; k.local_bytes[v] > 0 && opt.ctas_per_sm <= 0 && mb >= 1; --mb) {
+                JitOptions jo2 = jo;
+                jo2.min_blocks = mb;
+                JitProgram jp2;
+                std::vector<char> cb;
+                std::string log;
+                if (generate_jit(g, jo2, jp2, msg) != SPN_OK ||
+                    jit_compile(jp2.tasks[t].ptx[v], arch, cb, log) != SPN_OK)
+                    break;
+                JitKernel k2;
+                if (jit_load(cb, jp2.tasks[t].name, v, jo.block, k2, msg) != SPN_OK) break;
+                jit_unload_variant(k, v);
+                k.module[v] = k2.module[v];
+                k.fn[v] = k2.fn[v];
+                k.regs[v] = k2.regs[v];
+                k.occupancy[v] = k2.occupancy[v];
+                k.local_bytes[v] = k2.local_bytes[v];
+            }
+        }
+        // grid-stride loop over samples with exactly one wave of resident CTAs
+        // (per variant): every thread gets ceil or floor of n / threads samples
+        // (measured on C2: 4 waves left SMs idle for up to one extra iteration)
         const int occ = std::max(1, std::min(k.occupancy[0], k.occupancy[1]));
-        // grid-stride loop over samples with exactly one wave of resident CTAs:
-        // every thread gets ceil or floor of n / threads samples (measured on
-        // C2: 4 waves left SMs idle for up to one extra iteration per CTA)
-        P->jgrid_max.push_back(sms * occ);
+        P->jgrid_max.push_back(sms * std::max(1, k.occupancy[0]));
+        P->jgrid_max_m.push_back(sms * std::max(1, k.occupancy[1]));
         max_regs = std::max({max_regs, k.regs[0], k.regs[1]});
         min_occ = std::min(min_occ, occ);
     }

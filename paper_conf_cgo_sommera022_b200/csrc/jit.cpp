@@ -185,6 +185,7 @@ int jit_load(const std::vector<char> &cubin, const std::string &name, int v, int
     }
     k.fn[v] = f;
     d.fn_attr(&k.regs[v], CU_FUNC_ATTRIBUTE_NUM_REGS, f);
+    d.fn_attr(&k.local_bytes[v], CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, f);
     d.occ(&k.occupancy[v], f, block, 0);
     return SPN_OK;
 }
@@ -204,12 +205,14 @@ int jit_launch(const JitKernel &k, bool marg, int grid, int block, cudaStream_t 
     return SPN_OK;
 }
 
+void jit_unload_variant(JitKernel &k, int v) {
+    if (k.module[v] && driver().ok) driver().unload((CUmodule)k.module[v]);
+    k.module[v] = nullptr;
+    k.fn[v] = nullptr;
+}
+
 void jit_unload(JitKernel &k) {
-    for (int v = 0; v < 2; ++v) {
-        if (k.module[v] && driver().ok) driver().unload((CUmodule)k.module[v]);
-        k.module[v] = nullptr;
-        k.fn[v] = nullptr;
-    }
+    for (int v = 0; v < 2; ++v) jit_unload_variant(k, v);
 }
 
 }  // namespace spnb

@@ -23,6 +23,7 @@ struct JitKernel {
     void *fn[2] = {nullptr, nullptr};      // CUfunction: [0] joint, [1] marginal
     int regs[2] = {0, 0};
     int occupancy[2] = {0, 0};  // CTAs per SM at the launch block size
+    int local_bytes[2] = {0, 0};  // per-thread local memory (> 0: register spills)
 };
 
 // Load variant v's cubin (0 joint, 1 marginal) into the current context and
@@ -34,5 +35,6 @@ int jit_launch(const JitKernel &k, bool marg, int grid, int block, cudaStream_t 
                const float *x, long long n, long long ld, float *out, int R, int *argmax,
                const float *tab, std::string &msg);
 void jit_unload(JitKernel &k);
+void jit_unload_variant(JitKernel &k, int v);  // one of the two modules
 
 }  // namespace spnb

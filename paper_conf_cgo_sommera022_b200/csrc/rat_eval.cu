@@ -149,11 +149,31 @@ __device__ __forceinline__ uint32_t img_off(int row, int k, int rows) {
     return (uint32_t)((k >> 3) * (rows * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
 }
 
+// NaN-propagating max of V[i][m] over i < n: four independent chains (the
+// loads of a chain issue back to back instead of one dependent max per load)
+__device__ __forceinline__ float col_max(const float *V, int n, int m) {
+    float h[4] = {-CUDART_INF_F, -CUDART_INF_F, -CUDART_INF_F, -CUDART_INF_F};
+    int i = 0;
+    for (; i + 4 <= n; i += 4) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) h[k] = r_maxnan(h[k], V[(i + k) * RT + m]);
+    }
+    for (; i < n; ++i) h[0] = r_maxnan(h[0], V[i * RT + m]);
+    return r_maxnan(r_maxnan(h[0], h[1]), r_maxnan(h[2], h[3]));
+}
+
 // LEAF step: the region's feature rows xs[v][m] (128 samples) and its
 // parameter block ab[v][i] = (a, b), C[i] are in shared memory (one bulk-copy
 // stage).  256 threads = 32 sample quads x 8 distribution groups of DPT =
 // I/8 distributions; per variable a thread does 1 LDS.128 (x) + DPT LDS.64
 // (broadcast) for 8 DPT FFMA.
+#ifndef LEAF_UNROLL
+#define LEAF_UNROLL 8
+#endif
+constexpr int kLeafUnroll = LEAF_UNROLL;
+#ifndef W_CHUNKS
+#define W_CHUNKS 1  // concurrent bulk copies per weight-group part
+#endif  // variable loop of a LEAF step
 template <int DPT, bool MARG>
 __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const float *xs,
                                             const float *prm, int tid) {
@@ -170,7 +190,7 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
     }
     // log2 N = c - t^2 with c = log2(a) + K0 (used only to cancel a NaN leaf)
     const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi)
-#pragma unroll 2
+#pragma unroll (kLeafUnroll)
     for (int v = 0; v < V; ++v) {
         const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + mq);
         const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
@@ -291,14 +311,25 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             bulk_g2s(dst + v * RT * 4, p.xT + (int64_t)f * p.ldT + base, RT * 4, bar);
         }
     };
-    auto issue_w = [&](const LStep &ws, int g, int b) {  // one thread
-        const size_t gb = (size_t)ws.w_group_bytes;
-        const uint8_t *src = p.wimg + ws.w_off + 2 * gb * g;
+    // weight group g of step ws -> buffer b; issued by the lanes of warp 0 as
+    // W_CHUNKS concurrent bulk copies per operand part (one large copy per
+    // part measured slower: the copies of one SM are serviced in parallel)
+    auto issue_w = [&](const LStep &ws, int g, int b) {
+        const uint32_t gb = (uint32_t)ws.w_group_bytes;
+        const uint8_t *src = p.wimg + ws.w_off + 2 * (size_t)gb * g;
         const uint32_t bar = bar_w0 + 8 * b;
         const uint32_t dst = r_smem(wsm) + (uint32_t)(b * w_buf);
-        mbar_expect_tx(bar, (uint32_t)(gb * (p.prec == 3 ? 2 : 1)));
-        bulk_g2s(dst, src, (uint32_t)gb, bar);
-        if (p.prec == 3) bulk_g2s(dst + (uint32_t)w_part, src + gb, (uint32_t)gb, bar);
+        const int parts = p.prec == 3 ? 2 : 1;
+        if (lane == 0) mbar_expect_tx(bar, gb * parts);
+        __syncwarp();
+        const uint32_t cb = ((gb + W_CHUNKS - 1) / W_CHUNKS + 15) & ~15u;  // 16-B multiple
+        for (int k = lane; k < W_CHUNKS * parts; k += 32) {
+            const int part = k / W_CHUNKS;
+            const uint32_t o = (uint32_t)(k % W_CHUNKS) * cb;
+            if (o < gb)
+                bulk_g2s(dst + (uint32_t)part * (uint32_t)w_part + o, src + (size_t)part * gb + o,
+                         min(cb, gb - o), bar);
+        }
     };
 
     const int64_t n_tiles = (p.n + RT - 1) / RT;
@@ -342,7 +373,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             }
             // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
             const int G = st.n_groups;
-            if (tid == 0) {
+            if (warp == 0) {
                 issue_w(st, 0, 0);
                 if (p.wbufs == 2 && G > 1) issue_w(st, 1, 1);
             }
@@ -350,16 +381,14 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             if (tid < RT) {
                 const int m = tid;
                 const float *VA = act + st.buf_a;
-                float hi = -CUDART_INF_F;
-                for (int i = 0; i < na; ++i) hi = r_maxnan(hi, VA[i * RT + m]);
+                const float hi = col_max(VA, na, m);
                 const float hc = fmaxf(hi, -1e30f);
                 for (int i = 0; i < na; ++i) ea[i * RT + m] = r_ex2(VA[i * RT + m] - hc);
                 sa[m] = hi;
             } else {
                 const int m = tid - RT;
                 const float *VB = act + st.buf_b;
-                float hi = -CUDART_INF_F;
-                for (int j = 0; j < nb; ++j) hi = r_maxnan(hi, VB[j * RT + m]);
+                const float hi = col_max(VB, nb, m);
                 const float hc = fmaxf(hi, -1e30f);
                 for (int j0 = 0; j0 < kpad; j0 += 8) {  // 8 k-values = one 16-byte row
                     uint32_t hw[4], lw[4];
@@ -490,7 +519,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 fence_after();
                 prof_mark(6);  // 6: waiting for the MMA
                 // the MMA has consumed weight buffer wb: refill it
-                if (tid == 0 && g + p.wbufs < G) issue_w(st, g + p.wbufs, wb);
+                if (warp == 0 && g + p.wbufs < G) issue_w(st, g + p.wbufs, wb);
                 if (!ovl) epilogue(g, 0u);
                 fence_before();
                 __syncthreads();

@@ -26,6 +26,7 @@
 #include <cuda_runtime.h>
 #include <math_constants.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "layered.h"
 
@@ -34,7 +35,7 @@ namespace spnb {
 
 
 constexpr int RT = 128;   // samples per tile (= UMMA M, = TMEM lanes)
-constexpr int RTH = 256;  // threads per CTA
+// threads per CTA: template parameter NTH of rat_eval_kernel (256 or 512)
 constexpr uint32_t TMEM_BUF = 256;  // columns per accumulator buffer
 
 __device__ __forceinline__ float r_ex2(float x) {
@@ -174,9 +175,52 @@ constexpr int kLeafUnroll = LEAF_UNROLL;
 #ifndef W_CHUNKS
 #define W_CHUNKS 1  // concurrent bulk copies per weight-group part
 #endif  // variable loop of a LEAF step
+// 512-thread mapping: 64 sample pairs x 8 distribution groups of DPT; per
+// variable 1 LDS.64 (x pair) + DPT LDS.64 (broadcast (a, b)) for 2 DPT FFMA2.
 template <int DPT, bool MARG>
+__device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, const float *xs,
+                                                const float *prm, int tid) {
+    const int I = st.n_out, V = st.n_vars;
+    const int mp = (tid & 63) * 2;           // 2 samples
+    const int d0 = (tid >> 6) * DPT;         // first distribution
+    const float2 *ab = reinterpret_cast<const float2 *>(prm);
+    const float *C = prm + 2 * V * I;
+    float2 acc[DPT];
+#pragma unroll
+    for (int d = 0; d < DPT; ++d) acc[d] = make_float2(C[d0 + d], C[d0 + d]);
+    const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi)
+#pragma unroll (kLeafUnroll)
+    for (int v = 0; v < V; ++v) {
+        const float2 x2 = *reinterpret_cast<const float2 *>(xs + v * RT + mp);
+        bool anynan = false;
+        if constexpr (MARG) anynan = (x2.x != x2.x) | (x2.y != x2.y);
+#pragma unroll
+        for (int d = 0; d < DPT; ++d) {
+            const float2 q = ab[v * I + d0 + d];
+            if (MARG && anynan) {
+                const float cc = r_lg2(q.x) + K0;
+                const float t0 = fmaf(q.x, x2.x, -q.y), t1 = fmaf(q.x, x2.y, -q.y);
+                const bool n0 = x2.x != x2.x, n1 = x2.y != x2.y;
+                acc[d].x = fmaf(-(n0 ? cc : t0), n0 ? 1.f : t0, acc[d].x);
+                acc[d].y = fmaf(-(n1 ? cc : t1), n1 ? 1.f : t1, acc[d].y);
+            } else {
+                const float2 t = __ffma2_rn(x2, make_float2(q.x, q.x), make_float2(-q.y, -q.y));
+                acc[d] = __ffma2_rn(make_float2(-t.x, -t.y), t, acc[d]);
+            }
+        }
+    }
+#pragma unroll
+    for (int d = 0; d < DPT; ++d)
+        *reinterpret_cast<float2 *>(act + st.buf_out + (d0 + d) * RT + mp) = acc[d];
+}
+
+template <int DPT, bool MARG, int NTH>
 __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const float *xs,
                                             const float *prm, int tid) {
+    if constexpr (NTH == 512) {
+        leaf_step_pairs<DPT, MARG>(st, act, xs, prm, tid);
+        return;
+    }
     const int I = st.n_out, V = st.n_vars;
     const int mq = (tid & 31) * 4;           // 4 samples
     const int d0 = (tid >> 5) * DPT;         // first distribution
@@ -227,22 +271,24 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
             make_float4(acc[d][0], acc[d][1], acc[d][2], acc[d][3]);
 }
 
-template <bool MARG>
+template <bool MARG, int NTH>
 __device__ void leaf_step(const LStep &st, float *act, const float *xs, const float *prm, int tid) {
     switch (st.n_out >> 3) {
-        case 1: leaf_step_t<1, MARG>(st, act, xs, prm, tid); break;
-        case 2: leaf_step_t<2, MARG>(st, act, xs, prm, tid); break;
-        case 3: leaf_step_t<3, MARG>(st, act, xs, prm, tid); break;
-        case 4: leaf_step_t<4, MARG>(st, act, xs, prm, tid); break;
-        case 5: leaf_step_t<5, MARG>(st, act, xs, prm, tid); break;
-        case 6: leaf_step_t<6, MARG>(st, act, xs, prm, tid); break;
-        case 7: leaf_step_t<7, MARG>(st, act, xs, prm, tid); break;
-        case 8: leaf_step_t<8, MARG>(st, act, xs, prm, tid); break;
+        case 1: leaf_step_t<1, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 2: leaf_step_t<2, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 3: leaf_step_t<3, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 4: leaf_step_t<4, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 5: leaf_step_t<5, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 6: leaf_step_t<6, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 7: leaf_step_t<7, MARG, NTH>(st, act, xs, prm, tid); break;
+        case 8: leaf_step_t<8, MARG, NTH>(st, act, xs, prm, tid); break;
     }
 }
 
-template <bool MARG>
-__global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
+template <bool MARG, int NTH>
+__global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
+    constexpr int NSPLIT = NTH / RT;    // epilogue: warps per TMEM lane quarter
+    constexpr int EA_MAX = NTH == 512 ? 48 : 64;  // ea values per thread in registers
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
@@ -346,7 +392,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
     if (warp == 0 && (int64_t)blockIdx.x < n_tiles) issue_x(p.first_leaf, (int64_t)blockIdx.x * RT, 0);
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const int64_t base = tile * RT;
-        for (int i = tid; i < p.C * RT; i += RTH) racc[i] = -CUDART_INF_F;
+        for (int i = tid; i < p.C * RT; i += NTH) racc[i] = -CUDART_INF_F;
         __syncthreads();
         for (int si = 0; si < p.n_steps; ++si) {
             const LStep st = p.steps[si];  // by value: fields live in registers
@@ -364,7 +410,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 xbuf ^= 1;
                 {
                     const float *stg = xsb + (size_t)b * stage_floats;
-                    leaf_step<MARG>(st, act, stg, stg + (size_t)p.max_vars * RT, tid);
+                    leaf_step<MARG, NTH>(st, act, stg, stg + (size_t)p.max_vars * RT, tid);
                 }
                 prof_mark(1);  // 1: leaf compute
                 __syncthreads();
@@ -385,7 +431,7 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                 const float hc = fmaxf(hi, -1e30f);
                 for (int i = 0; i < na; ++i) ea[i * RT + m] = r_ex2(VA[i * RT + m] - hc);
                 sa[m] = hi;
-            } else {
+            } else if (tid < 2 * RT) {
                 const int m = tid - RT;
                 const float *VB = act + st.buf_b;
                 const float hi = col_max(VB, nb, m);
@@ -422,24 +468,24 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
             // lanes 32q..32q+31 (= samples); the two warp halves split the sums
             // this thread's sample (TMEM lane quarter) and its ea values in
             // registers, reused by every sum of every group of this step
-            const int qd = warp & 3, half = warp >> 2;
+            const int qd = warp & 3, part = warp >> 2;
             const int m_ep = qd * 32 + lane;
-            float ear[64];
+            float ear[EA_MAX];
 #pragma unroll
-            for (int i = 0; i < 64; ++i) ear[i] = i < na ? ea[i * RT + m_ep] : 0.f;
+            for (int i = 0; i < EA_MAX; ++i) ear[i] = i < na ? ea[i * RT + m_ep] : 0.f;
             const float shift = sa[m_ep] + sb[m_ep];
             auto epilogue = [&](int g, uint32_t tb) {
                 const int m = m_ep;
                 const int s0 = g * st.s_per_group;
                 const int ns = min(st.s_per_group, st.n_out - s0);
-                const int hcut = (ns + 1) >> 1;
-                const int sl0 = half ? hcut : 0, sl1 = half ? ns : hcut;
+                // the NSPLIT warps of a lane quarter split the group's sums
+                const int sl0 = (ns * part) / NSPLIT, sl1 = (ns * (part + 1)) / NSPLIT;
                 for (int sl = sl0; sl < sl1; ++sl) {
                     // TMEM loads in batches of up to 32 columns, one wait per batch
                     const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
                     float a4[4] = {0.f, 0.f, 0.f, 0.f};  // 4 independent FMA chains
 #pragma unroll
-                    for (int cb = 0; cb < 64; cb += 32) {
+                    for (int cb = 0; cb < EA_MAX; cb += 32) {
                         if (cb < na) {
                             float t[32];
 #pragma unroll
@@ -468,10 +514,12 @@ __global__ void __launch_bounds__(RTH, 1) rat_eval_kernel(const RParams p) {
                             float2 p01 = make_float2(a4[0], a4[1]), p23 = make_float2(a4[2], a4[3]);
 #pragma unroll
                             for (int i = 0; i < 32; i += 4) {
-                                p01 = __ffma2_rn(make_float2(ear[cb + i], ear[cb + i + 1]),
-                                                 make_float2(t[i], t[i + 1]), p01);
-                                p23 = __ffma2_rn(make_float2(ear[cb + i + 2], ear[cb + i + 3]),
-                                                 make_float2(t[i + 2], t[i + 3]), p23);
+                                if (cb + i + 4 <= EA_MAX) {  // compile-time bound of ear[]
+                                    p01 = __ffma2_rn(make_float2(ear[cb + i], ear[cb + i + 1]),
+                                                     make_float2(t[i], t[i + 1]), p01);
+                                    p23 = __ffma2_rn(make_float2(ear[cb + i + 2], ear[cb + i + 3]),
+                                                     make_float2(t[i + 2], t[i + 3]), p23);
+                                }
                             }
                             a4[0] = p01.x; a4[1] = p01.y; a4[2] = p23.x; a4[3] = p23.y;
                         }
@@ -587,10 +635,18 @@ size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_
 }
 
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st) {
-    auto fn = marg ? rat_eval_kernel<true> : rat_eval_kernel<false>;
+    // 512 threads (16 warps) when the ea rows fit the 48-register epilogue
+    // array, else 256; SPNB_RAT_THREADS=256 pins the 8-warp variant (A/B)
+    static const int pin = [] {
+        const char *e = getenv("SPNB_RAT_THREADS");
+        return e ? atoi(e) : 0;
+    }();
+    const int nth = (pin == 256 || p.max_na > 48) ? 256 : 512;
+    auto fn = nth == 512 ? (marg ? rat_eval_kernel<true, 512> : rat_eval_kernel<false, 512>)
+                         : (marg ? rat_eval_kernel<true, 256> : rat_eval_kernel<false, 256>);
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    fn<<<grid, RTH, smem, st>>>(p);
+    fn<<<grid, nth, smem, st>>>(p);
     return cudaGetLastError();
 }
 

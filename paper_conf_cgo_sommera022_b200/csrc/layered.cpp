@@ -368,10 +368,14 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
             st.vars_off = (int64_t)plan.vars.size();
             plan.vars.insert(plan.vars.end(), reg.vars.begin(), reg.vars.end());
             // staged parameter block (16-byte aligned, one bulk copy):
-            //   ab[v][i] = (a, b) float2, then C[i] (padded to a multiple of 4)
+            //   ab[v][g][k] = (a, b) float2 (see below), then C[i] (padded to a multiple of 4)
             while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
             st.par_off = (int64_t)plan.fparams.size();
-            std::vector<float> ab((size_t)V * I * 2, 0.f);
+            // (a, b) pairs grouped by the kernel's 8 distribution groups of
+            // DPT = I/8: ab[v][g][k] = pair of distribution g*DPT + k, DPT
+            // padded to even so a thread loads two pairs per LDS.128
+            const int32_t DPT = I / 8, DPTp = DPT + (DPT & 1);
+            std::vector<float> ab((size_t)V * 8 * DPTp * 2, 0.f);
             std::vector<double> Cs(I, 0.0);
             for (int32_t i = 0; i < I; ++i) {
                 const int64_t u = reg.nodes[i];
@@ -386,7 +390,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
                     const double *pp = g.params.data() + g.param_begin[o];
                     const double a = 1.0 / (pp[1] * std::sqrt(2.0 * M_LN2));
                     Cs[i] += -std::log2(pp[1] * std::sqrt(2.0 * M_PI));
-                    const size_t idx = ((size_t)v * I + (size_t)i) * 2;
+                    const size_t idx = (((size_t)v * 8 + (size_t)(i / DPT)) * DPTp + (size_t)(i % DPT)) * 2;
                     ab[idx] = (float)a;
                     ab[idx + 1] = (float)(a * pp[0]);
                 }

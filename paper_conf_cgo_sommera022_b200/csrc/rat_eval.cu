@@ -182,9 +182,10 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
                                                 const float *prm, int tid) {
     const int I = st.n_out, V = st.n_vars;
     const int mp = (tid & 63) * 2;           // 2 samples
-    const int d0 = (tid >> 6) * DPT;         // first distribution
-    const float2 *ab = reinterpret_cast<const float2 *>(prm);
-    const float *C = prm + 2 * V * I;
+    const int grp = tid >> 6, d0 = grp * DPT; // distribution group, first distribution
+    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
+    const float *C = prm + (st.cst_off - st.par_off);
     float2 acc[DPT];
 #pragma unroll
     for (int d = 0; d < DPT; ++d) acc[d] = make_float2(C[d0 + d], C[d0 + d]);
@@ -194,9 +195,16 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
         const float2 x2 = *reinterpret_cast<const float2 *>(xs + v * RT + mp);
         bool anynan = false;
         if constexpr (MARG) anynan = (x2.x != x2.x) | (x2.y != x2.y);
+        float2 qv[DPTP];
+#pragma unroll
+        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * 4 * DPTP + k];
+            qv[2 * k] = make_float2(q4.x, q4.y);
+            qv[2 * k + 1] = make_float2(q4.z, q4.w);
+        }
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
-            const float2 q = ab[v * I + d0 + d];
+            const float2 q = qv[d];
             if (MARG && anynan) {
                 const float cc = r_lg2(q.x) + K0;
                 const float t0 = fmaf(q.x, x2.x, -q.y), t1 = fmaf(q.x, x2.y, -q.y);
@@ -223,9 +231,10 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
     }
     const int I = st.n_out, V = st.n_vars;
     const int mq = (tid & 31) * 4;           // 4 samples
-    const int d0 = (tid >> 5) * DPT;         // first distribution
-    const float2 *ab = reinterpret_cast<const float2 *>(prm);
-    const float *C = prm + 2 * V * I;
+    const int grp = tid >> 5, d0 = grp * DPT; // distribution group, first distribution
+    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
+    const float *C = prm + (st.cst_off - st.par_off);
     float acc[DPT][4];
 #pragma unroll
     for (int d = 0; d < DPT; ++d) {
@@ -240,9 +249,16 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
         const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
         bool anynan = false;
         if constexpr (MARG) anynan = (xv[0] != xv[0]) | (xv[1] != xv[1]) | (xv[2] != xv[2]) | (xv[3] != xv[3]);
+        float2 qv[DPTP];
+#pragma unroll
+        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * 4 * DPTP + k];
+            qv[2 * k] = make_float2(q4.x, q4.y);
+            qv[2 * k + 1] = make_float2(q4.z, q4.w);
+        }
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
-            const float2 q = ab[v * I + d0 + d];
+            const float2 q = qv[d];
             if (MARG && anynan) {
                 const float cc = r_lg2(q.x) + K0;
 #pragma unroll

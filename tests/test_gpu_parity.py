@@ -307,3 +307,30 @@ def test_compiled_ragged(n):
     x = toy_data(n, seed=n)
     _parity(g, x, compiled_path=2)
     _parity(g, nan_mask(x, 0.3, n), marginal=True, compiled_path=2)
+
+
+def test_compiled_auto_skips_region_graphs():
+    """Auto selection keeps RAT-SPN cross products (hundreds of live values)
+    off the compiled path: prepare stays fast and the interpreter serves the
+    graph (regression: ptxas took minutes on this graph)."""
+    import time
+    g = rat_spn(21, F=96, D=3, R=3, S=8, I=8, C=4)
+    x, _ = ancestral_sample(g, 500, 23)
+    t = time.perf_counter()
+    err, P = _parity(g, x, layered_path=1)
+    assert P.info()["path"] == 0
+    assert time.perf_counter() - t < 60
+
+
+def test_compiled_spill_fallback_marginal_full_size():
+    """Config-2 graph, marginal kernel: launched without register spills
+    (per-variant launch bounds), parity on a sample of a 1M-sample batch."""
+    from spn_inputs import config_graph
+    g = config_graph("C2")
+    x, _ = ancestral_sample(g, 1_000_000, 2002)
+    x = nan_mask(x, 0.2, 48)
+    out, _, P = _run(g, x, marginal=True)
+    assert P.info()["path"] == 2
+    idx = np.random.default_rng(1).choice(len(x), 2000, replace=False)
+    ref, _ = oracle_eval(g, x[idx], marginal=True)
+    _cmp(out[idx], ref)

@@ -98,7 +98,7 @@ struct DevicePlan {
     int32_t prec = 3;
     int32_t smem_floats = 0, max_kpad = 0, max_ngroup = 0, max_na = 0;
     int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
-    int32_t tmem_overlap = 0;  // SPNB_TMEM_OVERLAP=1: epilogue under the next MMA (A/B)
+    int32_t tmem_overlap = 1;  // epilogue of group g-1 under MMA g (SPNB_TMEM_OVERLAP=0: serial, A/B)
     unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
     // compiled (per-SPN generated kernel) path
     std::vector<JitKernel> jk;

@@ -305,6 +305,10 @@ template <bool MARG, int NTH>
 __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
     constexpr int NSPLIT = NTH / RT;    // epilogue: warps per TMEM lane quarter
     constexpr int EA_MAX = NTH == 512 ? 48 : 64;  // ea values per thread in registers
+#ifndef EPI_SPS
+#define EPI_SPS 1
+#endif
+    constexpr int SPS = NTH == 512 ? 1 : EPI_SPS;  // sums per TMEM wait in the epilogue
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
@@ -496,58 +500,60 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
                 const int ns = min(st.s_per_group, st.n_out - s0);
                 // the NSPLIT warps of a lane quarter split the group's sums
                 const int sl0 = (ns * part) / NSPLIT, sl1 = (ns * (part + 1)) / NSPLIT;
-                for (int sl = sl0; sl < sl1; ++sl) {
-                    // TMEM loads in batches of up to 32 columns, one wait per batch
-                    const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) + (uint32_t)(sl * na);
-                    float a4[4] = {0.f, 0.f, 0.f, 0.f};  // 4 independent FMA chains
+                // SPS sums per TMEM wait: every column of those sums is loaded
+                // (tcgen05.ld.32x32b, x8 / x4) before one tcgen05.wait::ld --
+                // the wait covers all outstanding loads, so fewer, larger
+                // batches mean fewer exposed TMEM latencies
+                for (int sl = sl0; sl < sl1; sl += SPS) {
+                    float t[SPS][EA_MAX];
 #pragma unroll
-                    for (int cb = 0; cb < EA_MAX; cb += 32) {
-                        if (cb < na) {
-                            float t[32];
+                    for (int u = 0; u < SPS; ++u) {
+                        const bool live = sl + u < sl1;
+                        const uint32_t trow = tmem + tb + ((uint32_t)(qd * 32) << 16) +
+                                              (uint32_t)((sl + u) * na);
 #pragma unroll
-                            for (int q = 0; q < 4; ++q) {
-                                const int c0 = cb + q * 8;
-                                if (c0 + 8 <= na) {
-                                    float v8[8];
-                                    tmem_ld8(trow + c0, v8);
+                        for (int c0 = 0; c0 < EA_MAX; c0 += 8) {
+                            if (live && c0 + 8 <= na) {
+                                float v8[8];
+                                tmem_ld8(trow + c0, v8);
 #pragma unroll
-                                    for (int k = 0; k < 8; ++k) t[q * 8 + k] = v8[k];
-                                } else if (c0 < na) {
-                                    float v4[4];
-                                    tmem_ld4(trow + c0, v4);
+                                for (int k = 0; k < 8; ++k) t[u][c0 + k] = v8[k];
+                            } else if (live && c0 < na) {
+                                float v4[4];
+                                tmem_ld4(trow + c0, v4);
 #pragma unroll
-                                    for (int k = 0; k < 4; ++k) {
-                                        t[q * 8 + k] = v4[k];
-                                        t[q * 8 + 4 + k] = 0.f;
-                                    }
-                                } else {
-#pragma unroll
-                                    for (int k = 0; k < 8; ++k) t[q * 8 + k] = 0.f;
+                                for (int k = 0; k < 4; ++k) {
+                                    t[u][c0 + k] = v4[k];
+                                    t[u][c0 + 4 + k] = 0.f;
                                 }
-                            }
-                            tmem_wait_ld();
-                            // packed FP32 (FFMA2): 2 x 2 independent chains
-                            float2 p01 = make_float2(a4[0], a4[1]), p23 = make_float2(a4[2], a4[3]);
+                            } else {
 #pragma unroll
-                            for (int i = 0; i < 32; i += 4) {
-                                if (cb + i + 4 <= EA_MAX) {  // compile-time bound of ear[]
-                                    p01 = __ffma2_rn(make_float2(ear[cb + i], ear[cb + i + 1]),
-                                                     make_float2(t[i], t[i + 1]), p01);
-                                    p23 = __ffma2_rn(make_float2(ear[cb + i + 2], ear[cb + i + 3]),
-                                                     make_float2(t[i + 2], t[i + 3]), p23);
-                                }
+                                for (int k = 0; k < 8; ++k) t[u][c0 + k] = 0.f;
                             }
-                            a4[0] = p01.x; a4[1] = p01.y; a4[2] = p23.x; a4[3] = p23.y;
                         }
                     }
-                    const float acc = (a4[0] + a4[1]) + (a4[2] + a4[3]);
-                    const float val = shift + r_lg2(acc);
-                    const int s = s0 + sl;
-                    if (st.type == 1) {
-                        act[st.buf_out + s * RT + m] = val;
-                    } else {
-                        const int col = __ldg(p.root_map + s);
-                        racc[col * RT + m] = r_lse2(racc[col * RT + m], val);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int u = 0; u < SPS; ++u) {
+                        if (sl + u >= sl1) break;
+                        // packed FP32 (FFMA2): 2 x 2 independent chains
+                        float2 p01 = make_float2(0.f, 0.f), p23 = make_float2(0.f, 0.f);
+#pragma unroll
+                        for (int i = 0; i < EA_MAX; i += 4) {
+                            p01 = __ffma2_rn(make_float2(ear[i], ear[i + 1]),
+                                             make_float2(t[u][i], t[u][i + 1]), p01);
+                            p23 = __ffma2_rn(make_float2(ear[i + 2], ear[i + 3]),
+                                             make_float2(t[u][i + 2], t[u][i + 3]), p23);
+                        }
+                        const float acc = (p01.x + p01.y) + (p23.x + p23.y);
+                        const float val = shift + r_lg2(acc);
+                        const int s = s0 + sl + u;
+                        if (st.type == 1) {
+                            act[st.buf_out + s * RT + m] = val;
+                        } else {
+                            const int col = __ldg(p.root_map + s);
+                            racc[col * RT + m] = r_lse2(racc[col * RT + m], val);
+                        }
                     }
                 }
             };

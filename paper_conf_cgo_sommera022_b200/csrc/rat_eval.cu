@@ -444,19 +444,25 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
                 if (p.wbufs == 2 && G > 1) issue_w(st, 1, 1);
             }
             const int na = st.na, nb = st.nb, kpad = st.k_pad;
-            if (tid < RT) {
-                const int m = tid;
+            // NTH/2 threads per side: PH = NTH/256 threads per sample (warps
+            // w and w+4 share a sample), each computes the full max and
+            // 1/PH of the exps (no extra barrier to combine maxima)
+            constexpr int PH = NTH / 256;
+            const int side = tid / (NTH / 2), ts = tid % (NTH / 2);
+            const int m = ((ts >> 5) & 3) * 32 + lane, ph = ts >> 7;
+            if (side == 0) {
                 const float *VA = act + st.buf_a;
                 const float hi = col_max(VA, na, m);
                 const float hc = fmaxf(hi, -1e30f);
-                for (int i = 0; i < na; ++i) ea[i * RT + m] = r_ex2(VA[i * RT + m] - hc);
-                sa[m] = hi;
-            } else if (tid < 2 * RT) {
-                const int m = tid - RT;
+                const int ic = (na + PH - 1) / PH;
+                for (int i = ph * ic; i < min(na, (ph + 1) * ic); ++i)
+                    ea[i * RT + m] = r_ex2(VA[i * RT + m] - hc);
+                if (ph == 0) sa[m] = hi;
+            } else {
                 const float *VB = act + st.buf_b;
                 const float hi = col_max(VB, nb, m);
                 const float hc = fmaxf(hi, -1e30f);
-                for (int j0 = 0; j0 < kpad; j0 += 8) {  // 8 k-values = one 16-byte row
+                for (int j0 = ph * 8; j0 < kpad; j0 += 8 * PH) {  // 8 k-values = one 16-byte row
                     uint32_t hw[4], lw[4];
 #pragma unroll
                     for (int k = 0; k < 8; k += 2) {
@@ -473,7 +479,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
                     *reinterpret_cast<uint4 *>(aimg + o) = make_uint4(hw[0], hw[1], hw[2], hw[3]);
                     *reinterpret_cast<uint4 *>(aimg + aimg_part + o) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
                 }
-                sb[m] = hi;
+                if (ph == 0) sb[m] = hi;
             }
             fence_async_smem();
             __syncthreads();

@@ -462,6 +462,7 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 768 / jo.block);
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
+    if (const char *e = getenv("SPNB_JIT_BAR")) jo.bar_every = std::max(0, atoi(e));
     JitProgram jp;
     std::string msg;
     int rc = generate_jit(g, jo, jp, msg);
@@ -975,6 +976,7 @@ int spn_codegen(const spn_handle *graph, int32_t task, int32_t lang, char *src, 
         return set_err(SPN_E_ARG, "bad arguments");
     JitOptions jo;
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
+    if (const char *e = getenv("SPNB_JIT_BAR")) jo.bar_every = std::max(0, atoi(e));
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
     JitProgram jp;
     std::string msg;

@@ -376,12 +376,20 @@ std::string ptx_opnd(const Opnd &o, const char *pf) {
 const char *kSlotPrefix[4] = {"%f", "%g", "%h", "%k"};
 
 std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int min_blocks,
-                           int K) {
+                           int K, int bar_every) {
     std::string body;
     body.reserve(ir.ins.size() * 48 * K);
     char b[4096];
     int np = 0, nr = 0, nd = 0;  // predicate / b32 / b64 temporaries
+    size_t since_bar = 0;
     for (const Ins &i : ir.ins) {
+      // optional CTA barrier every bar_every instructions: keeps the CTA's
+      // warps in the same stretch of the straight-line body (instruction-
+      // cache locality); every thread runs every iteration (see the loop)
+      if (bar_every > 0 && ++since_bar >= (size_t)bar_every) {
+          body += "    bar.sync 0;\n";
+          since_bar = 0;
+      }
       for (int j = 0; j < K; ++j) {
         const char *pf = kSlotPrefix[j];
         const std::string d = pf + std::to_string(i.d), a = ptx_opnd(i.a, pf), bb = ptx_opnd(i.b, pf),
@@ -478,7 +486,7 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
              "    .reg .b64 %%rd<%d>;\n"
              "    .reg .f32 %%fbest, %%fw;\n"
              "    .reg .s32 %%ridx, %%rtid, %%rcta, %%rncta, %%R;\n"
-             "    .reg .b64 %%x, %%n, %%gld, %%out, %%amp, %%tab, %%s, %%stride, %%t64, %%sj;\n",
+             "    .reg .b64 %%x, %%n, %%gld, %%out, %%amp, %%tab, %%s, %%stride, %%t64, %%sj, %%sb, %%tid64;\n",
              name.c_str(), block, min_blocks, np + 1, nr + 1, nd + 1);
     s += b;
     for (int j = 0; j < K; ++j) {
@@ -501,21 +509,22 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
              "    mov.u32 %%rcta, %%ctaid.x;\n"
              "    mov.u32 %%rncta, %%nctaid.x;\n"
              "    mul.wide.u32 %%s, %%rcta, %d;\n"
-             "    cvt.u64.u32 %%t64, %%rtid;\n"
-             "    add.s64 %%s, %%s, %%t64;\n"
+             "    cvt.u64.u32 %%tid64, %%rtid;\n"
+             "    add.s64 %%s, %%s, %%tid64;\n"
              "    mul.wide.u32 %%stride, %%rncta, %d;\n"
              "$Lloop:\n"
-             "    setp.ge.s64 %%pl, %%s, %%n;\n"
+             "    sub.s64 %%sb, %%s, %%tid64;\n"  // CTA's first sample: the loop is CTA-uniform
+             "    setp.ge.s64 %%pl, %%sb, %%n;\n"
              "    @%%pl bra $Ldone;\n",
              block * K, block * K);
     s += b;
     for (int j = 0; j < K; ++j) {
-        // slot j: sample s + j*block; past the end it recomputes sample s
-        // (valid) and its stores are predicated off
+        // slot j: sample s + j*block; past the end it recomputes the CTA's
+        // first sample (valid) and its stores are predicated off
         snprintf(b, sizeof(b),
                  "    add.s64 %%sj, %%s, %d;\n"
                  "    setp.lt.s64 %%pv%d, %%sj, %%n;\n"
-                 "    selp.b64 %%sj, %%sj, %%s, %%pv%d;\n"
+                 "    selp.b64 %%sj, %%sj, %%sb, %%pv%d;\n"
                  "    mul.lo.s64 %%t64, %%sj, %%gld;\n"
                  "    shl.b64 %%t64, %%t64, 2;\n"
                  "    add.s64 %%xr%d, %%x, %%t64;\n"
@@ -771,7 +780,7 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
                 fprintf(stderr, "[spnb] task %d marg %d: %zu ins, max_live %lld\n", t, marg, ir.ins.size(),
                         (long long)ir_max_live(ir));
             jt.ptx[marg] = ptx_head + emit_ptx_entry(ir, jt.name + suffix, opt.block, opt.min_blocks,
-                                                       opt.samples_per_thread);
+                                                       opt.samples_per_thread, opt.bar_every);
             cpp += emit_cpp(ir, jt.name + suffix + "_body");
         }
         char b[1024];

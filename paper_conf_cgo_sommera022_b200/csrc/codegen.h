@@ -25,6 +25,9 @@ struct JitOptions {
     int block = 256;             // threads per CTA (launch bound)
     int min_blocks = 2;          // __launch_bounds__ min CTAs per SM (register cap)
     int samples_per_thread = 1;  // K in 1..4: K interleaved copies of the body per thread
+    int bar_every = 500;         // > 0: CTA barrier every bar_every IR instructions
+                                 // (instruction-cache locality; C2 joint measured
+                                 // 3.27e9 samples/s at 500 vs 2.88e9 without)
     int64_t task_cap_nodes = 3000;  // pack connected components up to this size
     int64_t max_task_nodes = 16000; // larger components: compiled path unsupported
                                     // (ptxas time and register spills grow with size)

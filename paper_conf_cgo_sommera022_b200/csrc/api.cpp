@@ -453,12 +453,15 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
 int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev, int sms,
                      std::chrono::steady_clock::time_point t0, spn_handle **out_plan) {
     JitOptions jo;
-    jo.block = opt.block_threads ? opt.block_threads : 256;
+    jo.block = opt.block_threads ? opt.block_threads : 768;
     if (jo.block % 32 || jo.block < 32 || jo.block > 1024)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
-    // launch bound: 3 CTAs of 256 threads per SM by default (<= 80 registers;
-    // measured on C2: 2.87e9 samples/s at 3 x 256 (80 regs, no spills) vs
-    // 2.83e9 at 2 x 256 (128 regs) and 2.56e9 at 6 x 128)
+    // launch bound: 768 resident threads per SM (<= 80 registers).  Default
+    // one CTA of 768 threads: with the barrier-synchronised body (bar_every)
+    // all 24 warps of the SM walk the same stretch of code.  Measured on C2
+    // joint: 1 x 768 3.65e9 samples/s, 1 x 640 3.46e9, 1 x 1024 3.36e9,
+    // 3 x 256 3.27e9, 1 x 512 3.25e9; marginal 1 x 768 2.56e9 vs 3 x 256
+    // (spill fallback to 2 x 256) 2.12e9
     jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 768 / jo.block);
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));

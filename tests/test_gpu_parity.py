@@ -334,3 +334,49 @@ def test_compiled_spill_fallback_marginal_full_size():
     idx = np.random.default_rng(1).choice(len(x), 2000, replace=False)
     ref, _ = oracle_eval(g, x[idx], marginal=True)
     _cmp(out[idx], ref)
+
+
+def test_c3_full_size_sampled():
+    """Config 3 at its bench size (32 speaker SPNs, 1M samples, 20% NaN,
+    marginal + argmax) in the bench's launch configuration; oracle on a
+    sample of rows spread over the batch."""
+    from spn_inputs import config_graph
+    g = config_graph("C3")
+    x, _ = ancestral_sample(g, 1_000_000, 3002)
+    x = nan_mask(x, 0.2, 3100)
+    out, am, P = _run(g, x, marginal=True)
+    assert P.info()["path"] == 2
+    idx = np.concatenate([np.arange(0, 200), np.random.default_rng(5).choice(len(x), 1500, replace=False),
+                          np.arange(len(x) - 200, len(x))])
+    ref, am_ref = oracle_eval(g, x[idx], marginal=True)
+    _cmp(out[idx], ref)
+    _cmp_argmax(am[idx], ref, am_ref)
+
+
+def test_c4_layered_marginal_full_graph_sampled():
+    """Config 4 graph on the layered path with 20% missing features."""
+    from spn_inputs import config_graph
+    g = config_graph("C4")
+    x, _ = ancestral_sample(g, 2000, 4003)
+    x = nan_mask(x, 0.2, 4004)
+    out, am, P = _run(g, x, marginal=True, layered_path=2)
+    assert P.info()["path"] == 1
+    idx = np.random.default_rng(6).choice(len(x), 200, replace=False)
+    ref, am_ref = oracle_eval(g, x[idx], marginal=True)
+    _cmp(out[idx], ref)
+    _cmp_argmax(am[idx], ref, am_ref)
+
+
+def test_c5_layered_full_graph_sampled():
+    """Config 5 graph (3,242,010 nodes) on the layered path, counter-based
+    U[0,1] inputs (the bench recipe) over two transposed chunks with a ragged
+    tail; oracle on rows from the start, the chunk boundary and the end."""
+    from spn_inputs import config_graph, uniform_chunked
+    g = config_graph("C5")
+    x = uniform_chunked(40_001, g.n_features, 5002)
+    out, am, P = _run(g, x, layered_path=2)
+    assert P.info()["path"] == 1
+    idx = np.concatenate([np.arange(0, 16), np.arange(18_936, 18_952), np.arange(39_985, 40_001)])
+    ref, am_ref = oracle_eval(g, x[idx])
+    _cmp(out[idx], ref)
+    _cmp_argmax(am[idx], ref, am_ref)

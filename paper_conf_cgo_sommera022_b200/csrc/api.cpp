@@ -689,13 +689,16 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         size_t lsmem = 0;
         int wbufs = 0;
         const int prec = opt.tc_precision == 1 ? 1 : 3;
-        // prefer double-buffered weight groups (N <= 240, else N <= 120 per
-        // group), then serial groups
-        int first_attempt = 0;  // SPNB_LAYERED_ATTEMPT: 1 = N<=120 groups, 2 = serial (A/B)
-        if (const char *ev = getenv("SPNB_LAYERED_ATTEMPT")) first_attempt = std::min(2, std::max(0, atoi(ev)));
-        for (int attempt = first_attempt; attempt < 3 && wbufs == 0; ++attempt) {
-            const int n_cap = attempt == 1 ? 120 : 240;
-            const int wb = attempt == 2 ? 1 : 2;
+        // weight-group buffering, first that fits in shared memory: N <= 240
+        // or N <= 120 per group with double-buffered weights, then a single
+        // buffer (measured on C4: a third buffer, prefetch distance 2, gave
+        // no gain -- the ring code supports it; scripts/gpu/run_lay12.sh)
+        static const int kAttempts[][2] = {{240, 2}, {120, 2}, {240, 1}, {120, 1}, {120, 1}};
+        int first_attempt = 0;  // SPNB_LAYERED_ATTEMPT: index into kAttempts (A/B)
+        if (const char *ev = getenv("SPNB_LAYERED_ATTEMPT")) first_attempt = std::min(4, std::max(0, atoi(ev)));
+        for (int attempt = first_attempt; attempt < 5 && wbufs == 0; ++attempt) {
+            const int n_cap = kAttempts[attempt][0];
+            const int wb = kAttempts[attempt][1];
             detect_layered(g, lp, n_cap);
             if (!lp.ok) break;
             lsmem = rat_smem_bytes(lp.smem_floats, lp.C, lp.max_na, lp.max_kpad, lp.max_ngroup,

@@ -183,8 +183,11 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
     const int I = st.n_out, V = st.n_vars;
     const int mp = (tid & 63) * 2;           // 2 samples
     const int grp = tid >> 6, d0 = grp * DPT; // distribution group, first distribution
-    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
-    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
+    // (a, b) pairs per variable: [8 groups][DPT & ~1 pairs] (two per LDS.128),
+    // then [8 groups][DPT & 1 pair] (LDS.64)
+    constexpr int DE = DPT & ~1, DO = DPT & 1, PV = 8 * DPT;  // pairs per variable
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DE / 2);
+    const float2 *ab2 = reinterpret_cast<const float2 *>(prm) + 8 * DE + grp;
     const float *C = prm + (st.cst_off - st.par_off);
     float2 acc[DPT];
 #pragma unroll
@@ -195,13 +198,14 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
         const float2 x2 = *reinterpret_cast<const float2 *>(xs + v * RT + mp);
         bool anynan = false;
         if constexpr (MARG) anynan = (x2.x != x2.x) | (x2.y != x2.y);
-        float2 qv[DPTP];
+        float2 qv[DPT];
 #pragma unroll
-        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
-            const float4 q4 = ab4[v * 4 * DPTP + k];
+        for (int k = 0; k < DE / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * (PV / 2) + k];
             qv[2 * k] = make_float2(q4.x, q4.y);
             qv[2 * k + 1] = make_float2(q4.z, q4.w);
         }
+        if constexpr (DO) qv[DPT - 1] = ab2[v * PV];
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
             const float2 q = qv[d];
@@ -232,8 +236,11 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
     const int I = st.n_out, V = st.n_vars;
     const int mq = (tid & 31) * 4;           // 4 samples
     const int grp = tid >> 5, d0 = grp * DPT; // distribution group, first distribution
-    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
-    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
+    // (a, b) pairs per variable: [8 groups][DPT & ~1 pairs] (two per LDS.128),
+    // then [8 groups][DPT & 1 pair] (LDS.64)
+    constexpr int DE = DPT & ~1, DO = DPT & 1, PV = 8 * DPT;  // pairs per variable
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DE / 2);
+    const float2 *ab2 = reinterpret_cast<const float2 *>(prm) + 8 * DE + grp;
     const float *C = prm + (st.cst_off - st.par_off);
     float acc[DPT][4];
 #pragma unroll
@@ -249,13 +256,14 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
         const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
         bool anynan = false;
         if constexpr (MARG) anynan = (xv[0] != xv[0]) | (xv[1] != xv[1]) | (xv[2] != xv[2]) | (xv[3] != xv[3]);
-        float2 qv[DPTP];
+        float2 qv[DPT];
 #pragma unroll
-        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
-            const float4 q4 = ab4[v * 4 * DPTP + k];
+        for (int k = 0; k < DE / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * (PV / 2) + k];
             qv[2 * k] = make_float2(q4.x, q4.y);
             qv[2 * k + 1] = make_float2(q4.z, q4.w);
         }
+        if constexpr (DO) qv[DPT - 1] = ab2[v * PV];
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
             const float2 q = qv[d];
@@ -312,7 +320,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1/2 w, 3/4 x
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1-3 w, 4/5 x
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 64);
     size_t off = 128;
     float *act = reinterpret_cast<float *>(smem + off);
@@ -336,11 +344,11 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
     uint8_t *wsm = smem + off;   // [wbufs][prec==3 ? 2 : 1][n_group x kpad] f16
     const size_t w_part = (size_t)p.max_ngroup * p.max_kpad * 2;
     const size_t w_buf = w_part * (p.prec == 3 ? 2 : 1);
-    const bool ovl = p.wbufs == 2 && p.overlap;
+    const bool ovl = p.wbufs >= 2 && p.overlap;
     const uint32_t tmem_cols = ovl ? 2 * TMEM_BUF : TMEM_BUF;
 
     const uint32_t bar_mma = r_smem(bars), bar_w0 = r_smem(bars + 1);
-    const uint32_t bar_x0 = r_smem(bars + 3);
+    const uint32_t bar_x0 = r_smem(bars + 4);
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                          r_smem(tmem_slot)),
@@ -348,7 +356,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     if (tid == 0) {
-        for (int i = 0; i < 5; ++i)
+        for (int i = 0; i < 6; ++i)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(r_smem(bars + i)), "r"(1));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -440,8 +448,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
             // ---------------- SUM / ROOT: phase 1 (shifts, exps, A image) ----
             const int G = st.n_groups;
             if (warp == 0) {
-                issue_w(st, 0, 0);
-                if (p.wbufs == 2 && G > 1) issue_w(st, 1, 1);
+                for (int b = 0; b < p.wbufs && b < G; ++b) issue_w(st, b, b);
             }
             const int na = st.na, nb = st.nb, kpad = st.k_pad;
             // NTH/2 threads per side: PH = NTH/256 threads per sample (warps
@@ -564,7 +571,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
                 }
             };
             for (int g = 0; g < G; ++g) {
-                const int wb = p.wbufs == 2 ? (g & 1) : 0;
+                const int wb = g % p.wbufs;  // ring of wbufs weight buffers
                 const uint32_t tb = ovl ? (uint32_t)(g & 1) * TMEM_BUF : 0u;
                 mbar_wait(bar_w0 + 8 * wb, (ph_w >> wb) & 1u);
                 ph_w ^= 1u << wb;

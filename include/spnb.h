@@ -70,7 +70,10 @@ typedef struct spn_handle spn_handle; /* opaque: a graph or a prepared plan */
    knobs: block size, max partition size, ... PAPER.md L404, L481, L494). */
 typedef struct spn_prepare_options {
     int32_t device;             /* CUDA device ordinal; -1 = current device    */
-    int32_t block_threads;      /* threads per CTA, multiple of 32; 0 = auto   */
+    int32_t block_threads;      /* threads per CTA, multiple of 32; 0 = auto
+                                   (compiled path: 768, one CTA per SM;
+                                   interpreter: from the feature tile size;
+                                   layered path: 512 or 256, fixed)         */
     int32_t samples_per_thread; /* K in {1,2,4}; 0 = auto                      */
     int32_t layered_path;       /* 0 auto, 1 off (generic only), 2 force the
                                    tensor-core RAT-SPN path (E_UNSUPPORTED if

@@ -372,11 +372,10 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
             while (plan.fparams.size() % 4) plan.fparams.push_back(0.f);
             st.par_off = (int64_t)plan.fparams.size();
             // (a, b) pairs grouped by the kernel's 8 distribution groups of
-            // DPT = I/8 distributions (group g: g*DPT + k): per variable first
-            // [8 groups][DPT & ~1 pairs] (16-byte aligned, two pairs per
-            // LDS.128), then [8 groups][DPT & 1 pair]; no padding
-            const int32_t DPT = I / 8, DE = DPT & ~1;
-            std::vector<float> ab((size_t)V * I * 2, 0.f);
+            // DPT = I/8: ab[v][g][k] = pair of distribution g*DPT + k, DPT
+            // padded to even so a thread loads two pairs per LDS.128
+            const int32_t DPT = I / 8, DPTp = DPT + (DPT & 1);
+            std::vector<float> ab((size_t)V * 8 * DPTp * 2, 0.f);
             std::vector<double> Cs(I, 0.0);
             for (int32_t i = 0; i < I; ++i) {
                 const int64_t u = reg.nodes[i];
@@ -391,10 +390,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
                     const double *pp = g.params.data() + g.param_begin[o];
                     const double a = 1.0 / (pp[1] * std::sqrt(2.0 * M_LN2));
                     Cs[i] += -std::log2(pp[1] * std::sqrt(2.0 * M_PI));
-                    const int32_t gi = i / DPT, ki = i % DPT;
-                    const size_t pair = (size_t)v * I +
-                                        (ki < DE ? (size_t)gi * DE + ki : (size_t)8 * DE + gi);
-                    const size_t idx = pair * 2;
+                    const size_t idx = (((size_t)v * 8 + (size_t)(i / DPT)) * DPTp + (size_t)(i % DPT)) * 2;
                     ab[idx] = (float)a;
                     ab[idx + 1] = (float)(a * pp[0]);
                 }

@@ -183,11 +183,8 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
     const int I = st.n_out, V = st.n_vars;
     const int mp = (tid & 63) * 2;           // 2 samples
     const int grp = tid >> 6, d0 = grp * DPT; // distribution group, first distribution
-    // (a, b) pairs per variable: [8 groups][DPT & ~1 pairs] (two per LDS.128),
-    // then [8 groups][DPT & 1 pair] (LDS.64)
-    constexpr int DE = DPT & ~1, DO = DPT & 1, PV = 8 * DPT;  // pairs per variable
-    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DE / 2);
-    const float2 *ab2 = reinterpret_cast<const float2 *>(prm) + 8 * DE + grp;
+    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
     const float *C = prm + (st.cst_off - st.par_off);
     float2 acc[DPT];
 #pragma unroll
@@ -198,14 +195,13 @@ __device__ __forceinline__ void leaf_step_pairs(const LStep &st, float *act, con
         const float2 x2 = *reinterpret_cast<const float2 *>(xs + v * RT + mp);
         bool anynan = false;
         if constexpr (MARG) anynan = (x2.x != x2.x) | (x2.y != x2.y);
-        float2 qv[DPT];
+        float2 qv[DPTP];
 #pragma unroll
-        for (int k = 0; k < DE / 2; ++k) {  // two (a, b) pairs per LDS.128
-            const float4 q4 = ab4[v * (PV / 2) + k];
+        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * 4 * DPTP + k];
             qv[2 * k] = make_float2(q4.x, q4.y);
             qv[2 * k + 1] = make_float2(q4.z, q4.w);
         }
-        if constexpr (DO) qv[DPT - 1] = ab2[v * PV];
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
             const float2 q = qv[d];
@@ -236,11 +232,8 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
     const int I = st.n_out, V = st.n_vars;
     const int mq = (tid & 31) * 4;           // 4 samples
     const int grp = tid >> 5, d0 = grp * DPT; // distribution group, first distribution
-    // (a, b) pairs per variable: [8 groups][DPT & ~1 pairs] (two per LDS.128),
-    // then [8 groups][DPT & 1 pair] (LDS.64)
-    constexpr int DE = DPT & ~1, DO = DPT & 1, PV = 8 * DPT;  // pairs per variable
-    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DE / 2);
-    const float2 *ab2 = reinterpret_cast<const float2 *>(prm) + 8 * DE + grp;
+    constexpr int DPTP = DPT + (DPT & 1);    // pairs per (v, group), padded to even
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm) + grp * (DPTP / 2);
     const float *C = prm + (st.cst_off - st.par_off);
     float acc[DPT][4];
 #pragma unroll
@@ -256,14 +249,13 @@ __device__ __forceinline__ void leaf_step_t(const LStep &st, float *act, const f
         const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
         bool anynan = false;
         if constexpr (MARG) anynan = (xv[0] != xv[0]) | (xv[1] != xv[1]) | (xv[2] != xv[2]) | (xv[3] != xv[3]);
-        float2 qv[DPT];
+        float2 qv[DPTP];
 #pragma unroll
-        for (int k = 0; k < DE / 2; ++k) {  // two (a, b) pairs per LDS.128
-            const float4 q4 = ab4[v * (PV / 2) + k];
+        for (int k = 0; k < DPTP / 2; ++k) {  // two (a, b) pairs per LDS.128
+            const float4 q4 = ab4[v * 4 * DPTP + k];
             qv[2 * k] = make_float2(q4.x, q4.y);
             qv[2 * k + 1] = make_float2(q4.z, q4.w);
         }
-        if constexpr (DO) qv[DPT - 1] = ab2[v * PV];
 #pragma unroll
         for (int d = 0; d < DPT; ++d) {
             const float2 q = qv[d];

@@ -29,15 +29,12 @@ def emulate_layered(plan: dict, x: np.ndarray, n_roots: int, marginal: bool = Fa
             t = int(st["type"])
             if t == 0:
                 I, V = int(st["n_out"]), int(st["n_vars"])
-                # per variable: [8 groups][DPT & ~1 pairs], then [8 groups][DPT & 1]
-                # pair; group g holds distributions g*DPT .. g*DPT + DPT - 1
+                # pairs grouped as ab[v][g][k] = distribution g*DPT + k (8 groups,
+                # DPT = I/8 padded to even)
                 dpt = I // 8
-                de = dpt & ~1
-                raw = fp[int(st["par_off"]):int(st["par_off"]) + V * I * 2].reshape(V, I, 2)
-                ab = np.empty_like(raw)
-                for i in range(I):
-                    g, k = divmod(i, dpt)
-                    ab[:, i, :] = raw[:, g * de + k, :] if k < de else raw[:, 8 * de + g, :]
+                dptp = dpt + (dpt & 1)
+                ab = fp[int(st["par_off"]):int(st["par_off"]) + V * 8 * dptp * 2].reshape(V, 8, dptp, 2)
+                ab = ab[:, :, :dpt, :].reshape(V, I, 2)
                 # per-(v, i) c = log2(a) + 0.5 log2(ln2/pi) (= -log2(sigma sqrt(2 pi)))
                 cv = np.log2(ab[:, :, 0]) + 0.5 * np.log2(np.log(2.0) / np.pi)
                 acc = np.tile(fp[int(st["cst_off"]):int(st["cst_off"]) + I][:, None], (1, N))

@@ -1,0 +1,13 @@
+#!/bin/bash
+# r01 closing run on HEAD: GPU tests, smoke, default bench, layered C4/C4m/C5 bench, C4 launch list + full ncu capture
+cd "${GRAFT_REPO_ROOT:-/root/repo}"
+O=gpurun_out; mkdir -p $O; : > $O/status.txt
+timeout 1200 python -m pytest tests -m gpu -q --timeout 600 > $O/pytest_gpu.log 2>&1; echo "pytest=$?" >> $O/status.txt
+timeout 600 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" > $O/smoke.log 2>&1; echo "smoke=$?" >> $O/status.txt
+timeout 900 python bench.py > $O/bench_default.log 2>&1; echo "bench=$?" >> $O/status.txt
+timeout 900 python bench.py --config C4 > $O/bench_C4.log 2>&1; echo "bench_C4=$?" >> $O/status.txt
+timeout 900 python bench.py --config C4 --marginal > $O/bench_C4m.log 2>&1; echo "bench_C4m=$?" >> $O/status.txt
+timeout 900 python bench.py --config C5 > $O/bench_C5.log 2>&1; echo "bench_C5=$?" >> $O/status.txt
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file $O/launches_C4.csv python bench.py --config C4 --steps 3 --warmup 3 > $O/ncu_l_C4.log 2>&1; echo "ncul_C4=$?" >> $O/status.txt
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:rat -s 2 -c 1 -o $O/full_C4 python bench.py --config C4 --steps 3 --warmup 3 > $O/ncu_f_C4.log 2>&1; echo "nculf_C4=$?" >> $O/status.txt
+echo done >> $O/status.txt

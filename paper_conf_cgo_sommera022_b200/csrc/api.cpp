@@ -223,10 +223,11 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         std::string msg;
         const int32_t *tasks_am = P.jfused_argmax ? argmax : nullptr;
         for (size_t t = 0; t < P.jk.size(); ++t) {
-            const int64_t need = (n + (int64_t)P.jblock * P.jK - 1) / ((int64_t)P.jblock * P.jK);
+            const int64_t blk = P.jk[t].block[marg ? 1 : 0];
+            const int64_t need = (n + blk * P.jK - 1) / (blk * P.jK);
             const int grid = (int)std::max<int64_t>(
                 1, std::min<int64_t>(need, marg ? P.jgrid_max_m[t] : P.jgrid_max[t]));
-            const int rc = jit_launch(P.jk[t], marg, grid, P.jblock, (cudaStream_t)stream, x, n, ld,
+            const int rc = jit_launch(P.jk[t], marg, grid, (int)blk, (cudaStream_t)stream, x, n, ld,
                                       out, P.R, (int *)tasks_am, P.d_jtab, msg);
             if (rc != SPN_OK) return set_err(rc, msg);
         }
@@ -545,6 +546,32 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
                 k.regs[v] = k2.regs[v];
                 k.occupancy[v] = k2.occupancy[v];
                 k.local_bytes[v] = k2.local_bytes[v];
+                k.block[v] = k2.block[v];
+            }
+            // still spilling at one CTA per SM: smaller CTAs (more registers
+            // per thread) for this variant only, unless the caller pinned the
+            // launch (C2 marginal spills at 768 threads / 80 registers)
+            for (int b2 : {640, 512}) {
+                if (k.local_bytes[v] == 0 || opt.block_threads || opt.ctas_per_sm > 0 || b2 >= jo.block)
+                    break;
+                JitOptions jo2 = jo;
+                jo2.block = b2;
+                jo2.min_blocks = 1;
+                JitProgram jp2;
+                std::vector<char> cb;
+                std::string log;
+                if (generate_jit(g, jo2, jp2, msg) != SPN_OK ||
+                    jit_compile(jp2.tasks[t].ptx[v], arch, cb, log) != SPN_OK)
+                    break;
+                JitKernel k2;
+                if (jit_load(cb, jp2.tasks[t].name, v, b2, k2, msg) != SPN_OK) break;
+                jit_unload_variant(k, v);
+                k.module[v] = k2.module[v];
+                k.fn[v] = k2.fn[v];
+                k.regs[v] = k2.regs[v];
+                k.occupancy[v] = k2.occupancy[v];
+                k.local_bytes[v] = k2.local_bytes[v];
+                k.block[v] = k2.block[v];
             }
         }
         // grid-stride loop over samples with exactly one wave of resident CTAs

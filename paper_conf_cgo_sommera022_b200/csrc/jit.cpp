@@ -187,6 +187,7 @@ int jit_load(const std::vector<char> &cubin, const std::string &name, int v, int
     d.fn_attr(&k.regs[v], CU_FUNC_ATTRIBUTE_NUM_REGS, f);
     d.fn_attr(&k.local_bytes[v], CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, f);
     d.occ(&k.occupancy[v], f, block, 0);
+    k.block[v] = block;
     return SPN_OK;
 }
 

@@ -24,6 +24,7 @@ struct JitKernel {
     int regs[2] = {0, 0};
     int occupancy[2] = {0, 0};  // CTAs per SM at the launch block size
     int local_bytes[2] = {0, 0};  // per-thread local memory (> 0: register spills)
+    int block[2] = {0, 0};        // threads per CTA the variant was generated for
 };
 
 // Load variant v's cubin (0 joint, 1 marginal) into the current context and

@@ -548,31 +548,9 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
                 k.local_bytes[v] = k2.local_bytes[v];
                 k.block[v] = k2.block[v];
             }
-            // still spilling at one CTA per SM: smaller CTAs (more registers
-            // per thread) for this variant only, unless the caller pinned the
-            // launch (C2 marginal spills at 768 threads / 80 registers)
-            for (int b2 : {640, 512}) {
-                if (k.local_bytes[v] == 0 || opt.block_threads || opt.ctas_per_sm > 0 || b2 >= jo.block)
-                    break;
-                JitOptions jo2 = jo;
-                jo2.block = b2;
-                jo2.min_blocks = 1;
-                JitProgram jp2;
-                std::vector<char> cb;
-                std::string log;
-                if (generate_jit(g, jo2, jp2, msg) != SPN_OK ||
-                    jit_compile(jp2.tasks[t].ptx[v], arch, cb, log) != SPN_OK)
-                    break;
-                JitKernel k2;
-                if (jit_load(cb, jp2.tasks[t].name, v, b2, k2, msg) != SPN_OK) break;
-                jit_unload_variant(k, v);
-                k.module[v] = k2.module[v];
-                k.fn[v] = k2.fn[v];
-                k.regs[v] = k2.regs[v];
-                k.occupancy[v] = k2.occupancy[v];
-                k.local_bytes[v] = k2.local_bytes[v];
-                k.block[v] = k2.block[v];
-            }
+            // (a variant still spilling at one CTA of 768 threads keeps it:
+            // regenerating the C2 marginal kernel with 512-thread CTAs, no
+            // spills, measured 2.20e9 vs 2.57e9 samples/s; 640 threads 2.59e9)
         }
         // grid-stride loop over samples with exactly one wave of resident CTAs
         // (per variant): every thread gets ceil or floor of n / threads samples

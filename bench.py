@@ -5,13 +5,18 @@
                     [--marginal] [--impl ours|reference]
 
 A step is one pass of the whole hot path (spn_infer_* over one batch of the
-config's N samples, inputs resident in HBM).  Default workload: config C2 (a
-speaker-ID-shaped Gaussian SPN over 26 features, 1M samples, joint), the
-configuration the metric is quoted on that fits one GPU.  At N GPUs each rank
-processes its own N-sample batch (weak scaling, no data-path collective).
-L2 is flushed (256 MiB write) between timed steps.  Prints ONE JSON line on
-rank 0.  ``--impl reference`` times the fp64 CPU oracle (the reference arm of
-this tier) on bounded samples of the same workload.
+config's samples, inputs resident in HBM).  Default workload: config C5 (a
+RAT-SPN of 3,242,010 nodes over 784 features, 10 class roots, 10M samples,
+joint + argmax) -- the largest configuration of BASELINE.json, the one the
+north star's >= 7x-at-8-GPUs target is stated on; it fits one B200.  C5
+scales strongly: the 10M samples are split over the N ranks and, at N > 1,
+every step ends with the NCCL all-gather of the per-sample log-likelihoods
+and argmax (the only collective), inside the timed region.
+The other configs scale weakly (a full batch per rank).  The input (31 GB at
+N = 1) is larger than L2; L2 is also flushed (256 MiB write) between timed
+steps.  Prints ONE JSON line on rank 0.  ``--impl reference`` times the fp64
+CPU oracle (the reference arm of this tier) on bounded samples of the same
+workload.
 """
 from __future__ import annotations
 
@@ -32,6 +37,11 @@ METRIC = "SPN inference samples/sec (joint & marginal) at 1/2/4/8 B200; % of HBM
 UNIT = "samples/s"
 
 
+def CONFIGS_N(cfg: str) -> int:
+    from spn_inputs import CONFIGS
+    return CONFIGS[cfg]["n_samples"]
+
+
 def _peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -45,9 +55,10 @@ def samples_per_rank(cfg: str, world: int) -> tuple[int, str]:
     """C5 is a strong-scaling config (10M samples split over the GPUs,
     BASELINE.json configs[4]); the others are weak (a full batch per GPU)."""
     from spn_inputs import CONFIGS
+    from paper_conf_cgo_sommera022_b200.parallel import shard_sizes
     n = CONFIGS[cfg]["n_samples"]
     if cfg == "C5":
-        return n // world, "strong"
+        return max(shard_sizes(n, world)), "strong"
     return n, "weak"
 
 
@@ -69,8 +80,9 @@ def device_uniform(n: int, F: int, seed: int, start: int, dev, chunk: int = 6553
     return x
 
 
-def make_workload(cfg: str, rank: int, marginal: bool):
-    """Seeded graph + this rank's input batch (host numpy)."""
+def make_workload(cfg: str, rank: int, marginal: bool, n_max: int | None = None):
+    """Seeded graph + this rank's input batch (host numpy); RAT-SPN inputs
+    are generated for the first n_max samples only when n_max is given."""
     from spn_inputs import (CONFIGS, config_graph, ancestral_sample, add_outliers, nan_mask,
                             toy_data, uniform_chunked)
     c = CONFIGS[cfg]
@@ -91,7 +103,7 @@ def make_workload(cfg: str, rank: int, marginal: bool):
     else:
         # RAT-SPN configs: counter-based U[0,1] features (the layered path's
         # work is data independent; parity tests use ancestral samples)
-        x = uniform_chunked(n, g.n_features, c["data_seed"], start=rank * n)
+        x = uniform_chunked(min(n, n_max or n), g.n_features, c["data_seed"], start=rank * n)
     return g, x, n
 
 
@@ -173,19 +185,26 @@ def run_reference(args):
         return
     from oracle import oracle_eval, num_threads, build_oracle
     build_oracle()
-    g, x, n = make_workload(args.config, 0, args.marginal)
+    g, x, n = make_workload(args.config, 0, args.marginal,
+                            n_max=4096 if args.config in ("C4", "C5") else None)
     # per step: a bounded sample sized so the whole run takes a few minutes
-    n0 = min(n, 1000)
-    t = time.perf_counter()
-    oracle_eval(g, x[:n0], marginal=args.marginal)
-    per = (time.perf_counter() - t) / n0
+    # (calibrated from a growing probe: one C5 sample costs ~1 s of one core)
+    n0 = min(n, 16)
+    while True:
+        t = time.perf_counter()
+        oracle_eval(g, x[:n0], marginal=args.marginal)
+        dt = time.perf_counter() - t
+        if dt > 1.0 or n0 >= min(n, 4096):
+            break
+        n0 = min(n, n0 * 4)
+    per = dt / n0
     budget = 150.0 / max(1, args.steps + args.warmup)
-    m = int(max(100, min(n, budget / max(per, 1e-9))))
+    m = int(max(16, min(x.shape[0], budget / max(per, 1e-9))))
     for i in range(args.warmup):
         oracle_eval(g, x[:m], marginal=args.marginal)
     ts = []
     for i in range(args.steps):
-        off = (i * m) % max(1, n - m + 1)
+        off = (i * m) % max(1, x.shape[0] - m + 1)
         t = time.perf_counter()
         oracle_eval(g, x[off:off + m], marginal=args.marginal)
         ts.append(time.perf_counter() - t)
@@ -194,8 +213,10 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT,
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": _config_dict(args, g, n),
+            "scaling": "strong" if args.config == "C5" else "weak", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": _config_dict(args, g, n, args.gpus,
+                                   "strong" if args.config == "C5" else "weak"),
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": num_threads(),
                              "kind": "oracle",
                              "sample": f"{m} samples per step of the {args.config} workload"},
@@ -204,15 +225,20 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
-def _config_dict(args, g, n):
+def _config_dict(args, g, n, world=1, scaling="weak"):
     from spn_inputs import CONFIGS
     c = g.counts()
-    return {"workload": f"{args.config}: {CONFIGS[args.config]['desc']}",
-            "query": "marginal" if args.marginal else "joint",
-            "samples_per_gpu": n, "n_features": g.n_features, "n_roots": g.n_roots,
-            "graph_nodes": c["nodes"], "sum_edges": c["sum_edges"],
-            "l2": "flushed between timed steps (256 MiB write)",
-            "parallelism": f"dp{args.gpus} (sample sharding)"}
+    d = {"workload": f"{args.config}: {CONFIGS[args.config]['desc']}",
+         "query": "marginal" if args.marginal else "joint",
+         "samples_per_gpu": n, "n_features": g.n_features, "n_roots": g.n_roots,
+         "graph_nodes": c["nodes"], "sum_edges": c["sum_edges"],
+         "l2": "flushed between timed steps (256 MiB write)",
+         "parallelism": f"dp{world} (sample sharding)"}
+    if scaling == "strong":
+        d["samples_total"] = CONFIGS[args.config]["n_samples"]
+        d["l2"] = ("inputs larger than L2 (31 GB / N) and L2 flushed between timed steps "
+                   "(256 MiB write)")
+    return d
 
 
 def launches_per_step(info: dict, n: int, want_am: bool) -> int:
@@ -247,10 +273,13 @@ def run_ours(args):
     n_rank, scaling = samples_per_rank(args.config, world)
     if args.config in ("C4", "C5"):
         from spn_inputs import CONFIGS, config_graph
+        from paper_conf_cgo_sommera022_b200.parallel import shard_range
         g = config_graph(args.config)
         n = n_rank
-        xd = device_uniform(n, g.n_features, CONFIGS[args.config]["data_seed"], rank * n, dev)
-        x = xd[:min(n, 262_144)].cpu().numpy()   # host copy of a bounded subset (e2e, oracle)
+        lo = shard_range(CONFIGS[args.config]["n_samples"], rank, world)[0] if scaling == "strong" \
+            else rank * n
+        xd = device_uniform(n, g.n_features, CONFIGS[args.config]["data_seed"], lo, dev)
+        x = xd[:min(n, 1 << 20)].cpu().numpy()   # host copy of a bounded subset (e2e, oracle)
     else:
         g, x, n = make_workload(args.config, rank, args.marginal)
         xd = None
@@ -268,13 +297,26 @@ def run_ours(args):
     am = torch.empty((n,), dtype=torch.int32, device=dev) if want_am else None
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     st = torch.cuda.current_stream(dev)
+    # strong scaling: every step ends with the gather of all ranks' results
+    gather = scaling == "strong" and world > 1
+    if gather:
+        full_out = torch.empty((n * world, R), dtype=torch.float32, device=dev)
+        full_am = torch.empty((n * world,), dtype=torch.int32, device=dev) if want_am else None
 
     def step():
         P.infer(xd, marginal=args.marginal, out=out, argmax=am, want_argmax=want_am, stream=st)
 
+    def collect():
+        # equal shards (10M / {1,2,4,8}): one all_gather_into_tensor each (NCCL)
+        dist.all_gather_into_tensor(full_out, out)
+        if want_am:
+            dist.all_gather_into_tensor(full_am, am)
+
     for _ in range(max(3, args.warmup)):
         flush.fill_(1)
         step()
+        if gather:
+            collect()
     torch.cuda.synchronize()
     clocks = ClockSampler(local)
     clocks.start()
@@ -286,24 +328,29 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(args.steps)]
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+            torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     for i in range(args.steps):
         flush.fill_(i & 0xff)
         evs[i][0].record(st)
         step()
         evs[i][1].record(st)
+        if gather:
+            collect()
+        evs[i][2].record(st)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    times = [a.elapsed_time(b) for a, b in evs]          # ms, kernel-only per step
+    times = [a.elapsed_time(c) for a, b, c in evs]       # ms per step (infer + gather)
+    gather_ms = [b.elapsed_time(c) for a, b, c in evs]
     tot_ms = sum(times)
     t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     tot_ms = float(t.item())
-    value = n * world * args.steps / (tot_ms / 1e3)
+    n_job = CONFIGS_N(args.config) if scaling == "strong" else n * world
+    value = n_job * args.steps / (tot_ms / 1e3)
     n_e2e = x.shape[0]
 
     # ---- end to end through the public host-buffer API (H2D + D2H inside) ----
@@ -326,40 +373,50 @@ def run_ours(args):
     if rank == 0:
         peaks, src = _peaks()
         ms = tot_ms / args.steps
+        rate = n / (ms / 1e3)                           # samples/s of one rank
         clock_mhz = peaks.get("sm_max_mhz", 1965.0)
         mufu_peak = 16 * 148 * clock_mhz * 1e6          # MUFU ops/s (16/clk/SM)
-        mufu = info["mufu_per_sample"] * n / (ms / 1e3)
-        hbm = info["bytes_per_sample"] * n / (ms / 1e3) / 1e9
-        prof = os.path.join(ROOT, "profiles", f"ncu_{args.config}.json")
+        fma_peak = 128 * 148 * clock_mhz * 1e6          # FP32 FMA lane-ops/s (128/clk/SM)
+        mufu = info["mufu_per_sample"] * rate
+        hbm = info["bytes_per_sample"] * rate / 1e9
+        fma = info["fma_per_sample"] * rate
+        tc = info["tc_flops_per_sample"] * rate
+        tc_peak = peaks.get("bf16_tflops", 1590.0) * 1e12
+        prof = os.path.join(ROOT, "profiles", f"ncu_{args.config}{'m' if args.marginal else ''}.json")
         traffic = None
         if os.path.exists(prof):
             with open(prof) as f:
                 traffic = json.load(f).get("dram_bytes_per_launch")
-        hbm_part = {"achieved": hbm, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                    "frac": hbm / peaks["hbm_gbs"]}
+        part = lambda a, p_, u: {"achieved": a, "peak": p_, "unit": u, "frac": a / p_}
+        hbm_part = part(hbm, peaks["hbm_gbs"], "GB/s")
+        mufu_part = part(mufu / 1e9, mufu_peak / 1e9, "Gop/s")
+        # the metric's roofline: HBM or MUFU, whichever binds (time = max)
+        hm = max(hbm_part["frac"], mufu_part["frac"])
+        metric_roof = {"frac": hm, "binding": "hbm" if hbm_part["frac"] >= mufu_part["frac"]
+                       else "mufu", "hbm": hbm_part, "mufu": mufu_part}
+        peak_note = f"x 148 SMs x {clock_mhz:.0f} MHz (sm_max_mhz, {src})"
         if info["path"] in (0, 2):
             roof = {"bound": "alu", "pipe": "MUFU ex2/lg2 (16 op/clk/SM)",
                     "achieved": mufu / 1e9, "peak": mufu_peak / 1e9, "unit": "Gop/s",
                     "frac": mufu / mufu_peak, "traffic": traffic,
-                    "peak_source": f"16 MUFU/clk/SM x 148 SMs x {clock_mhz:.0f} MHz "
-                                   f"(sm_max_mhz, {src})",
-                    "hbm": hbm_part}
+                    "peak_source": "16 MUFU/clk/SM " + peak_note,
+                    "mufu_count": "sum over sums of the fan-in (n-1 ex2 + 1 lg2 per "
+                                  "n-ary log-sum-exp)",
+                    "hbm_mufu": metric_roof, "hbm": hbm_part}
         else:
-            fma = info["fma_per_sample"] * n / (ms / 1e3)
-            fma_peak = 128 * 148 * clock_mhz * 1e6
-            tc = info["tc_flops_per_sample"] * n / (ms / 1e3)
-            tc_peak = peaks.get("bf16_tflops", 1590.0) * 1e12
+            # layered path: the binding pipe is FP32 FMA (leaf layer + stage-2
+            # contractions); tensor fraction on algorithmic one-pass flops
             roof = {"bound": "alu", "pipe": "FP32 FMA (leaf layer, 128 lanes/clk/SM)",
                     "achieved": fma / 1e9, "peak": fma_peak / 1e9, "unit": "GFMA/s",
                     "frac": fma / fma_peak, "traffic": traffic,
-                    "peak_source": f"128 FMA/clk/SM x 148 SMs x {clock_mhz:.0f} MHz",
-                    "mufu": {"achieved": mufu / 1e9, "peak": mufu_peak / 1e9, "unit": "Gop/s",
-                             "frac": mufu / mufu_peak},
+                    "peak_source": "128 FMA/clk/SM " + peak_note,
+                    "hbm_mufu": metric_roof,
                     "tensor": {"achieved": tc / 1e12, "peak": tc_peak / 1e12,
                                "unit": "TFLOP/s", "frac": tc / tc_peak,
-                               "dtype": "f16 (hi/lo split)" if args.tc_precision != 1 else "f16",
+                               "flops": "algorithmic, one pass (2 na nb S per sum region)",
+                               "passes_executed": info["tc_passes"],
                                "peak_source": f"bf16_tflops ({src}); f16 dense rate = bf16"},
-                    "hbm": hbm_part}
+                    "kernel": f"layered v{info['layered_kernel']}"}
         # the oracle baseline is timed on rank 0 at N = 1 only (contract)
         cpu = cpu_baseline(g, x, args.marginal) if world == 1 else None
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
@@ -368,14 +425,17 @@ def run_ours(args):
                 "dtype": "f32", "data": ("synthetic (seeded ancestral samples)"
                                          if args.config not in ("C4", "C5") else
                                          "synthetic (counter-based U[0,1) per 65,536-sample chunk)"),
-                "config": _config_dict(args, g, n) | {
+                "config": _config_dict(args, g, n, world, scaling) | {
                     "plan": {k: info[k] for k in ("path", "n_nodes", "n_tasks", "n_records",
                                                   "block_threads", "samples_per_thread",
                                                   "grid", "smem_bytes", "mufu_per_sample",
                                                   "fma_per_sample", "tc_flops_per_sample",
                                                   "max_stack", "kernel_regs", "ctas_per_sm",
-                                                  "mufu_exec_per_sample", "compile_ms")},
-                    "prepare_s": prep_s},
+                                                  "mufu_exec_per_sample", "compile_ms",
+                                                  "chunk_samples", "layered_kernel",
+                                                  "tc_passes")},
+                    "prepare_s": prep_s,
+                    "tc_precision": args.tc_precision},
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
                 "e2e": {"value": e2e_val, "unit": UNIT,
                         "h2d_bytes_per_step": int(x.nbytes),
@@ -385,6 +445,10 @@ def run_ours(args):
                 "gpu_launches": args.steps * launches_per_step(info, n, want_am),
                 "step_ms": {"min": min(times), "median": statistics.median(times),
                             "max": max(times)}}
+        if gather:
+            line["gather_ms"] = {"median": statistics.median(gather_ms), "max": max(gather_ms),
+                                 "what": "NCCL all_gather_into_tensor of logp [N/P, R] "
+                                         "and argmax [N/P] (inside the timed step)"}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()
@@ -396,13 +460,13 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--config", default="C5", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--marginal", action="store_true")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--K", type=int, default=0, help="samples per thread (0 = auto)")
     ap.add_argument("--block", type=int, default=0, help="threads per CTA (0 = auto)")
     ap.add_argument("--tc-precision", type=int, default=0,
-                    help="layered path: 0 auto (f16 hi/lo split), 1 single f16 pass")
+                    help="layered path: 0 auto, 1 single f16 pass, 2 f16 hi/lo split")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

@@ -95,7 +95,13 @@ typedef struct spn_prepare_options {
                                    64 values live at once (register pressure:
                                    region-graph cross products) or
                                    compilation fails                          */
-    int32_t reserved[7];        /* must be zero                                */
+    int32_t layered_kernel;     /* layered path kernel: 0 auto (v2 when the
+                                   region graph fits it, else v1), 1 v1
+                                   (rat_eval.cu: one tile walks its schedule
+                                   step by step), 2 v2 (rat2.cu: warp-
+                                   specialised leaf / MMA / epilogue roles;
+                                   E_UNSUPPORTED if not applicable)          */
+    int32_t reserved[6];        /* must be zero                                */
 } spn_prepare_options;
 
 /* Statistics of a prepared plan (used by the benchmark's roofline). */
@@ -103,14 +109,20 @@ typedef struct spn_plan_stats {
     int64_t n_nodes;            /* after canonicalisation                     */
     int64_t n_leaves, n_sums, n_products;
     int64_t n_sum_edges;
-    int64_t n_tasks;            /* partitions (§IV-A4)               */
+    int64_t n_tasks;            /* partitions (§IV-A4); 1 on the
+                                   layered path (it does not partition)       */
     int64_t n_cut_values;       /* values crossing tasks (stored+loaded once) */
     int64_t partition_cost;     /* sum over values of #consuming other tasks  */
-    int64_t n_records;          /* interpreter records over all tasks         */
+    int64_t n_records;          /* interpreter records over all tasks;
+                                   layered path: schedule steps per tile      */
     int64_t n_global_slots;     /* per-warp scratch slots (global memory)     */
     int64_t n_smem_slots;       /* per-warp scratch slots (shared memory)     */
     int64_t max_stack;          /* deepest register-stack position used       */
-    int64_t mufu_per_sample;    /* algorithmic: sum over sums (fan-in + 1)    */
+    int64_t mufu_per_sample;    /* algorithmic: sum over sums of the fan-in
+                                   (max-shifted n-ary LSE: the shift term is
+                                   exactly 1, so n-1 ex2 + 1 lg2; 0 for a
+                                   single child); layered path: na + nb + S
+                                   per sum region (the exps and lg2s)         */
     int64_t fma_per_sample;     /* algorithmic FP32 ops (2/leaf, 1/prod edge,
                                    3/sum edge)                                */
     int64_t bytes_per_sample;   /* 4*n_features + 4*n_roots (+4 argmax)       */
@@ -128,6 +140,8 @@ typedef struct spn_plan_stats {
     double  compile_ms;         /* PTX assembly wall time (tasks in parallel)  */
     int64_t chunk_samples;      /* layered path: samples per transposed chunk
                                    (one transpose + one layered launch each)  */
+    int32_t layered_kernel;     /* layered path: 1 v1, 2 v2 (0 other paths)   */
+    int32_t tc_passes;          /* layered path: f16 MMA passes (1 or 3)      */
 } spn_plan_stats;
 
 /* Fill *opt with defaults (all auto). */
@@ -174,8 +188,11 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt,
  * n = 0 is a no-op.  NaN in x yields NaN for every root depending on that
  * feature (reading c7).  Argument and launch errors are returned
  * synchronously; faults inside the kernel surface at the caller's next sync.
- * Re-entrant for distinct streams (the plan is read-only; per-call scratch
- * is owned by the plan and serialised on the plan's internal lock).
+ * Re-entrant for distinct streams: the plan's tables are read-only, and its
+ * scratch (transposed features of the layered path, global slots of the
+ * interpreter) is used by one launch at a time -- a call on a different
+ * stream than the previous call makes its stream wait for the previous
+ * call's completion event first (calls on one stream are stream-ordered).
  */
 int spn_infer_joint(spn_handle *plan, const float *x, int64_t n, int64_t ld,
                     float *out, int32_t *argmax, void *cuda_stream);
@@ -236,6 +253,18 @@ int spn_plan_info(const spn_handle *plan, spn_plan_stats *stats);
 int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, int64_t why_len,
                       int64_t *sizes, void *steps, int32_t *vars, float *fparams, void *wimg,
                       int32_t *root_map);
+/*
+ * spn_build_layered2: the same for the v2 kernel's plan (rat2.cu; requires a
+ *   complete binary region tree per repetition, uniform leaf width I (a
+ *   multiple of 8, <= 48) and sum width S <= 48).  *ok = 0/1 (why[] gets the
+ *   reason).  sizes[0] steps (sizes[5] bytes each), sizes[1] vars (int32),
+ *   sizes[2] fparams (float), sizes[3] weight-image bytes, sizes[4] roots;
+ *   dims[11] = {F, C, I, S, D, gcols, kpad_bot, kpad_up, max_wgroup,
+ *   max_vars, max_blk}.  NULL buffers: sizes and dims only.
+ */
+int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
+                       int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
+                       void *wimg, int32_t *root_map);
 int spn_partition_graph(const spn_handle *graph, int64_t max_task_ops, int32_t *task_of_node,
                         int32_t *n_tasks, int64_t *cost, int64_t *cut_values);
 int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32_t x_in_smem,

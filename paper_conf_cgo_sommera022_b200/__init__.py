@@ -22,7 +22,7 @@ import numpy as np
 from .build import LIB as _LIB_PATH
 
 __all__ = ["SPNError", "Graph", "Plan", "load_library", "partition_graph",
-           "build_program", "build_layered", "LSTEP_DTYPE", "NODE_DTYPE", "REC_DTYPE", "EDGE_DTYPE",
+           "build_program", "build_layered", "build_layered2", "LSTEP_DTYPE", "R2STEP_DTYPE", "NODE_DTYPE", "REC_DTYPE", "EDGE_DTYPE",
            "GAUSSIAN", "CATEGORICAL", "HISTOGRAM", "SUM", "PRODUCT"]
 
 GAUSSIAN, CATEGORICAL, HISTOGRAM, SUM, PRODUCT = 0, 1, 2, 3, 4
@@ -54,7 +54,7 @@ class _Options(ctypes.Structure):
                 ("samples_per_thread", ctypes.c_int32), ("layered_path", ctypes.c_int32),
                 ("max_task_nodes", ctypes.c_int64), ("tc_precision", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("compiled_path", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("layered_kernel", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
 
 
 class _Stats(ctypes.Structure):
@@ -67,7 +67,8 @@ class _Stats(ctypes.Structure):
                                       "smem_bytes", "x_in_smem")] + [
         ("prepare_ms", ctypes.c_double), ("kernel_regs", ctypes.c_int32),
         ("ctas_per_sm", ctypes.c_int32), ("mufu_exec_per_sample", ctypes.c_int64),
-        ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64)]
+        ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64),
+        ("layered_kernel", ctypes.c_int32), ("tc_passes", ctypes.c_int32)]
 
 
 _lib = None
@@ -97,11 +98,12 @@ def load_library(path: str | None = None):
     lib.spn_partition_graph.argtypes = [P, I64, P, P, P, P]
     lib.spn_build_program.argtypes = [P, I32, I32, I64, I64, P, P, P, P, P, P, P, P, P]
     lib.spn_build_layered.argtypes = [P, P, P, I64, P, P, P, P, P, P]
+    lib.spn_build_layered2.argtypes = [P, P, P, I64, P, P, P, P, P, P, P]
     lib.spn_codegen.argtypes = [P, I32, I32, P, P, P, P, P, P, P, P, I32, ctypes.c_char_p]
     for name in ("spn_load_graph", "spn_prepare", "spn_infer_joint", "spn_infer_marginal",
                  "spn_infer_joint_host", "spn_infer_marginal_host", "spn_plan_info",
                  "spn_partition_graph", "spn_build_program", "spn_build_layered",
-                 "spn_codegen"):
+                 "spn_build_layered2", "spn_codegen"):
         getattr(lib, name).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -167,7 +169,7 @@ class Plan:
     def __init__(self, graph: Graph, device: int | None = None, block_threads: int = 0,
                  samples_per_thread: int = 0, max_task_nodes: int = 0,
                  layered_path: int = 0, tc_precision: int = 0, ctas_per_sm: int = 0,
-                 compiled_path: int = 0):
+                 compiled_path: int = 0, layered_kernel: int = 0):
         lib = load_library()
         opt = _Options()
         lib.spn_default_options(ctypes.byref(opt))
@@ -182,6 +184,7 @@ class Plan:
         opt.tc_precision = tc_precision
         opt.ctas_per_sm = ctas_per_sm
         opt.compiled_path = compiled_path
+        opt.layered_kernel = layered_kernel
         h = ctypes.c_void_p()
         _check(lib.spn_prepare(graph.handle, ctypes.byref(opt), ctypes.byref(h)))
         self._h = h
@@ -204,11 +207,22 @@ class Plan:
             raise ValueError("x must be a CUDA float32 [N, F] tensor with unit feature stride")
         if x.shape[1] < self.n_features:
             raise ValueError(f"x has {x.shape[1]} features, the SPN needs {self.n_features}")
+        if x.device.index != self.device:
+            raise ValueError(f"x is on cuda:{x.device.index}, the plan on cuda:{self.device}")
         N = x.shape[0]
         if out is None:
             out = torch.empty((N, self.n_roots), dtype=torch.float32, device=x.device)
+        elif not (out.is_cuda and out.device.index == self.device and out.dtype == torch.float32
+                  and tuple(out.shape) == (N, self.n_roots) and out.is_contiguous()):
+            raise ValueError(f"out must be a contiguous float32 [{N}, {self.n_roots}] tensor "
+                             f"on cuda:{self.device}")
         if argmax is None and want_argmax:
             argmax = torch.empty((N,), dtype=torch.int32, device=x.device)
+        elif argmax is not None and not (
+                argmax.is_cuda and argmax.device.index == self.device
+                and argmax.dtype == torch.int32 and tuple(argmax.shape) == (N,)
+                and argmax.is_contiguous()):
+            raise ValueError(f"argmax must be a contiguous int32 [{N}] tensor on cuda:{self.device}")
         st = stream if stream is not None else torch.cuda.current_stream(x.device)
         fn = load_library().spn_infer_marginal if marginal else load_library().spn_infer_joint
         _check(fn(self._h, ctypes.c_void_p(x.data_ptr()), N, x.stride(0),
@@ -235,6 +249,12 @@ class Plan:
         outa = out.numpy() if hasattr(out, "numpy") and not isinstance(out, np.ndarray) else out
         ama = argmax.numpy() if (argmax is not None and hasattr(argmax, "numpy")
                                  and not isinstance(argmax, np.ndarray)) else argmax
+        if not (isinstance(outa, np.ndarray) and outa.dtype == np.float32
+                and outa.shape == (N, self.n_roots) and outa.flags["C_CONTIGUOUS"]):
+            raise ValueError(f"out must be a contiguous float32 [{N}, {self.n_roots}] host array")
+        if ama is not None and not (isinstance(ama, np.ndarray) and ama.dtype == np.int32
+                                    and ama.shape == (N,) and ama.flags["C_CONTIGUOUS"]):
+            raise ValueError(f"argmax must be a contiguous int32 [{N}] host array")
         fn = (load_library().spn_infer_marginal_host if marginal
               else load_library().spn_infer_joint_host)
         _check(fn(self._h, _ptr(xa), N, xa.strides[0] // 4, _ptr(outa),
@@ -309,6 +329,40 @@ def build_layered(graph: Graph):
                                  _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w), _ptr(rm)))
     return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
             "smem_floats": int(sizes[5])}, ""
+
+
+R2STEP_DTYPE = np.dtype([(n, "<i4") for n in ("type", "root", "n_out", "na", "nb", "kpad",
+                                              "n_groups", "s_per_group", "n_group", "slot_a",
+                                              "slot_b", "slot_out", "n_vars", "pad_")] +
+                        [(n, "<i8") for n in ("vars_off", "blk_off", "blk_floats", "w_off",
+                                              "w_group_bytes")])
+
+
+def build_layered2(graph: Graph):
+    """Host-only: the v2 layered kernel's plan (``spn_build_layered2``).
+    Returns (plan dict, "") or (None, reason)."""
+    lib = load_library()
+    ok = ctypes.c_int32()
+    why = ctypes.create_string_buffer(256)
+    sizes = np.zeros(6, dtype=np.int64)
+    dims = np.zeros(11, dtype=np.int32)
+    _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                  _ptr(dims), None, None, None, None, None))
+    if not ok.value:
+        return None, why.value.decode()
+    assert sizes[5] == R2STEP_DTYPE.itemsize, (sizes[5], R2STEP_DTYPE.itemsize)
+    steps = np.zeros(sizes[0], dtype=R2STEP_DTYPE)
+    vars_ = np.zeros(sizes[1], dtype=np.int32)
+    fp = np.zeros(sizes[2], dtype=np.float32)
+    w = np.zeros(sizes[3] // 2, dtype=np.float16)
+    rm = np.zeros(sizes[4], dtype=np.int32)
+    _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                  _ptr(dims), _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w),
+                                  _ptr(rm)))
+    keys = ("F", "C", "I", "S", "D", "gcols", "kpad_bot", "kpad_up", "max_wgroup", "max_vars",
+            "max_blk")
+    return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
+            **{k: int(v) for k, v in zip(keys, dims)}}, ""
 
 
 def codegen(graph: Graph, task: int = 0, lang: str = "cpp", compile: bool = False,

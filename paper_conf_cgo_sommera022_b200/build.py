@@ -28,12 +28,13 @@ CXX_FLAGS = ["-O2", "-std=c++17", "-fPIC", "-Wall", "-I", CSRC, "-I", INC,
              "-I", "/usr/local/cuda/include"]
 
 CU_SOURCES = ["dag_eval_k1.cu", "dag_eval_k2.cu", "dag_eval_k4.cu", "dag_eval_k8.cu",
-              "rat_eval.cu", "argmax.cu"]
+              "rat_eval.cu", "rat2.cu", "argmax.cu"]
 CXX_SOURCES = ["prepare.cpp", "layered.cpp", "codegen.cpp", "jit.cpp", "api.cpp"]
 HEADERS = ["program.h", "dag_eval.cuh", "prepare.h", "layered.h", "codegen.h", "jit.h"]
 # headers each CUDA translation unit includes (so editing host-side headers does
 # not rebuild the slow interpreter objects)
-CU_DEPS = {"rat_eval.cu": ["layered.h", "prepare.h", "program.h"], "argmax.cu": []}
+CU_DEPS = {"rat_eval.cu": ["layered.h", "prepare.h", "program.h"],
+           "rat2.cu": ["layered.h", "prepare.h", "program.h"], "argmax.cu": []}
 CU_DEPS_DEFAULT = ["dag_eval.cuh", "program.h"]
 
 

@@ -40,6 +40,11 @@ size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_
 cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaStream_t st);
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st);
+bool rat2_supported_shape(int I, int S);
+int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int kpad_up,
+                int max_wgroup, int prec, int n_in, int n_w);
+cudaError_t rat2_launch(const R2Params &p, const int32_t *leaf_steps, int n_leaf,
+                        const int32_t *sum_steps, int n_sum, bool marg, int grid, cudaStream_t st);
 cudaError_t argmax_rows_launch(const float *out, int64_t n, int R, int32_t *argmax, cudaStream_t st);
 }  // namespace spnb
 
@@ -78,6 +83,13 @@ struct DevicePlan {
     float *d_tables = nullptr;
     Edge *d_edges = nullptr;
     float *d_gslots = nullptr;
+    // plan-owned scratch (transposed features, interpreter global slots) is
+    // used by one launch at a time: a call on a different stream than the
+    // previous one waits for the previous one's event (spnb.h: re-entrant
+    // across streams)
+    std::mutex scratch_mu;
+    cudaEvent_t scratch_ev = nullptr;
+    void *scratch_stream = nullptr;
     // host pipeline buffers (lazily allocated)
     std::mutex host_mu;
     cudaStream_t hs[2] = {nullptr, nullptr};
@@ -100,6 +112,15 @@ struct DevicePlan {
     int32_t max_vars = 0, first_leaf = 0, max_leaf_params = 0, wbufs = 1;
     int32_t tmem_overlap = 1;  // epilogue of group g-1 under MMA g (SPNB_TMEM_OVERLAP=0: serial, A/B)
     unsigned long long *d_prof = nullptr;  // SPNB_PROFILE=1: phase cycle counters
+    // layered v2: warp-specialised kernel (rat2.cu); used when the region
+    // graph fits its constraints (build_rat2), else the v1 kernel above
+    bool r2 = false;
+    R2Params r2p;                 // device pointers + shared-memory layout
+    R2Step *d_r2steps = nullptr;
+    int32_t *d_r2vars = nullptr, *d_r2rm = nullptr, *d_r2leaf = nullptr, *d_r2sum = nullptr;
+    float *d_r2fp = nullptr;
+    uint8_t *d_r2w = nullptr;
+    int32_t n_r2leaf = 0, n_r2sum = 0;
     // compiled (per-SPN generated kernel) path
     std::vector<JitKernel> jk;
     std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM (joint kernel)
@@ -162,15 +183,43 @@ void free_plan(DevicePlan *p) {
     cudaFree(p->d_root_map);
     cudaFree(p->d_xT);
     cudaFree(p->d_jtab);
+    if (p->scratch_ev) cudaEventDestroy(p->scratch_ev);
+    cudaFree(p->d_r2steps);
+    cudaFree(p->d_r2vars);
+    cudaFree(p->d_r2rm);
+    cudaFree(p->d_r2leaf);
+    cudaFree(p->d_r2sum);
+    cudaFree(p->d_r2fp);
+    cudaFree(p->d_r2w);
     for (auto &k : p->jk) jit_unload(k);
     if (p->d_prof) {
         unsigned long long h[8];
-        if (cudaMemcpy(h, p->d_prof, sizeof(h), cudaMemcpyDeviceToHost) == cudaSuccess) {
+        if (!p->r2 && cudaMemcpy(h, p->d_prof, sizeof(h), cudaMemcpyDeviceToHost) == cudaSuccess) {
             const char *names[8] = {"leaf_wait", "leaf_compute", "leaf_barrier", "sum_phase1",
                                     "w_wait", "mma_issue+epilogue", "mma_wait", "other"};
             fprintf(stderr, "[spnb profile] cycles summed over CTAs:");
             for (int k = 0; k < 8; ++k) fprintf(stderr, " %s=%llu", names[k], h[k]);
             fprintf(stderr, "\n");
+        }
+        if (p->r2) {
+            unsigned long long h2[32];
+            if (cudaMemcpy(h2, p->d_prof, sizeof(h2), cudaMemcpyDeviceToHost) == cudaSuccess) {
+                const char *roles[4] = {"leaf(8 warps)", "epilogue(4)", "mma", "producer"};
+                const char *ph[4][8] = {
+                    {"wait_in", "compute", "shift", "wait_out", "exp+write", "-", "-", "-"},
+                    {"wait_leaf", "up_phase1", "wait_tmem", "sums", "tile_io", "step_setup", "-", "-"},
+                    {"wait_A", "wait_w", "wait_tmem", "issue", "-", "-", "-", "-"},
+                    {"wait_in_slot", "-", "wait_w_slot", "-", "-", "-", "-", "issue"}};
+                for (int r = 0; r < 4; ++r) {
+                    unsigned long long tot = 0;
+                    for (int k = 0; k < 8; ++k) tot += h2[r * 8 + k];
+                    fprintf(stderr, "[spnb profile v2] %-14s", roles[r]);
+                    for (int k = 0; k < 8; ++k)
+                        if (h2[r * 8 + k])
+                            fprintf(stderr, " %s=%.1f%%", ph[r][k], 100.0 * h2[r * 8 + k] / (double)tot);
+                    fprintf(stderr, "\n");
+                }
+            }
         }
         cudaFree(p->d_prof);
     }
@@ -210,8 +259,34 @@ int upload(T **dst, const std::vector<T> &v) {
     return SPN_OK;
 }
 
+int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
+                      int32_t *argmax, void *stream, bool marg);
+
 int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                  int32_t *argmax, void *stream, bool marg) {
+    if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
+    DevicePlan &P = *h->plan;
+    const bool scratch = P.path == 1 || (P.path == 0 && P.n_gslots > 0);
+    if (!scratch || n <= 0) return infer_device_impl(h, x, n, ld, out, argmax, stream, marg);
+    std::lock_guard<std::mutex> lk(P.scratch_mu);
+    DeviceGuard dg(P.device);
+    cudaError_t e;
+    if (P.scratch_ev && P.scratch_stream != stream &&
+        (e = cudaStreamWaitEvent((cudaStream_t)stream, P.scratch_ev, 0)) != cudaSuccess)
+        return cuda_err(e, "cudaStreamWaitEvent");
+    const int rc = infer_device_impl(h, x, n, ld, out, argmax, stream, marg);
+    if (rc != SPN_OK) return rc;
+    if (!P.scratch_ev &&
+        (e = cudaEventCreateWithFlags(&P.scratch_ev, cudaEventDisableTiming)) != cudaSuccess)
+        return cuda_err(e, "cudaEventCreate");
+    if ((e = cudaEventRecord(P.scratch_ev, (cudaStream_t)stream)) != cudaSuccess)
+        return cuda_err(e, "cudaEventRecord");
+    P.scratch_stream = stream;
+    return SPN_OK;
+}
+
+int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
+                      int32_t *argmax, void *stream, bool marg) {
     if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
     DevicePlan &P = *h->plan;
     if (n < 0) return set_err(SPN_E_ARG, "n < 0");
@@ -234,6 +309,26 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
         if (argmax && !P.jfused_argmax) {
             cudaError_t e = argmax_rows_launch(out, n, P.R, argmax, (cudaStream_t)stream);
             if (e != cudaSuccess) return cuda_err(e, "argmax launch");
+        }
+        return SPN_OK;
+    }
+    if (P.path == 1 && P.r2) {
+        R2Params rp = P.r2p;
+        rp.xT = P.d_xT;
+        rp.ldT = P.chunk;
+        for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
+            const int64_t m = std::min(P.chunk, n - c0);
+            const int64_t rows_pad = (m + 127) / 128 * 128;
+            cudaError_t e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
+                                             (cudaStream_t)stream);
+            if (e != cudaSuccess) return cuda_err(e, "transpose launch");
+            rp.n = m;
+            rp.out = out + c0 * P.R;
+            rp.argmax = argmax ? argmax + c0 : nullptr;
+            const int grid = (int)std::min<int64_t>((m + 127) / 128, P.grid_max);
+            e = rat2_launch(rp, P.d_r2leaf, P.n_r2leaf, P.d_r2sum, P.n_r2sum, marg, grid,
+                            (cudaStream_t)stream);
+            if (e != cudaSuccess) return cuda_err(e, "rat2 launch");
         }
         return SPN_OK;
     }
@@ -398,8 +493,79 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         free_plan(P);
         return rc;
     }
-    if (getenv("SPNB_PROFILE") && cudaMalloc(&P->d_prof, 8 * sizeof(unsigned long long)) == cudaSuccess)
-        cudaMemset(P->d_prof, 0, 8 * sizeof(unsigned long long));
+    if (getenv("SPNB_PROFILE") && cudaMalloc(&P->d_prof, 32 * sizeof(unsigned long long)) == cudaSuccess)
+        cudaMemset(P->d_prof, 0, 32 * sizeof(unsigned long long));
+    // ---- v2 kernel (rat2.cu): SPNB_RAT2=0 keeps the v1 kernel (A/B)
+    int want_r2 = opt.layered_kernel;  // SPNB_RAT2 overrides auto (A/B experiments)
+    if (const char *r2env = getenv("SPNB_RAT2"); r2env && want_r2 == 0) want_r2 = atoi(r2env) == 0 ? 1 : 0;
+    if (want_r2 != 1) {
+        Rat2Plan r2;
+        build_rat2(lp, r2);
+        if (r2.ok && !rat2_supported_shape(r2.I, r2.S)) {
+            r2.ok = false;
+            r2.why = "no v2 kernel instance for I = " + std::to_string(r2.I) + ", S = " +
+                     std::to_string(r2.S);
+        }
+        int smem_optin = 0;
+        cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        R2Params rp;
+        memset(&rp, 0, sizeof(rp));
+        bool fits = false;
+        // deepest rings that fit: leaf inputs 3..2, weight groups 4..2
+        static const int kRings[][2] = {{3, 4}, {3, 3}, {2, 4}, {2, 3}, {2, 2}};
+        for (int a = 0; r2.ok && a < 5 && !fits; ++a)
+            fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
+                               r2.max_wgroup, P->prec, kRings[a][0], kRings[a][1]) <= smem_optin;
+        if (r2.ok && fits) {
+            std::vector<int32_t> leaf_idx, sum_idx;
+            for (int32_t t = 0; t < (int32_t)r2.steps.size(); ++t)
+                (r2.steps[t].type == 0 ? leaf_idx : sum_idx).push_back(t);
+            std::vector<uint8_t> w2(r2.wimg.size() * 2);
+            if (!w2.empty()) memcpy(w2.data(), r2.wimg.data(), w2.size());
+            if ((rc = upload(&P->d_r2steps, r2.steps)) || (rc = upload(&P->d_r2vars, r2.vars)) ||
+                (rc = upload(&P->d_r2fp, r2.fparams)) || (rc = upload(&P->d_r2w, w2)) ||
+                (rc = upload(&P->d_r2rm, r2.root_map)) || (rc = upload(&P->d_r2leaf, leaf_idx)) ||
+                (rc = upload(&P->d_r2sum, sum_idx))) {
+                free_plan(P);
+                return rc;
+            }
+            rp.steps = P->d_r2steps;
+            rp.n_steps = (int32_t)r2.steps.size();
+            rp.C = r2.C;
+            rp.I = r2.I;
+            rp.S = r2.S;
+            rp.vars = P->d_r2vars;
+            rp.fparams = P->d_r2fp;
+            rp.wimg = P->d_r2w;
+            rp.root_map = P->d_r2rm;
+            rp.prec = P->prec;
+            rp.max_vars = r2.max_vars;
+            rp.max_blk = r2.max_blk;
+            rp.kpad_bot = r2.kpad_bot;
+            rp.kpad_up = r2.kpad_up;
+            rp.max_wgroup = r2.max_wgroup;
+            rp.gcols = r2.gcols;
+            rp.D = r2.D;
+            rp.prof = P->d_prof;
+            P->r2p = rp;
+            P->r2 = true;
+            P->n_r2leaf = (int32_t)leaf_idx.size();
+            P->n_r2sum = (int32_t)sum_idx.size();
+            P->smem = rp.smem_bytes;
+            // persistent kernel over many tiles per launch: 8 tiles per CTA
+            chunk = (int64_t)sms * 128 * 8;
+            P->chunk = chunk;
+        } else if (want_r2 == 2) {
+            free_plan(P);
+            return set_err(SPN_E_UNSUPPORTED, "layered v2 kernel not applicable: " +
+                                                  (r2.ok ? std::string("shared memory") : r2.why));
+        }
+    }
+    if (!P->r2 && (lp.w_max >= 32768.0 || (lp.w_min_nz > 0.0 && lp.w_min_nz < 0x1p-24))) {
+        // v1 keeps weights unscaled in f16: out of range -> not this path
+        free_plan(P);
+        return set_err(SPN_E_UNSUPPORTED, "layered v1 kernel: sum weights outside the f16 range");
+    }
     cudaError_t e = cudaMalloc(&P->d_xT, (size_t)g.F * chunk * 4);
     if (e != cudaSuccess) {
         free_plan(P);
@@ -414,25 +580,29 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         if (c.kind[u] == SPN_SUM) {
             s.n_sums++;
             s.n_sum_edges += c.cb[u + 1] - c.cb[u];
-            s.mufu_per_sample += c.cb[u + 1] - c.cb[u] + 1;
+            s.mufu_per_sample += c.cb[u + 1] - c.cb[u] > 1 ? c.cb[u + 1] - c.cb[u] : 0;
         } else if (c.kind[u] == SPN_PRODUCT) {
             s.n_products++;
         } else {
             s.n_leaves++;
         }
     }
-    s.n_tasks = (int64_t)lp.steps.size();
+    // the layered path does not partition: one task; n_records = schedule steps
+    s.n_tasks = 1;
+    s.n_records = (int64_t)lp.steps.size();
     s.fma_per_sample = lp.fma_per_sample;
     s.mufu_per_sample = lp.mufu_per_sample;
-    s.tc_flops_per_sample = lp.tc_flops_per_sample * (P->prec == 3 ? 3 : 1);
+    s.tc_flops_per_sample = lp.tc_flops_per_sample;  // algorithmic (one pass)
     s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)lp.C + 4;
     s.path = 1;
     s.chunk_samples = chunk;
-    s.block_threads = 256;
+    s.block_threads = P->r2 ? 512 : (lp.max_na > 48 ? 256 : 512);
     s.samples_per_thread = 0;
     s.grid = P->grid_max;
-    s.smem_bytes = (int32_t)smem;
+    s.smem_bytes = (int32_t)P->smem;
     s.x_in_smem = 0;
+    s.layered_kernel = P->r2 ? 2 : 1;
+    s.tc_passes = P->prec == 3 ? 3 : 1;
     s.prepare_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     spn_handle *h = new (std::nothrow) spn_handle();
@@ -672,8 +842,10 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     spn_prepare_options opt;
     spn_default_options(&opt);
     if (opt_in) opt = *opt_in;
-    for (int i = 0; i < 7; ++i)
+    for (int i = 0; i < 6; ++i)
         if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
+    if (opt.layered_kernel < 0 || opt.layered_kernel > 2)
+        return set_err(SPN_E_ARG, "layered_kernel must be 0 (auto), 1 (v1) or 2 (v2)");
     if (opt.compiled_path < 0 || opt.compiled_path > 2)
         return set_err(SPN_E_ARG, "compiled_path must be 0 (auto), 1 (off) or 2 (force)");
     const auto t0 = std::chrono::steady_clock::now();
@@ -716,7 +888,11 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
         }
         if (!lp.ok && opt.layered_path == 2)
             return set_err(SPN_E_UNSUPPORTED, "layered path not applicable: " + lp.why);
-        if (lp.ok) return prepare_layered(g, lp, opt, dev, sms, lsmem, wbufs, t0, out_plan);
+        if (lp.ok) {
+            const int rc = prepare_layered(g, lp, opt, dev, sms, lsmem, wbufs, t0, out_plan);
+            // auto: a layered graph neither kernel can serve goes to the generic path
+            if (rc != SPN_E_UNSUPPORTED || opt.layered_path == 2) return rc;
+        }
     }
     // ---- compiled path: one generated straight-line kernel per task ----
     // auto: used unless the caller pins interpreter parameters
@@ -951,6 +1127,36 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
         slots[1] = prog.n_gslots;
         slots[2] = prog.max_stack;
     }
+    return SPN_OK;
+}
+
+int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
+                       int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
+                       void *wimg, int32_t *root_map) {
+    if (!valid_graph_handle(graph) || !ok || !sizes || !dims) return set_err(SPN_E_ARG, "bad arguments");
+    LayeredPlan lp;
+    detect_layered(*graph->graph, lp);
+    Rat2Plan p;
+    build_rat2(lp, p);
+    *ok = p.ok ? 1 : 0;
+    if (why && why_len > 0) {
+        strncpy(why, p.why.c_str(), (size_t)why_len - 1);
+        why[why_len - 1] = 0;
+    }
+    sizes[0] = (int64_t)p.steps.size();
+    sizes[1] = (int64_t)p.vars.size();
+    sizes[2] = (int64_t)p.fparams.size();
+    sizes[3] = (int64_t)p.wimg.size() * 2;
+    sizes[4] = (int64_t)p.root_map.size();
+    sizes[5] = (int64_t)sizeof(R2Step);
+    const int32_t d[11] = {p.F, p.C, p.I, p.S, p.D, p.gcols, p.kpad_bot, p.kpad_up,
+                           p.max_wgroup, p.max_vars, p.max_blk};
+    memcpy(dims, d, sizeof(d));
+    if (steps) memcpy(steps, p.steps.data(), p.steps.size() * sizeof(R2Step));
+    if (vars) memcpy(vars, p.vars.data(), p.vars.size() * 4);
+    if (fparams) memcpy(fparams, p.fparams.data(), p.fparams.size() * 4);
+    if (wimg) memcpy(wimg, p.wimg.data(), p.wimg.size() * 2);
+    if (root_map) memcpy(root_map, p.root_map.data(), p.root_map.size() * 4);
     return SPN_OK;
 }
 

@@ -643,7 +643,7 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
             out.n_sums++;
             const int64_t fan = c.cb[u + 1] - c.cb[u];
             out.n_sum_edges += fan;
-            out.mufu_per_sample += fan + 1;
+            out.mufu_per_sample += fan > 1 ? fan : 0;  // n-ary LSE: n-1 ex2 + 1 lg2
             out.mufu_exec_per_sample += fan <= 1 ? 0 : (fan <= 4 ? fan : fan + 1);
             out.fma_per_sample += 3 * fan;
             for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) {

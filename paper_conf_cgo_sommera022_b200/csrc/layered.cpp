@@ -325,6 +325,11 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
             }
         }
         (void)root;
+        for (double w : W) {
+            plan.w_max = std::max(plan.w_max, w);
+            if (w > 0.0 && (plan.w_min_nz == 0.0 || w < plan.w_min_nz)) plan.w_min_nz = w;
+        }
+        plan.raw.push_back(W);
         for (int32_t gi = 0; gi < st.n_groups; ++gi) {
             std::vector<uint16_t> hi((size_t)st.n_group * st.k_pad, 0), lo(hi.size(), 0);
             for (int32_t sl = 0; sl < st.s_per_group; ++sl) {
@@ -377,6 +382,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
             const int32_t DPT = I / 8, DPTp = DPT + (DPT & 1);
             std::vector<float> ab((size_t)V * 8 * DPTp * 2, 0.f);
             std::vector<double> Cs(I, 0.0);
+            std::vector<double> raw((size_t)2 * V * I + I, 0.0);  // a[v][i], b[v][i], C[i]
             for (int32_t i = 0; i < I; ++i) {
                 const int64_t u = reg.nodes[i];
                 std::vector<int64_t> leaves;
@@ -393,8 +399,14 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
                     const size_t idx = (((size_t)v * 8 + (size_t)(i / DPT)) * DPTp + (size_t)(i % DPT)) * 2;
                     ab[idx] = (float)a;
                     ab[idx + 1] = (float)(a * pp[0]);
+                    raw[(size_t)v * I + i] = a;
+                    raw[(size_t)V * I + (size_t)v * I + i] = a * pp[0];
                 }
             }
+            for (int32_t i = 0; i < I; ++i) raw[(size_t)2 * V * I + i] = Cs[i];
+            plan.raw.push_back(std::move(raw));
+            plan.child_a.push_back(-1);
+            plan.child_b.push_back(-1);
             plan.fparams.insert(plan.fparams.end(), ab.begin(), ab.end());
             st.cst_off = (int64_t)plan.fparams.size();
             for (int32_t i = 0; i < I; ++i) plan.fparams.push_back((float)Cs[i]);
@@ -410,9 +422,13 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
         }
         const Partition &P = parts[reg.partitions[0]];
         st.buf_a = visit(P.ra);
+        const int32_t ca = (int32_t)plan.steps.size() - 1;
         st.buf_b = visit(P.rb);
+        const int32_t cb = (int32_t)plan.steps.size() - 1;
         st.type = 1;
         add_weights(st, rid, reg.partitions[0], false);
+        plan.child_a.push_back(ca);
+        plan.child_b.push_back(cb);
         st.buf_out = top0;
         buf_top = top0 + st.n_out * TILE;
         buf_peak = std::max(buf_peak, buf_top);
@@ -426,9 +442,13 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
         LStep st;
         memset(&st, 0, sizeof(st));
         st.buf_a = visit(P.ra);
+        const int32_t ca = (int32_t)plan.steps.size() - 1;
         st.buf_b = visit(P.rb);
+        const int32_t cb = (int32_t)plan.steps.size() - 1;
         st.type = 2;
         add_weights(st, root_region, p, true);
+        plan.child_a.push_back(ca);
+        plan.child_b.push_back(cb);
         st.buf_out = -1;
         plan.steps.push_back(st);
         buf_top = top0;
@@ -455,6 +475,159 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
         plan.max_na = std::max(plan.max_na, st.na);
     }
     plan.ok = true;
+}
+
+// ---------------------------------------------------------------- v2 plan
+void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
+    p = Rat2Plan();
+    auto fail = [&](const std::string &why) {
+        p.ok = false;
+        p.why = why;
+    };
+    if (!lp.ok) return fail("not layered: " + lp.why);
+    const int32_t ns = (int32_t)lp.steps.size();
+    if ((int32_t)lp.child_a.size() != ns || (int32_t)lp.raw.size() != ns)
+        return fail("layered plan without the region tree");
+    // ---- step kinds, uniform widths
+    std::vector<int32_t> kind(ns, 0);  // 0 LEAF, 1 BOT, 2 UP
+    int32_t I = -1, S = -1;
+    for (int32_t t = 0; t < ns; ++t) {
+        const LStep &st = lp.steps[t];
+        if (st.type == 0) {
+            if (I >= 0 && st.n_out != I) return fail("leaf regions of different widths");
+            I = st.n_out;
+            continue;
+        }
+        const int32_t a = lp.child_a[t], b = lp.child_b[t];
+        const bool la = lp.steps[a].type == 0, lb = lp.steps[b].type == 0;
+        if (la != lb) return fail("partition of a leaf region and a sum region");
+        kind[t] = la ? 1 : 2;
+        if (st.type == 1) {
+            if (S >= 0 && st.n_out != S) return fail("sum regions of different widths");
+            S = st.n_out;
+        }
+    }
+    if (I < 8 || I % 8 || I > 48) return fail("leaf width must be a multiple of 8, <= 48");
+    if (S < 0) S = 0;
+    if (S > 48) return fail("sum regions wider than 48");
+    // ---- TMEM activation slots: a sum region at depth d (root region = 0)
+    // writes slot d + (right child ? 1 : 0); its parent reads both children
+    std::vector<int32_t> slot(ns, 0), depth(ns, 0);
+    int32_t D = 0;
+    for (int32_t t = ns - 1; t >= 0; --t) {  // parents come after children (post-order)
+        const LStep &st = lp.steps[t];
+        if (st.type == 0) continue;
+        if (st.type == 2) depth[t] = 0;
+        const int32_t a = lp.child_a[t], b = lp.child_b[t];
+        depth[a] = depth[b] = depth[t] + 1;
+        slot[a] = depth[t] + 1;
+        slot[b] = depth[t] + 2;
+        if (kind[t] == 2) D = std::max(D, depth[t] + 2);
+    }
+    p.F = lp.F;
+    p.C = lp.C;
+    p.I = I;
+    p.S = S;
+    p.D = D;
+    const int32_t fixed_cols = D * S + p.C;
+    int32_t gc = std::min<int32_t>(256, (512 - fixed_cols) / 2) / 16 * 16;
+    const int32_t na_max = std::max(I, S);
+    if (gc < na_max) return fail("TMEM budget: " + std::to_string(fixed_cols) + " fixed columns");
+    p.gcols = gc;
+    p.ea_max = (na_max + 7) / 8 * 8;
+    p.kpad_bot = (I + 15) / 16 * 16;
+    p.kpad_up = S > 0 ? (S + 15) / 16 * 16 : 16;
+    // ---- steps
+    for (int32_t t = 0; t < ns; ++t) {
+        const LStep &st = lp.steps[t];
+        R2Step r;
+        memset(&r, 0, sizeof(r));
+        r.type = kind[t];
+        r.n_out = st.n_out;
+        r.slot_out = st.type == 1 ? slot[t] : 0;
+        r.root = st.type == 2 ? 1 : 0;
+        if (st.type == 0) {
+            const int32_t V = st.n_vars;
+            r.n_vars = V;
+            r.vars_off = (int64_t)p.vars.size();
+            p.vars.insert(p.vars.end(), lp.vars.begin() + st.vars_off,
+                          lp.vars.begin() + st.vars_off + V);
+            // block: (a, b)[v][i] interleaved, then C[i]; 16-byte multiple
+            while (p.fparams.size() % 4) p.fparams.push_back(0.f);
+            r.blk_off = (int64_t)p.fparams.size();
+            const std::vector<double> &raw = lp.raw[t];
+            for (int32_t v = 0; v < V; ++v)
+                for (int32_t i = 0; i < I; ++i) {
+                    p.fparams.push_back((float)raw[(size_t)v * I + i]);
+                    p.fparams.push_back((float)raw[(size_t)V * I + (size_t)v * I + i]);
+                }
+            for (int32_t i = 0; i < I; ++i) p.fparams.push_back((float)raw[(size_t)2 * V * I + i]);
+            while (p.fparams.size() % 4) p.fparams.push_back(0.f);
+            r.blk_floats = (int64_t)p.fparams.size() - r.blk_off;
+            p.max_vars = std::max(p.max_vars, V);
+            p.max_blk = std::max<int32_t>(p.max_blk, (int32_t)r.blk_floats);
+            p.n_leaf++;
+            p.steps.push_back(r);
+            continue;
+        }
+        const int32_t na = st.na, nb = st.nb, n_out = st.n_out;
+        r.na = na;
+        r.nb = nb;
+        r.kpad = (nb + 15) / 16 * 16;
+        if (r.type == 2) {
+            r.slot_a = slot[lp.child_a[t]];
+            r.slot_b = slot[lp.child_b[t]];
+        }
+        int32_t spg = std::max(1, gc / na);
+        int32_t ng = (n_out + spg - 1) / spg;
+        spg = (n_out + ng - 1) / ng;  // balanced groups
+        r.n_groups = ng;
+        r.s_per_group = spg;
+        r.n_group = (spg * na + 15) / 16 * 16;
+        // per-sum scale exponents: w' = w 2^k with max_ij w' in [1, 2)
+        const std::vector<double> &W = lp.raw[t];
+        while (p.fparams.size() % 4) p.fparams.push_back(0.f);
+        r.blk_off = (int64_t)p.fparams.size();
+        std::vector<double> scale(n_out, 1.0);
+        for (int32_t s2 = 0; s2 < n_out; ++s2) {
+            double mx = 0.0;
+            for (int64_t c = 0; c < (int64_t)na * nb; ++c) mx = std::max(mx, W[(size_t)s2 * na * nb + c]);
+            const int k = mx > 0.0 ? -(int)std::floor(std::log2(mx)) : 0;
+            scale[s2] = std::ldexp(1.0, k);
+            p.fparams.push_back((float)k);
+        }
+        while (p.fparams.size() % 4) p.fparams.push_back(0.f);
+        r.w_group_bytes = (int64_t)r.n_group * r.kpad * 2;
+        while (p.wimg.size() % 64) p.wimg.push_back(0);  // 128-byte aligned images
+        r.w_off = (int64_t)p.wimg.size() * 2;
+        const size_t gel = (size_t)r.n_group * r.kpad;
+        for (int32_t gi = 0; gi < ng; ++gi) {
+            std::vector<uint16_t> hi(gel, 0), lo(gel, 0);
+            for (int32_t sl = 0; sl < spg; ++sl) {
+                const int32_t s2 = gi * spg + sl;
+                if (s2 >= n_out) break;
+                for (int32_t i = 0; i < na; ++i)
+                    for (int32_t j = 0; j < nb; ++j) {
+                        const int32_t row = sl * na + i;
+                        const double w = W[(size_t)s2 * na * nb + (size_t)i * nb + j] * scale[s2];
+                        const uint16_t h = f32_to_f16((float)w);
+                        const uint16_t l = f32_to_f16((float)(w - (double)f16_to_f32(h)));
+                        const size_t idx = (size_t)(j / 8) * ((size_t)r.n_group / 8) * 64 +
+                                           (size_t)(row / 8) * 64 + (size_t)(row % 8) * 8 +
+                                           (size_t)(j % 8);
+                        hi[idx] = h;
+                        lo[idx] = l;
+                    }
+            }
+            p.wimg.insert(p.wimg.end(), hi.begin(), hi.end());
+            p.wimg.insert(p.wimg.end(), lo.begin(), lo.end());
+        }
+        p.max_wgroup = std::max<int32_t>(p.max_wgroup, (int32_t)r.w_group_bytes);
+        p.n_sum++;
+        p.steps.push_back(r);
+    }
+    p.root_map = lp.root_map;
+    p.ok = true;
 }
 
 }  // namespace spnb

@@ -59,6 +59,80 @@ struct LayeredPlan {
     int64_t fma_per_sample = 0;
     int64_t mufu_per_sample = 0;
     int64_t n_leaf_regions = 0, n_sum_regions = 0;
+    // region tree kept for the v2 kernel (rat2.cu): per step the child steps
+    // (SUM / ROOT) and the unpacked parameters -- SUM / ROOT: linear weights
+    // W[s][i][j] (na x nb cells per sum); LEAF: a[v][i], b[v][i] (log2-domain
+    // Gaussian constants, log2 N = c - (a x - b)^2) then C[i] = sum_v c_vi
+    std::vector<int32_t> child_a, child_b;
+    std::vector<std::vector<double>> raw;
+    // weight range (the v1 kernel stores weights unscaled as f16 hi/lo: a
+    // weight >= 65504 would be inf, a non-zero one < 2^-24 would flush to 0)
+    double w_min_nz = 0.0, w_max = 0.0;
+};
+
+// ---------------------------------------------------------------- v2 plan
+// Plan of the warp-specialised layered kernel (rat2.cu).  Accepted when
+// every repetition is a complete binary region tree whose partitions pair
+// either two leaf regions ("BOT") or two sum regions ("UP"), with uniform
+// leaf-region width I (multiple of 4, <= 48) and sum-region width S.
+struct R2Step {
+    int32_t type;        // 0 LEAF, 1 BOT (children: two leaf regions), 2 UP (two sum regions)
+    int32_t root;        // 1: the outputs are root (class) values, accumulated over repetitions
+    int32_t n_out, na, nb, kpad;
+    int32_t n_groups, s_per_group, n_group;  // N groups: sums per group, columns (x16)
+    int32_t slot_a, slot_b, slot_out;        // TMEM activation slots (1-based; UP inputs, output)
+    int32_t n_vars;      // LEAF: variables of the region
+    int32_t pad_;
+    int64_t vars_off;    // LEAF: int32 offset into vars
+    int64_t blk_off;     // LEAF: float offset of the block (a,b)[v][I], C[I]; SUM: kscale[n_out]
+    int64_t blk_floats;  // LEAF: block size in floats (multiple of 4)
+    int64_t w_off;       // SUM: byte offset of the group images (group-major, [hi, lo] per group)
+    int64_t w_group_bytes;  // bytes of one (group, part) image
+};
+
+struct Rat2Plan {
+    bool ok = false;
+    std::string why;
+    int32_t F = 0, C = 0, I = 0, S = 0, D = 0;  // D: TMEM activation slots used (1..D)
+    int32_t max_vars = 0, max_blk = 0;          // largest leaf region / parameter block (floats)
+    int32_t kpad_bot = 0, kpad_up = 0;          // K of the BOT / UP contractions (x16)
+    int32_t max_wgroup = 0;                     // bytes of the largest (group, part) image
+    int32_t gcols = 0;                          // TMEM columns per accumulator buffer
+    int32_t ea_max = 0;                         // max(I, S) rounded up to 8
+    std::vector<R2Step> steps;
+    std::vector<int32_t> vars;
+    std::vector<float> fparams;                 // leaf blocks, then per-sum scale exponents
+    std::vector<uint16_t> wimg;                 // f16 images
+    std::vector<int32_t> root_map;
+    int64_t n_leaf = 0, n_sum = 0;
+};
+
+// Builds the v2 plan from a detected layered plan; fails (ok = false, why)
+// when the structure is outside the v2 kernel's constraints.
+void build_rat2(const LayeredPlan &lp, Rat2Plan &p);
+
+// Kernel parameters of rat2_kernel.
+struct R2Params {
+    const R2Step *steps;
+    int32_t n_steps;
+    int32_t C, I, S;
+    const int32_t *vars;
+    const float *fparams;
+    const uint8_t *wimg;
+    const int32_t *root_map;
+    const float *xT;      // transposed features [F][ldT]
+    int64_t ldT;
+    int64_t n;            // samples in this launch (rows of xT used)
+    float *out;
+    int32_t *argmax;
+    int32_t prec;         // 1: one f16 pass; 3: hi/lo split (3 MMAs)
+    int32_t max_vars, max_blk, kpad_bot, kpad_up, max_wgroup, gcols, D;
+    int32_t n_in, n_w;    // ring depths: leaf inputs, weight groups
+    // shared-memory carve-up (byte offsets, computed on the host)
+    int32_t off_in, in_bytes, off_ea, ea_bytes, off_bimg, bimg_bytes, off_uimg, uimg_bytes,
+        off_w, w_bytes, off_bar;
+    int32_t smem_bytes;
+    unsigned long long *prof;  // optional: per-role phase cycles [4 roles][8] (SPNB_PROFILE)
 };
 
 // Detects the structure; on success fills plan (ok = true).

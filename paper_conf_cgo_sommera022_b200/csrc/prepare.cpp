@@ -93,7 +93,10 @@ int validate_graph(const GraphData &g, std::string &msg) {
                         return fail(msg, SPN_E_GRAPH, "histogram %lld: bucket %lld needs integer lb < ub", u, b / 3);
                     if (!(pr >= 0.0 && pr <= 1.0))
                         return fail(msg, SPN_E_GRAPH, "histogram %lld: bucket %lld probability not in [0,1]", u, b / 3);
-                    if (std::fabs(lb) > 1e9 || std::fabs(ub) > 1e9)
+                    // fp32 inputs are exact integers only up to 2^24: the kernels compare
+                    // x against the bounds in fp32 (larger bounds could
+                    // index outside the table)
+                    if (std::fabs(lb) > 16777216.0 || std::fabs(ub) > 16777216.0)
                         return fail(msg, SPN_E_UNSUPPORTED, "histogram %lld: bounds too large", u);
                     iv.push_back({lb, ub});
                     lo = std::min(lo, lb);
@@ -386,7 +389,7 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
         } else if (c.kind[u] == SPN_SUM) {
             out.n_sums++;
             out.n_sum_edges += nc;
-            out.mufu_per_sample += nc + 1;
+            out.mufu_per_sample += nc > 1 ? nc : 0;  // n-ary LSE: n-1 ex2 + 1 lg2
             out.fma_per_sample += 3 * nc;
         } else {
             out.n_products++;

@@ -1,0 +1,845 @@
+// rat2.cu -- warp-specialised layered RAT-SPN kernel for sm_100a (KB2/KC2).
+//
+// Same method as rat_eval.cu (§V-B: leaf regions of
+// factorised Gaussians, partitions = cross products of two regions, sum
+// regions of S weighted sums; semantics of every node L82-86), restructured
+// so that the FP32 leaf layer, the tensor-core contractions and the FP32
+// epilogues of DIFFERENT regions run concurrently on one SM:
+//
+//   warps 0-7   two LEAF groups of 4 warps.  Group 0 evaluates the left
+//               (A-side) leaf region of every bottom partition, group 1 the
+//               right (B-side) one: L[i][m] = C_i - sum_v (a_iv x_mv - b_iv)^2
+//               (log2), then the per-sample shift h = max_i L and the exps.
+//               A side -> ea[i][m] (fp32, shared memory); B side -> the f16
+//               UMMA operand image of eb'[m][j] = 2^(L_j - h + 15).
+//   warps 8-11  EPILOGUE, one thread per sample (= TMEM lane).  For every
+//               sum step: out_s = ha + hb + lg2(sum_i ea_i T[m,(s,i)]) - k_s,
+//               T read from TMEM; upper-level shifts / exps / operand images;
+//               the root's online log-sum-exp over repetitions.  Sum-region
+//               outputs wait in TMEM "activation slots" for their parent.
+//   warp 12     PRODUCER: TMA bulk copies of each leaf region's transposed
+//               feature rows + parameter block, and of every weight group.
+//   warp 13     MMA: tcgen05.mma (kind::f16, M=128) per weight group,
+//               T[m,(s,i)] = sum_j eb'[m,j] W'[s,i,j] into a double-buffered
+//               TMEM accumulator; completion by tcgen05.commit -> mbarrier.
+//
+// Every hand-off is an mbarrier ring (full/empty), so no role waits for the
+// CTA: while the epilogue finishes repetition r's upper levels the leaf
+// groups already compute the next leaf regions and the producer streams
+// the next weight groups.  One persistent CTA per SM walks 128-sample tiles.
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <stdint.h>
+
+#include "layered.h"
+
+namespace spnb {
+namespace r2 {
+
+constexpr int RT = 128;           // samples per tile = UMMA M = TMEM lanes
+// 16 warps = 4 warpgroups: leaf group 0, leaf group 1, epilogue, and
+// {leaf producer, MMA, weight producer, idle}.  setmaxnreg moves registers
+// from the last warpgroup (40 each) to the epilogue (216 each); the leaf
+// warpgroups keep the launch's 128: 2*128 + 216 + 40 = 512 per SMSP lane.
+constexpr int NTHREADS = 16 * 32;
+constexpr int W_EPI0 = 8, W_PROD = 12, W_MMA = 13, W_WPROD = 14;
+constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
+
+__device__ __forceinline__ float ex2(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float lg2(float x) {
+    float y;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float maxnan(float a, float b) {
+    float r;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+// log2(2^a + 2^b), NaN-propagating, -inf safe
+__device__ __forceinline__ float lse2(float a, float b) {
+    const float hi = maxnan(a, b), lo = fminf(a, b);
+    return hi + lg2(1.f + ex2(lo - fmaxf(hi, -1e30f)));
+}
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// ---- mbarriers -------------------------------------------------------------
+__device__ __forceinline__ void bar_init(uint32_t b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(b), "r"(count));
+}
+__device__ __forceinline__ void bar_wait(uint32_t b, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}\n"
+            : "=r"(done)
+            : "r"(b), "r"(parity)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void bar_arrive(uint32_t b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(b) : "memory");
+}
+__device__ __forceinline__ void bar_expect_tx(uint32_t b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes,
+                                         uint32_t b) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            dst),
+        "l"(src), "r"(bytes), "r"(b)
+        : "memory");
+}
+__device__ __forceinline__ void fence_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ---- tcgen05 -----------------------------------------------------------------
+__device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    // K-major, no swizzle: core matrices of 8 rows x 16 bytes; LBO = stride
+    // between core matrices along K, SBO = along M/N; version 1 (sm_100)
+    uint64_t d = 0;
+    d |= (uint64_t)((addr >> 4) & 0x3FFFu);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+    d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+    d |= (uint64_t)1 << 46;
+    return d;
+}
+__device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc,
+                                         uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void umma_commit(uint32_t b) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(b)
+                 : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, float *v) {
+    uint32_t r[8];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = __uint_as_float(r[k]);
+}
+__device__ __forceinline__ void tmem_ld4(uint32_t taddr, float *v) {
+    uint32_t r[4];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+                 : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = __uint_as_float(r[k]);
+}
+__device__ __forceinline__ void tmem_ld1(uint32_t taddr, float &v) {
+    uint32_t r;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%1];" : "=r"(r) : "r"(taddr));
+    v = __uint_as_float(r);
+}
+__device__ __forceinline__ void tmem_st1(uint32_t taddr, float v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr),
+                 "r"(__float_as_uint(v)));
+}
+__device__ __forceinline__ void tmem_wait_ld() {
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() {
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+
+// byte offset of element (row, k) of a K-major no-swizzle f16 operand image
+// with RT rows
+__device__ __forceinline__ uint32_t img_off(int row, int k) {
+    return (uint32_t)((k >> 3) * (RT * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
+}
+__device__ __forceinline__ uint32_t pack_h2(float a, float b) {
+    const __half ha = __float2half_rn(a), hb = __float2half_rn(b);
+    return (uint32_t)__half_as_ushort(ha) | ((uint32_t)__half_as_ushort(hb) << 16);
+}
+// hi/lo split of a pair: hi = f16(v), lo = f16(v - hi)
+__device__ __forceinline__ void split_h2(float a, float b, uint32_t &hi, uint32_t &lo) {
+    const __half ha = __float2half_rn(a), hb = __float2half_rn(b);
+    hi = (uint32_t)__half_as_ushort(ha) | ((uint32_t)__half_as_ushort(hb) << 16);
+    lo = pack_h2(a - __half2float(ha), b - __half2float(hb));
+}
+
+// optional phase-cycle counters (R2Params::prof, SPNB_PROFILE=1): every role
+// attributes the cycles since its previous mark to a phase; lane 0 of each
+// role's warps adds them to prof[role * 8 + phase] at exit
+__device__ __forceinline__ long long clk64() {
+    long long t;
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
+    return t;
+}
+struct Prof {
+    unsigned long long *acc;  // shared-memory counters of this role (nullptr: off)
+    long long t;
+    __device__ Prof(unsigned long long *a, bool on) : acc(on ? a : nullptr), t(clk64()) {}
+    __device__ __forceinline__ void mark(int k) {
+        if (acc) {
+            const long long now = clk64();
+            if ((threadIdx.x & 31) == 0) atomicAdd(acc + k, (unsigned long long)(now - t));
+            t = now;
+        }
+    }
+};
+
+// shared-memory layout: barrier indices
+enum {
+    B_IN_FULL = 0,    // [4]
+    B_IN_EMPTY = 4,   // [4]
+    B_A_FULL = 8,     // [2]
+    B_A_EMPTY = 10,   // [2]
+    B_B_FULL = 12,    // [2]
+    B_B_EMPTY = 14,   // [2]
+    B_U_FULL = 16,
+    B_U_EMPTY = 17,
+    B_W_FULL = 18,    // [4]
+    B_W_EMPTY = 22,   // [4]
+    B_T_FULL = 26,    // [2]
+    B_T_EMPTY = 28,   // [2]
+    B_COUNT = 30
+};
+
+struct Smem {
+    // offsets are read from the kernel parameter (constant bank) at each use
+    // instead of being copied into registers that live across the role loops
+    uint8_t *base;
+    const R2Params &p;
+    __device__ Smem(uint8_t *b, const R2Params &pp) : base(b), p(pp) {}
+    __device__ uint32_t bar(int i) const { return smem_u32(base + p.off_bar) + 8u * (uint32_t)i; }
+    // profiling counters: [4 roles][8] after the barriers and the TMEM slot
+    __device__ unsigned long long *prof(int role) const {
+        return reinterpret_cast<unsigned long long *>(base + p.off_bar + 8 * B_COUNT + 16) + role * 8;
+    }
+    __device__ float *in_x(int s) const {
+        return reinterpret_cast<float *>(base + p.off_in + s * p.in_bytes);
+    }
+    __device__ float *in_prm(int s) const { return in_x(s) + p.max_vars * RT; }
+    __device__ float *ea(int s) const {
+        return reinterpret_cast<float *>(base + p.off_ea + s * p.ea_bytes);
+    }
+    // per A-slot: ea[I][RT], ha[RT], hb[RT]
+    __device__ float *ha(int s) const { return ea(s) + p.I * RT; }
+    __device__ float *hb(int s) const { return ha(s) + RT; }
+    __device__ uint8_t *bimg(int s) const { return base + p.off_bimg + s * p.bimg_bytes; }
+    __device__ uint8_t *uimg() const { return base + p.off_uimg; }
+    __device__ uint8_t *wbuf(int s) const { return base + p.off_w + s * p.w_bytes; }
+};
+
+// ============================================================== LEAF groups
+// Thread (gw, q, b): samples m0 = 32 gw + 4 q .. +3, distributions
+// d0 = b DPB .. +DPB-1 (DPB = I / 4).  Per variable: one LDS.128 of the four
+// samples' features (a warp reads 128 contiguous bytes) and DPB/2 LDS.128 of
+// (a, b) pairs (4 distinct addresses per warp), then 2 DPB FFMA2.
+template <int DPB, bool MARG>
+__device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, int V, int I,
+                                             int m0, int d0, float (&acc)[DPB][4]) {
+    const float *C = prm + 2 * V * I;
+#pragma unroll
+    for (int d = 0; d < DPB; ++d) {
+        const float c = C[d0 + d];
+        acc[d][0] = c; acc[d][1] = c; acc[d][2] = c; acc[d][3] = c;
+    }
+    const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi): c_v = log2(a) + K0
+    const float4 *ab4 = reinterpret_cast<const float4 *>(prm + 2 * d0);
+    const int vstride = I / 2;  // float4 per variable
+#pragma unroll 4
+    for (int v = 0; v < V; ++v) {
+        const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + m0);
+        float2 q[DPB];
+#pragma unroll
+        for (int k = 0; k < DPB / 2; ++k) {
+            const float4 t = ab4[v * vstride + k];
+            q[2 * k] = make_float2(t.x, t.y);
+            q[2 * k + 1] = make_float2(t.z, t.w);
+        }
+        bool anynan = false;
+        if constexpr (MARG) anynan = (x4.x != x4.x) | (x4.y != x4.y) | (x4.z != x4.z) | (x4.w != x4.w);
+        if (MARG && anynan) {
+            const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
+#pragma unroll
+            for (int d = 0; d < DPB; ++d) {
+                const float cc = lg2(q[d].x) + K0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const bool nan = xv[k] != xv[k];
+                    const float t = fmaf(q[d].x, xv[k], -q[d].y);
+                    acc[d][k] = fmaf(-(nan ? cc : t), nan ? 1.f : t, acc[d][k]);
+                }
+            }
+        } else {
+            const float2 x01 = make_float2(x4.x, x4.y), x23 = make_float2(x4.z, x4.w);
+#pragma unroll
+            for (int d = 0; d < DPB; ++d) {
+                const float2 a2 = make_float2(q[d].x, q[d].x), nb2 = make_float2(-q[d].y, -q[d].y);
+                const float2 t01 = __ffma2_rn(x01, a2, nb2);
+                const float2 t23 = __ffma2_rn(x23, a2, nb2);
+                const float2 s01 = __ffma2_rn(make_float2(-t01.x, -t01.y), t01,
+                                              make_float2(acc[d][0], acc[d][1]));
+                const float2 s23 = __ffma2_rn(make_float2(-t23.x, -t23.y), t23,
+                                              make_float2(acc[d][2], acc[d][3]));
+                acc[d][0] = s01.x; acc[d][1] = s01.y; acc[d][2] = s23.x; acc[d][3] = s23.y;
+            }
+        }
+    }
+}
+
+template <int DPB, bool MARG>
+__device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
+                          int n_leaf, int warp, int lane) {
+    const int g = warp >> 2, gw = warp & 3;
+    const int q = lane >> 2, b = lane & 3;
+    const int m0 = gw * 32 + q * 4, d0 = b * DPB;
+    const int I = p.I;
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint32_t li = (uint32_t)g;  // global leaf-region counter of this group (step 2)
+    uint32_t j = 0;             // this group's region count = bottom-partition counter
+    Prof pf(sm.prof(0), p.prof != nullptr);  // 0 wait input, 1 compute, 2 shifts, 3 wait output slot, 4 exps + write
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int l = g; l < n_leaf; l += 2, li += 2, ++j) {
+            const R2Step &st = p.steps[leaf_steps[l]];
+            const int s = (int)(li % (uint32_t)p.n_in);
+            bar_wait(sm.bar(B_IN_FULL + s), (li / (uint32_t)p.n_in) & 1u);
+            pf.mark(0);
+            float acc[DPB][4];
+            leaf_compute<DPB, MARG>(sm.in_x(s), sm.in_prm(s), st.n_vars, I, m0, d0, acc);
+            __syncwarp();
+            if (lane == 0) bar_arrive(sm.bar(B_IN_EMPTY + s));
+            pf.mark(1);
+            // per-sample shift over the I distributions: local max over DPB,
+            // then across the 4 lanes of the sample quad (xor 1, 2)
+            float h[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                float v = acc[0][k];
+#pragma unroll
+                for (int d = 1; d < DPB; ++d) v = maxnan(v, acc[d][k]);
+                v = maxnan(v, __shfl_xor_sync(0xffffffffu, v, 1));
+                v = maxnan(v, __shfl_xor_sync(0xffffffffu, v, 2));
+                h[k] = v;
+            }
+            const int ab = (int)(j & 1u);
+            const uint32_t ph = (j >> 1) & 1u;
+            pf.mark(2);
+            // both sides wait for the A slot (it also carries hb)
+            bar_wait(sm.bar(B_A_EMPTY + ab), ph ^ 1u);
+            if (g == 1) bar_wait(sm.bar(B_B_EMPTY + ab), ph ^ 1u);
+            pf.mark(3);
+            if (g == 0) {
+                float *ea = sm.ea(ab);
+#pragma unroll
+                for (int d = 0; d < DPB; ++d) {
+                    float e[4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) e[k] = ex2(acc[d][k] - fmaxf(h[k], -1e30f));
+                    *reinterpret_cast<float4 *>(ea + (d0 + d) * RT + m0) =
+                        make_float4(e[0], e[1], e[2], e[3]);
+                }
+                if (b == 0)
+                    *reinterpret_cast<float4 *>(sm.ha(ab) + m0) = make_float4(h[0], h[1], h[2], h[3]);
+                bar_arrive(sm.bar(B_A_FULL + ab));
+            } else {
+                uint8_t *img = sm.bimg(ab);
+                const int part = p.bimg_bytes / 2;  // lo image after hi (prec 3)
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const float hc = fmaxf(h[k], -1e30f) - EB_SHIFT;
+#pragma unroll
+                    for (int d = 0; d < DPB; d += 2) {
+                        const float e0 = ex2(acc[d][k] - hc), e1 = ex2(acc[d + 1][k] - hc);
+                        const uint32_t o = img_off(m0 + k, d0 + d);
+                        if (p.prec == 3) {
+                            uint32_t hi, lo;
+                            split_h2(e0, e1, hi, lo);
+                            *reinterpret_cast<uint32_t *>(img + o) = hi;
+                            *reinterpret_cast<uint32_t *>(img + part + o) = lo;
+                        } else {
+                            *reinterpret_cast<uint32_t *>(img + o) = pack_h2(e0, e1);
+                        }
+                    }
+                }
+                if (b == 0)
+                    *reinterpret_cast<float4 *>(sm.hb(ab) + m0) =
+                        make_float4(h[0] - EB_SHIFT, h[1] - EB_SHIFT, h[2] - EB_SHIFT, h[3] - EB_SHIFT);
+                fence_async_smem();
+                bar_arrive(sm.bar(B_B_FULL + ab));
+            }
+            pf.mark(4);
+        }
+    }
+}
+
+// ============================================================== PRODUCERS
+// Two warps so leaf inputs never queue behind weight groups (the weight
+// ring drains at the pace of the epilogue): warp W_PROD streams each leaf
+// region's feature rows + parameter block, warp W_WPROD every weight group.
+__device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
+                                   int n_leaf, int lane) {
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint32_t li = 0;
+    Prof pf(sm.prof(3), p.prof != nullptr);  // 0 wait leaf slot, 7 issue
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        const int64_t base = tile * RT;
+        for (int l = 0; l < n_leaf; ++l, ++li) {
+            const R2Step &st = p.steps[leaf_steps[l]];
+            const int s = (int)(li % (uint32_t)p.n_in);
+            pf.mark(7);
+            bar_wait(sm.bar(B_IN_EMPTY + s), ((li / (uint32_t)p.n_in) & 1u) ^ 1u);
+            pf.mark(0);
+            const uint32_t full = sm.bar(B_IN_FULL + s);
+            const uint32_t pbytes = (uint32_t)st.blk_floats * 4;
+            const uint32_t dst = smem_u32(sm.in_x(s));
+            if (lane == 0) {
+                bar_expect_tx(full, (uint32_t)st.n_vars * RT * 4 + pbytes);
+                bulk_g2s(smem_u32(sm.in_prm(s)), p.fparams + st.blk_off, pbytes, full);
+            }
+            __syncwarp();
+            for (int v = lane; v < st.n_vars; v += 32) {
+                const int f = __ldg(p.vars + st.vars_off + v);
+                bulk_g2s(dst + v * RT * 4, p.xT + (int64_t)f * p.ldT + base, RT * 4, full);
+            }
+        }
+    }
+    pf.mark(7);
+}
+
+__device__ void weight_producer_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps,
+                                     int n_sum, int lane) {
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint32_t wi = 0;
+    const int parts = p.prec == 3 ? 2 : 1;
+    Prof pf(sm.prof(3), p.prof != nullptr);  // 2 wait weight slot, 7 issue
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int si = 0; si < n_sum; ++si) {
+            const R2Step &st = p.steps[sum_steps[si]];
+            const uint32_t gb = (uint32_t)st.w_group_bytes;
+            for (int gi = 0; gi < st.n_groups; ++gi, ++wi) {
+                const int s = (int)(wi % (uint32_t)p.n_w);
+                pf.mark(7);
+                bar_wait(sm.bar(B_W_EMPTY + s), ((wi / (uint32_t)p.n_w) & 1u) ^ 1u);
+                pf.mark(2);
+                const uint32_t full = sm.bar(B_W_FULL + s);
+                if (lane == 0) {
+                    bar_expect_tx(full, gb * parts);
+                    const uint8_t *src = p.wimg + st.w_off + (size_t)2 * gb * gi;
+                    for (int pt = 0; pt < parts; ++pt)
+                        bulk_g2s(smem_u32(sm.wbuf(s)) + pt * (uint32_t)p.max_wgroup,
+                                 src + (size_t)pt * gb, gb, full);
+                }
+                __syncwarp();
+            }
+        }
+    }
+    pf.mark(7);
+}
+
+// ============================================================== MMA issuer
+__device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps, int n_sum,
+                         uint32_t tmem, int lane) {
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint32_t kb = 0, ku = 0, wi = 0, ti = 0;
+    const uint32_t lbo_a = RT * 16;
+    Prof pf(sm.prof(2), p.prof != nullptr);  // 0 wait A operand, 1 wait weights, 2 wait TMEM buffer, 3 issue
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int si = 0; si < n_sum; ++si) {
+            const R2Step &st = p.steps[sum_steps[si]];
+            const bool bot = st.type == 1;
+            uint32_t a_hi;
+            if (bot) {
+                const int ab = (int)(kb & 1u);
+                bar_wait(sm.bar(B_B_FULL + ab), (kb >> 1) & 1u);
+                a_hi = smem_u32(sm.bimg(ab));
+            } else {
+                bar_wait(sm.bar(B_U_FULL), ku & 1u);
+                a_hi = smem_u32(sm.uimg());
+            }
+            pf.mark(0);
+            const uint32_t a_lo = a_hi + (uint32_t)(bot ? p.bimg_bytes : p.uimg_bytes) / 2;
+            const uint32_t lbo_b = (uint32_t)st.n_group * 16;
+            const uint32_t idesc = (1u << 4) | ((uint32_t)(st.n_group >> 3) << 17) |
+                                   ((uint32_t)(RT >> 4) << 24);
+            for (int gi = 0; gi < st.n_groups; ++gi, ++wi, ++ti) {
+                const int ws = (int)(wi % (uint32_t)p.n_w);
+                const int tb = (int)(ti & 1u);
+                pf.mark(3);
+                bar_wait(sm.bar(B_W_FULL + ws), (wi / (uint32_t)p.n_w) & 1u);
+                pf.mark(1);
+                bar_wait(sm.bar(B_T_EMPTY + tb), ((ti >> 1) & 1u) ^ 1u);
+                pf.mark(2);
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t w_hi = smem_u32(sm.wbuf(ws)), w_lo = w_hi + (uint32_t)p.max_wgroup;
+                    const uint32_t d = tmem + (uint32_t)(tb * p.gcols);
+                    for (int kk = 0; kk < st.kpad / 16; ++kk) {
+                        const uint32_t ka = kk * 2 * lbo_a, kw = kk * 2 * lbo_b;
+                        umma_f16(d, umma_desc(a_hi + ka, lbo_a, 128), umma_desc(w_hi + kw, lbo_b, 128),
+                                 idesc, kk > 0);
+                        if (p.prec == 3) {
+                            umma_f16(d, umma_desc(a_lo + ka, lbo_a, 128),
+                                     umma_desc(w_hi + kw, lbo_b, 128), idesc, 1);
+                            umma_f16(d, umma_desc(a_hi + ka, lbo_a, 128),
+                                     umma_desc(w_lo + kw, lbo_b, 128), idesc, 1);
+                        }
+                    }
+                    umma_commit(sm.bar(B_T_FULL + tb));
+                    umma_commit(sm.bar(B_W_EMPTY + ws));
+                }
+                __syncwarp();
+            }
+            if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb & 1u) : B_U_EMPTY));
+            __syncwarp();
+            if (bot) ++kb;
+            else ++ku;
+            pf.mark(3);
+        }
+    }
+}
+
+// ============================================================== EPILOGUE
+// Thread = sample m = TMEM lane.  TMEM columns: [0, 2 gcols) accumulators,
+// then D activation slots of S columns, then C root accumulators.  Widths
+// are template parameters (I: leaf regions, S: sum regions), so a sum's
+// stage-2 contraction is straight-line code: its columns are read in units
+// of U <= 24 columns, double-buffered (the next unit's tcgen05.ld is in
+// flight while this unit's FFMA2s run; tcgen05.wait::ld waits for both).
+
+// descriptor fields the epilogue needs, prefetched one step ahead
+struct EStep {
+    int type, root, n_out, n_groups, spg, slot_a, slot_b, slot_out;
+    int64_t ks_off;
+};
+__device__ __forceinline__ EStep load_estep(const R2Step *steps, const int32_t *idx, int si) {
+    const R2Step &st = steps[__ldg(idx + si)];
+    return EStep{st.type, st.root, st.n_out, st.n_groups, st.s_per_group,
+                 st.slot_a, st.slot_b, st.slot_out, st.blk_off};
+}
+
+template <int U>
+__device__ __forceinline__ void ld_unit(uint32_t taddr, float (&t)[U]) {
+#pragma unroll
+    for (int c = 0; c + 8 <= U; c += 8) tmem_ld8(taddr + c, t + c);
+    if constexpr (U % 8) tmem_ld4(taddr + (U / 8) * 8, t + (U / 8) * 8);
+}
+template <int W>
+__device__ __forceinline__ void ld_unit_any(uint32_t taddr, float (&t)[W]) {
+#pragma unroll
+    for (int c = 0; c + 8 <= W; c += 8) tmem_ld8(taddr + c, t + c);
+    if constexpr (W % 8) tmem_ld4(taddr + (W / 8) * 8, t + (W / 8) * 8);
+}
+template <int U>
+__device__ __forceinline__ float dot_unit(const float *ea, const float (&t)[U]) {
+    float2 p0 = make_float2(0.f, 0.f), p1 = make_float2(0.f, 0.f);
+#pragma unroll
+    for (int i = 0; i + 4 <= U; i += 4) {
+        p0 = __ffma2_rn(make_float2(ea[i], ea[i + 1]), make_float2(t[i], t[i + 1]), p0);
+        p1 = __ffma2_rn(make_float2(ea[i + 2], ea[i + 3]), make_float2(t[i + 2], t[i + 3]), p1);
+    }
+    return (p0.x + p0.y) + (p1.x + p1.y);
+}
+
+// One sum step's groups: out_s = shift + lg2(sum_i ea_i T[s, i]) - k_s.
+template <int NA, bool ROOT>
+__device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const EStep &es,
+                                           const float (&ear)[NA], float shift, uint32_t lane_base,
+                                           uint32_t out_col, uint32_t col_root, uint32_t &ti,
+                                           Prof &pf) {
+    constexpr int U = NA > 24 ? NA / 2 : NA;  // columns per load unit
+    constexpr int UPS = NA / U;               // units per sum (1 or 2)
+    static_assert(U % 4 == 0 && U <= 24 && UPS * U == NA, "unit width");
+    const float *ks = p.fparams + es.ks_off;
+    for (int gi = 0; gi < es.n_groups; ++gi, ++ti) {
+        const int tb = (int)(ti & 1u);
+        const int s0 = gi * es.spg;
+        const int s1 = min(es.n_out, s0 + es.spg);
+        pf.mark(3);
+        bar_wait(sm.bar(B_T_FULL + tb), (ti >> 1) & 1u);
+        pf.mark(2);
+        tc_fence_after();
+        const uint32_t acc0 = lane_base + (uint32_t)(tb * p.gcols);
+        float b0[U], b1[U];
+        auto fin = [&](int s, float a) {
+            const float val = shift + lg2(a) - __ldg(ks + s);
+            if constexpr (ROOT) {
+                const uint32_t c = col_root + (uint32_t)__ldg(p.root_map + s);
+                float r;
+                tmem_ld1(lane_base + c, r);
+                tmem_wait_ld();
+                tmem_st1(lane_base + c, lse2(r, val));
+            } else {
+                tmem_st1(lane_base + out_col + s, val);
+            }
+        };
+        ld_unit<U>(acc0, b0);
+        tmem_wait_ld();
+        if constexpr (UPS == 2) {
+            for (int s = s0; s < s1; ++s) {
+                const uint32_t row = acc0 + (uint32_t)((s - s0) * NA);
+                ld_unit<U>(row + U, b1);                  // second half of s
+                float a = dot_unit<U>(ear, b0);
+                tmem_wait_ld();
+                if (s + 1 < s1) ld_unit<U>(row + NA, b0);  // first half of s + 1
+                a += dot_unit<U>(ear + U, b1);
+                fin(s, a);
+                if (s + 1 < s1) tmem_wait_ld();
+            }
+        } else {
+            for (int s = s0; s < s1; s += 2) {
+                const uint32_t row = acc0 + (uint32_t)((s - s0) * NA);
+                if (s + 1 < s1) ld_unit<U>(row + NA, b1);
+                fin(s, dot_unit<U>(ear, b0));
+                if (s + 1 < s1) {
+                    tmem_wait_ld();
+                    if (s + 2 < s1) ld_unit<U>(row + 2 * NA, b0);
+                    fin(s + 1, dot_unit<U>(ear, b1));
+                    if (s + 2 < s1) tmem_wait_ld();
+                }
+            }
+        }
+        tc_fence_before();
+        bar_arrive(sm.bar(B_T_EMPTY + tb));
+    }
+}
+
+template <int I, int S, bool MARG>
+__device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps,
+                              int n_sum, uint32_t tmem, int warp, int lane) {
+    const int qd = warp & 3;
+    const int m = qd * 32 + lane;
+    const uint32_t lane_base = tmem + ((uint32_t)(qd * 32) << 16);
+    const uint32_t col_slots = 2u * (uint32_t)p.gcols;
+    const uint32_t col_root = col_slots + (uint32_t)(p.D * S);
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint32_t kb = 0, ku = 0, ti = 0;
+    const int part_u = p.uimg_bytes / 2;
+    constexpr int SU = S > 0 ? S : 4;
+    Prof pf(sm.prof(1), p.prof != nullptr);  // 0 wait leaf outputs, 1 UP phase 1, 2 wait TMEM full, 3 sums, 4 tile I/O, 5 step setup
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int c = 0; c < p.C; ++c) tmem_st1(lane_base + col_root + c, -CUDART_INF_F);
+        tmem_wait_st();
+        EStep nx = load_estep(p.steps, sum_steps, 0);
+        for (int si = 0; si < n_sum; ++si) {
+            const EStep es = nx;
+            if (si + 1 < n_sum) nx = load_estep(p.steps, sum_steps, si + 1);
+            pf.mark(5);
+            const uint32_t out_col = col_slots + (uint32_t)((es.slot_out - 1) * S);
+            if (es.type == 1) {
+                // BOT: ea from leaf group 0, hb from leaf group 1
+                const int ab = (int)(kb & 1u);
+                const uint32_t ph = (kb >> 1) & 1u;
+                bar_wait(sm.bar(B_A_FULL + ab), ph);
+                bar_wait(sm.bar(B_B_FULL + ab), ph);
+                pf.mark(0);
+                const float *ea = sm.ea(ab);
+                float ear[I];
+#pragma unroll
+                for (int i = 0; i < I; ++i) ear[i] = ea[i * RT + m];
+                const float shift = sm.ha(ab)[m] + sm.hb(ab)[m];
+                bar_arrive(sm.bar(B_A_EMPTY + ab));
+                ++kb;
+                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+            } else {
+                // UP: children in activation slots; B side -> f16 image, A side -> registers
+                float vb[SU], ear[SU];
+                ld_unit_any<SU>(lane_base + col_slots + (uint32_t)((es.slot_b - 1) * S), vb);
+                ld_unit_any<SU>(lane_base + col_slots + (uint32_t)((es.slot_a - 1) * S), ear);
+                tmem_wait_ld();
+                float hb = vb[0], ha = ear[0];
+#pragma unroll
+                for (int i = 1; i < SU; ++i) {
+                    hb = maxnan(hb, vb[i]);
+                    ha = maxnan(ha, ear[i]);
+                }
+                bar_wait(sm.bar(B_U_EMPTY), (ku & 1u) ^ 1u);
+                uint8_t *img = sm.uimg();
+                const float hc = fmaxf(hb, -1e30f) - EB_SHIFT;
+#pragma unroll
+                for (int i = 0; i < SU; i += 2) {
+                    const float e0 = ex2(vb[i] - hc), e1 = i + 1 < SU ? ex2(vb[i + 1] - hc) : 0.f;
+                    const uint32_t o = img_off(m, i);
+                    if (p.prec == 3) {
+                        uint32_t hi, lo;
+                        split_h2(e0, e1, hi, lo);
+                        *reinterpret_cast<uint32_t *>(img + o) = hi;
+                        *reinterpret_cast<uint32_t *>(img + part_u + o) = lo;
+                    } else {
+                        *reinterpret_cast<uint32_t *>(img + o) = pack_h2(e0, e1);
+                    }
+                }
+                fence_async_smem();
+                bar_arrive(sm.bar(B_U_FULL));
+                ++ku;
+                const float hac = fmaxf(ha, -1e30f);
+#pragma unroll
+                for (int i = 0; i < SU; ++i) ear[i] = ex2(ear[i] - hac);
+                const float shift = ha + hb - EB_SHIFT;
+                pf.mark(1);
+                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+            }
+            tmem_wait_st();
+        }
+        pf.mark(3);
+        // ---- outputs of the tile (the TMEM loads stay warp-converged)
+        const int64_t row = tile * RT + m;
+        int best = -1;
+        float bv = -CUDART_INF_F;
+        for (int c = 0; c < p.C; ++c) {
+            float r;
+            tmem_ld1(lane_base + col_root + c, r);
+            tmem_wait_ld();
+            const float v = r * 0.6931471805599453f;
+            if (row < p.n) p.out[row * p.C + c] = v;
+            if (!(v != v) && (best < 0 || v > bv)) {
+                best = c;
+                bv = v;
+            }
+        }
+        if (row < p.n && p.argmax) p.argmax[row] = best;
+        pf.mark(4);
+    }
+}
+
+template <int I, int S, bool MARG>
+__global__ void __launch_bounds__(NTHREADS, 1)
+    rat2_kernel(const R2Params p, const int32_t *__restrict__ leaf_steps, int n_leaf,
+                const int32_t *__restrict__ sum_steps, int n_sum) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *base = reinterpret_cast<uint8_t *>(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const Smem sm(base, p);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(base + p.off_bar + 8 * B_COUNT);
+    if (warp == W_MMA) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(
+            smem_u32(tmem_slot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 0) {
+        for (int i = 0; i < 4; ++i) {
+            bar_init(sm.bar(B_IN_FULL + i), 1);
+            bar_init(sm.bar(B_IN_EMPTY + i), 4);
+            bar_init(sm.bar(B_W_FULL + i), 1);
+            bar_init(sm.bar(B_W_EMPTY + i), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            bar_init(sm.bar(B_A_FULL + i), 128);
+            bar_init(sm.bar(B_A_EMPTY + i), 128);
+            bar_init(sm.bar(B_B_FULL + i), 128);
+            bar_init(sm.bar(B_B_EMPTY + i), 1);
+            bar_init(sm.bar(B_T_FULL + i), 1);
+            bar_init(sm.bar(B_T_EMPTY + i), 128);
+        }
+        bar_init(sm.bar(B_U_FULL), 128);
+        bar_init(sm.bar(B_U_EMPTY), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int k = 0; k < 32; ++k) sm.prof(0)[k] = 0;
+    }
+    // zero the operand images once (the K padding columns stay zero)
+    for (int i = tid * 16; i < 2 * p.bimg_bytes + p.uimg_bytes; i += NTHREADS * 16)
+        *reinterpret_cast<uint4 *>(base + p.off_bimg + i) = make_uint4(0, 0, 0, 0);
+    fence_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 40;");
+    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 216;");
+    if (warp < W_EPI0) {
+        leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
+    } else if (warp < W_PROD) {
+        epilogue_role<I, S, MARG>(p, sm, sum_steps, n_sum, tmem, warp, lane);
+    } else if (warp == W_PROD) {
+        leaf_producer_role(p, sm, leaf_steps, n_leaf, lane);
+    } else if (warp == W_MMA) {
+        mma_role(p, sm, sum_steps, n_sum, tmem, lane);
+    } else if (warp == W_WPROD) {
+        weight_producer_role(p, sm, sum_steps, n_sum, lane);
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (p.prof && tid < 32) atomicAdd(p.prof + tid, sm.prof(0)[tid]);
+    if (warp == W_MMA) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+    }
+}
+
+}  // namespace r2
+
+// (I, S) pairs with a compiled kernel instance (S = 0: no sum regions)
+bool rat2_supported_shape(int I, int S) {
+    static const int kShapes[][2] = {{8, 4}, {16, 8}, {40, 20}, {32, 16}, {16, 16}, {48, 24}};
+    for (auto &k : kShapes)
+        if (k[0] == I && (k[1] == S || (S == 0 && 2 * k[1] == I))) return true;
+    return false;
+}
+
+// host: shared-memory carve-up for ring depths (n_in, n_w); returns bytes
+int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int kpad_up,
+                int max_wgroup, int prec, int n_in, int n_w) {
+    const int parts = prec == 3 ? 2 : 1;
+    auto up = [](int x, int a) { return (x + a - 1) / a * a; };
+    int off = 0;
+    p.off_bar = off;
+    off += 8 * r2::B_COUNT + 16 + 4 * 8 * 8;  // barriers, TMEM slot, profiling counters
+    off = up(off, 128);
+    p.n_in = n_in;
+    p.in_bytes = up(max_vars * r2::RT * 4 + max_blk * 4, 128);
+    p.off_in = off;
+    off += n_in * p.in_bytes;
+    p.ea_bytes = up((I + 2) * r2::RT * 4, 128);
+    p.off_ea = off;
+    off += 2 * p.ea_bytes;
+    off = up(off, 1024);
+    p.bimg_bytes = r2::RT * kpad_bot * 2 * parts;
+    p.off_bimg = off;
+    off += 2 * p.bimg_bytes;
+    p.uimg_bytes = r2::RT * kpad_up * 2 * parts;
+    p.off_uimg = off;  // contiguous with the B images (zeroed together)
+    off += p.uimg_bytes;
+    off = up(off, 1024);
+    p.n_w = n_w;
+    p.w_bytes = up(max_wgroup * parts, 1024);
+    p.off_w = off;
+    off += n_w * p.w_bytes;
+    p.smem_bytes = off + 1024;  // alignment slack of the dynamic base
+    return p.smem_bytes;
+}
+
+cudaError_t rat2_launch(const R2Params &p, const int32_t *leaf_steps, int n_leaf,
+                        const int32_t *sum_steps, int n_sum, bool marg, int grid, cudaStream_t st) {
+    void (*fn)(const R2Params, const int32_t *, int, const int32_t *, int) = nullptr;
+#define R2_CASE(I_, S_)                                                                          \
+    if (p.I == I_ && (p.S == S_ || (p.S == 0 && 2 * S_ == I_)))                                  \
+        fn = marg ? r2::rat2_kernel<I_, S_, true> : r2::rat2_kernel<I_, S_, false>;
+    R2_CASE(8, 4) R2_CASE(16, 8) R2_CASE(40, 20) R2_CASE(32, 16) R2_CASE(16, 16) R2_CASE(48, 24)
+#undef R2_CASE
+    if (!fn) return cudaErrorInvalidConfiguration;
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
+    if (e != cudaSuccess) return e;
+    fn<<<grid, r2::NTHREADS, p.smem_bytes, st>>>(p, leaf_steps, n_leaf, sum_steps, n_sum);
+    return cudaGetLastError();
+}
+
+}  // namespace spnb

@@ -637,7 +637,8 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
 __global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64_t ld, int F,
                                    float *__restrict__ xT, int64_t ldT, int64_t rows_pad) {
     __shared__ float t[32][33];
-    const int64_t s0 = (int64_t)blockIdx.y * 32, f0 = (int64_t)blockIdx.x * 32;
+    // row blocks on grid.x (up to 2^31-1), feature blocks on grid.y
+    const int64_t s0 = (int64_t)blockIdx.x * 32, f0 = (int64_t)blockIdx.y * 32;
     const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
     for (int k = ty; k < 32; k += 8) {
         const int64_t s = s0 + k, f = f0 + tx;
@@ -679,7 +680,7 @@ cudaError_t rat_launch(const RParams &p, bool marg, int grid, size_t smem, cudaS
 
 cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float *xT, int64_t ldT,
                              int64_t rows_pad, cudaStream_t st) {
-    dim3 grid((unsigned)((F + 31) / 32), (unsigned)((rows_pad + 31) / 32));
+    dim3 grid((unsigned)((rows_pad + 31) / 32), (unsigned)((F + 31) / 32));
     transpose_x_kernel<<<grid, dim3(32, 8), 0, st>>>(x, n, ld, F, xT, ldT, rows_pad);
     return cudaGetLastError();
 }

@@ -1,0 +1,95 @@
+"""Test-side reference executor of the v2 layered plan (``spn_build_layered2``,
+kernel rat2.cu), in fp64 numpy with the kernel's f16 operand rounding.  It
+restates the step semantics (LEAF / BOT / UP, TMEM activation slots, per-sum
+weight scale exponents, the 2^15 shift of the B-side exps) so the detector,
+the weight images and the slot schedule can be checked against the oracle on
+the CPU.  Not used by the product path."""
+from __future__ import annotations
+
+import numpy as np
+
+EB_SHIFT = 15.0
+
+
+def _img_index(row, k, rows):
+    """f16-element index of (row, k) in a K-major no-swizzle operand image."""
+    return (k // 8) * (rows * 8) + (row // 8) * 64 + (row % 8) * 8 + (k % 8)
+
+
+def _f16_split(v, prec):
+    hi = v.astype(np.float16).astype(np.float64)
+    if prec == 3:
+        lo = (v - hi).astype(np.float16).astype(np.float64)
+        return hi + lo
+    return hi
+
+
+def _decode_weights(plan, st, prec):
+    na, nb, S = int(st["na"]), int(st["nb"]), int(st["n_out"])
+    ng, kpad, spg = int(st["n_group"]), int(st["kpad"]), int(st["s_per_group"])
+    gel = ng * kpad
+    base = int(st["w_off"]) // 2
+    wimg = plan["wimg"]
+    W = np.zeros((S, na, nb))
+    for g in range(int(st["n_groups"])):
+        hi = wimg[base + 2 * g * gel: base + 2 * g * gel + gel].astype(np.float64)
+        lo = wimg[base + 2 * g * gel + gel: base + 2 * (g + 1) * gel].astype(np.float64)
+        wg = hi + (lo if prec == 3 else 0.0)
+        for sl in range(spg):
+            s = g * spg + sl
+            if s >= S:
+                break
+            for i in range(na):
+                row = sl * na + i
+                idx = [_img_index(row, j, ng) for j in range(nb)]
+                W[s, i, :] = wg[idx]
+    return W
+
+
+def emulate_layered2(plan: dict, x: np.ndarray, marginal: bool = False, prec: int = 3):
+    steps, vars_, fp = plan["steps"], plan["vars"], plan["fparams"].astype(np.float64)
+    C, I = plan["C"], plan["I"]
+    N = x.shape[0]
+    xd = x.astype(np.float64)
+    slots = {}
+    racc = np.full((C, N), -np.inf)
+    pending = []   # leaf outputs of the current bottom partition
+    K0 = 0.5 * np.log2(np.log(2.0) / np.pi)
+    with np.errstate(invalid="ignore", divide="ignore", over="ignore"):
+        for st in steps:
+            t = int(st["type"])
+            if t == 0:
+                V = int(st["n_vars"])
+                blk = fp[int(st["blk_off"]):int(st["blk_off"]) + int(st["blk_floats"])]
+                ab = blk[:2 * V * I].reshape(V, I, 2)
+                acc = np.tile(blk[2 * V * I:2 * V * I + I][:, None], (1, N))
+                for v in range(V):
+                    xv = xd[:, int(vars_[int(st["vars_off"]) + v])]
+                    tt = ab[v, :, 0:1] * xv[None, :] - ab[v, :, 1:2]
+                    if marginal:
+                        cv = np.log2(ab[v, :, 0]) + K0
+                        acc -= np.where(np.isnan(xv)[None, :], cv[:, None], tt * tt)
+                    else:
+                        acc -= tt * tt
+                pending.append(acc)
+                continue
+            if t == 1:
+                VA, VB = pending
+                pending = []
+            else:
+                VA, VB = slots[int(st["slot_a"])], slots[int(st["slot_b"])]
+            ha = np.max(VA, axis=0)
+            hb = np.max(VB, axis=0) - EB_SHIFT
+            ea = np.exp2(VA - np.maximum(ha, -1e30))
+            eb = _f16_split(np.exp2(VB - np.maximum(hb + EB_SHIFT, -1e30) + EB_SHIFT), prec)
+            W = _decode_weights(plan, st, prec)
+            ks = fp[int(st["blk_off"]):int(st["blk_off"]) + int(st["n_out"])]
+            T = np.einsum("jm,sij->sim", eb, W)
+            val = (ha + hb)[None, :] + np.log2(np.einsum("im,sim->sm", ea, T)) - ks[:, None]
+            if int(st["root"]):
+                for s in range(int(st["n_out"])):
+                    c = int(plan["root_map"][s])
+                    racc[c] = np.logaddexp2(racc[c], val[s])
+            else:
+                slots[int(st["slot_out"])] = val
+    return (racc * np.log(2.0)).T

@@ -269,3 +269,33 @@ def test_layered_plan_matches_oracle(shape):
         # single f16 pass: weight rounding only (2^-12 relative per weight)
         em1 = emulate_layered(plan, xx, g.n_roots, marginal=marg, prec=1)
         assert (np.abs(em1 - ref) / np.maximum(1.0, np.abs(ref))).max() < 5e-3
+
+
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (24, 1, 1, 4, 8, 2),
+                                   (96, 4, 2, 20, 40, 10)])
+def test_layered2_plan_matches_oracle(shape):
+    """The v2 kernel's plan (TMEM activation slots, per-sum weight scaling,
+    group images) executed by the test-side emulator equals the oracle."""
+    from spn_inputs import rat_spn
+    from tests.layered2_emulator import emulate_layered2
+    F, D, R, S, I, C = shape
+    g = rat_spn(7, F=F, D=D, R=R, S=S, I=I, C=C)
+    plan, why = spnb.build_layered2(spnb.Graph(g))
+    assert plan is not None, why
+    assert plan["D"] == (D if D > 1 else 0)
+    x, _ = ancestral_sample(g, 120, 3)
+    for marg, xx in ((False, x), (True, nan_mask(x, 0.2, 4))):
+        ref, _ = oracle_eval(g, xx, marginal=marg)
+        em = emulate_layered2(plan, xx, marginal=marg, prec=3)
+        err = np.abs(em - ref) / np.maximum(1.0, np.abs(ref))
+        assert err.max() < 1e-5, err.max()
+        em1 = emulate_layered2(plan, xx, marginal=marg, prec=1)
+        assert (np.abs(em1 - ref) / np.maximum(1.0, np.abs(ref))).max() < 5e-3
+
+
+def test_layered2_rejects_outside_constraints():
+    from spn_inputs import rat_spn
+    p, why = spnb.build_layered2(spnb.Graph(rat_spn(7, F=32, D=2, R=2, S=4, I=12, C=3)))
+    assert p is None and "multiple of 8" in why
+    p, why = spnb.build_layered2(spnb.Graph(speaker_spn(2001)))
+    assert p is None and why

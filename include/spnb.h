@@ -101,7 +101,15 @@ typedef struct spn_prepare_options {
                                    step by step), 2 v2 (rat2.cu: warp-
                                    specialised leaf / MMA / epilogue roles;
                                    E_UNSUPPORTED if not applicable)          */
-    int32_t reserved[6];        /* must be zero                                */
+    int32_t value_space;        /* compiled path: 0 auto, 1 log2 space, 2 linear
+                                   fp32 (the paper's deferred `probability`
+                                   datatype choice).  Auto picks
+                                   linear when every leaf is discrete and
+                                   interval bounds keep every non-zero value
+                                   in [2^-100, 2^100]: sums become FFMA chains
+                                   and the only MUFU op is one lg2 per root.
+                                   2 on an ineligible graph: E_UNSUPPORTED  */
+    int32_t reserved[5];        /* must be zero                                */
 } spn_prepare_options;
 
 /* Statistics of a prepared plan (used by the benchmark's roofline). */
@@ -142,6 +150,8 @@ typedef struct spn_plan_stats {
                                    (one transpose + one layered launch each)  */
     int32_t layered_kernel;     /* layered path: 1 v1, 2 v2 (0 other paths)   */
     int32_t tc_passes;          /* layered path: f16 MMA passes (1 or 3)      */
+    int32_t value_space;        /* 1 log2 space, 2 linear fp32 (compiled path) */
+    int32_t reserved_;
 } spn_plan_stats;
 
 /* Fill *opt with defaults (all auto). */
@@ -279,7 +289,9 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
  *   assembles (entries <name>_j / <name>_m), lang = 0 the same IR printed as
  *   plain C++ defining `<name>_host(x, n, ld, out, R, argmax, tab, marg)`,
  *   which the CPU test-suite compiles to check the generator against the
- *   oracle.  Sizes first (NULL buffers): *src_len (bytes incl. NUL),
+ *   oracle.  Bits 8..9 of lang select the value space (0 auto, 1 log2,
+ *   2 linear; see spn_prepare_options.value_space).
+ *   Sizes first (NULL buffers): *src_len (bytes incl. NUL),
  *   *n_roots, *n_tables (floats), *n_tasks; then again with buffers.
  *   name[64] receives the kernel base name; roots[] the output columns the
  *   task writes; tables[] the discrete-leaf tables (log2) passed as `tab`.

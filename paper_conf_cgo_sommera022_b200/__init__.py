@@ -54,7 +54,8 @@ class _Options(ctypes.Structure):
                 ("samples_per_thread", ctypes.c_int32), ("layered_path", ctypes.c_int32),
                 ("max_task_nodes", ctypes.c_int64), ("tc_precision", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("compiled_path", ctypes.c_int32),
-                ("layered_kernel", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
+                ("layered_kernel", ctypes.c_int32), ("value_space", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 5)]
 
 
 class _Stats(ctypes.Structure):
@@ -68,7 +69,8 @@ class _Stats(ctypes.Structure):
         ("prepare_ms", ctypes.c_double), ("kernel_regs", ctypes.c_int32),
         ("ctas_per_sm", ctypes.c_int32), ("mufu_exec_per_sample", ctypes.c_int64),
         ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64),
-        ("layered_kernel", ctypes.c_int32), ("tc_passes", ctypes.c_int32)]
+        ("layered_kernel", ctypes.c_int32), ("tc_passes", ctypes.c_int32),
+        ("value_space", ctypes.c_int32), ("reserved_", ctypes.c_int32)]
 
 
 _lib = None
@@ -169,7 +171,7 @@ class Plan:
     def __init__(self, graph: Graph, device: int | None = None, block_threads: int = 0,
                  samples_per_thread: int = 0, max_task_nodes: int = 0,
                  layered_path: int = 0, tc_precision: int = 0, ctas_per_sm: int = 0,
-                 compiled_path: int = 0, layered_kernel: int = 0):
+                 compiled_path: int = 0, layered_kernel: int = 0, value_space: int = 0):
         lib = load_library()
         opt = _Options()
         lib.spn_default_options(ctypes.byref(opt))
@@ -185,6 +187,7 @@ class Plan:
         opt.ctas_per_sm = ctas_per_sm
         opt.compiled_path = compiled_path
         opt.layered_kernel = layered_kernel
+        opt.value_space = value_space
         h = ctypes.c_void_p()
         _check(lib.spn_prepare(graph.handle, ctypes.byref(opt), ctypes.byref(h)))
         self._h = h
@@ -332,10 +335,10 @@ def build_layered(graph: Graph):
 
 
 R2STEP_DTYPE = np.dtype([(n, "<i4") for n in ("type", "root", "n_out", "na", "nb", "kpad",
-                                              "n_groups", "s_per_group", "n_group", "slot_a",
-                                              "slot_b", "slot_out", "n_vars", "pad_")] +
+                                              "n_groups", "spg_a", "ncol_a", "spg_b", "ncol_b",
+                                              "slot_a", "slot_b", "slot_out", "n_vars", "pad_")] +
                         [(n, "<i8") for n in ("vars_off", "blk_off", "blk_floats", "w_off",
-                                              "w_group_bytes")])
+                                              "wbytes_a", "wbytes_b")])
 
 
 def build_layered2(graph: Graph):
@@ -366,13 +369,13 @@ def build_layered2(graph: Graph):
 
 
 def codegen(graph: Graph, task: int = 0, lang: str = "cpp", compile: bool = False,
-            arch: str = "100a"):
+            arch: str = "100a", space: int = 0):
     """Host-only: the compiled path's generated code for one task
     (``spn_codegen``): lang "ptx" (what the library assembles) or "cpp" (the
     same IR as host C++, for CPU checks).  Returns dict(source, name, roots,
     tables, n_tasks).  compile=True also assembles the PTX for sm_<arch>
     with nvJitLink (raises SPNError on failure)."""
-    lg = {"cpp": 0, "ptx": 1}[lang]
+    lg = {"cpp": 0, "ptx": 1}[lang] | (int(space) << 8)   # space: 0 auto, 1 log2, 2 linear
     lib = load_library()
     sl, nt = ctypes.c_int64(), ctypes.c_int64()
     nr, ntask = ctypes.c_int32(), ctypes.c_int32()

@@ -207,7 +207,7 @@ void free_plan(DevicePlan *p) {
                 const char *roles[4] = {"leaf(8 warps)", "epilogue(4)", "mma", "producer"};
                 const char *ph[4][8] = {
                     {"wait_in", "compute", "shift", "wait_out", "exp+write", "-", "-", "-"},
-                    {"wait_leaf", "up_phase1", "wait_tmem", "sums", "tile_io", "step_setup", "-", "-"},
+                    {"wait_leaf", "up_phase1", "wait_mma", "sums", "tile_io", "step_end", "ld_issue", "ld_wait"},
                     {"wait_A", "wait_w", "wait_tmem", "issue", "-", "-", "-", "-"},
                     {"wait_in_slot", "-", "wait_w_slot", "-", "-", "-", "-", "issue"}};
                 for (int r = 0; r < 4; ++r) {
@@ -511,8 +511,9 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         R2Params rp;
         memset(&rp, 0, sizeof(rp));
         bool fits = false;
-        // deepest rings that fit: leaf inputs 3..2, weight groups 4..2
-        static const int kRings[][2] = {{3, 4}, {3, 3}, {2, 4}, {2, 3}, {2, 2}};
+        // deepest rings that fit: leaf inputs 3..2 (3 lets both leaf groups
+        // prefetch), weight groups 4..2 (the MMA warp holds a pair at once)
+        static const int kRings[][2] = {{3, 4}, {3, 3}, {3, 2}, {2, 4}, {2, 2}};
         for (int a = 0; r2.ok && a < 5 && !fits; ++a)
             fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
                                r2.max_wgroup, P->prec, kRings[a][0], kRings[a][1]) <= smem_optin;
@@ -625,6 +626,7 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
                      std::chrono::steady_clock::time_point t0, spn_handle **out_plan) {
     JitOptions jo;
     jo.block = opt.block_threads ? opt.block_threads : 768;
+    jo.space = opt.value_space;
     if (jo.block % 32 || jo.block < 32 || jo.block > 1024)
         return set_err(SPN_E_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
     // launch bound: 768 resident threads per SM (<= 80 registers).  Default
@@ -754,6 +756,7 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     s.kernel_regs = max_regs;
     s.ctas_per_sm = min_occ;
     s.mufu_exec_per_sample = jp.mufu_exec_per_sample;
+    s.value_space = jp.linear ? 2 : 1;
     s.compile_ms = compile_ms;
     s.prepare_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
@@ -842,8 +845,12 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     spn_prepare_options opt;
     spn_default_options(&opt);
     if (opt_in) opt = *opt_in;
-    for (int i = 0; i < 6; ++i)
+    for (int i = 0; i < 5; ++i)
         if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
+    if (opt.value_space < 0 || opt.value_space > 2)
+        return set_err(SPN_E_ARG, "value_space must be 0 (auto), 1 (log2) or 2 (linear)");
+    if (opt.value_space == 2 && (opt.compiled_path == 1 || opt.layered_path == 2))
+        return set_err(SPN_E_ARG, "value_space 2 (linear) needs the compiled path");
     if (opt.layered_kernel < 0 || opt.layered_kernel > 2)
         return set_err(SPN_E_ARG, "layered_kernel must be 0 (auto), 1 (v1) or 2 (v2)");
     if (opt.compiled_path < 0 || opt.compiled_path > 2)
@@ -861,7 +868,7 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
 
     // ---- layered (RAT-SPN) tensor-core path ----
-    if (opt.layered_path != 1) {
+    if (opt.layered_path != 1 && opt.value_space != 2) {
         LayeredPlan lp;
         size_t lsmem = 0;
         int wbufs = 0;
@@ -897,10 +904,12 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     // ---- compiled path: one generated straight-line kernel per task ----
     // auto: used unless the caller pins interpreter parameters
     // (samples_per_thread / max_task_nodes) or a component is too large
-    if (opt.compiled_path == 2 ||
+    if (opt.compiled_path == 2 || opt.value_space == 2 ||
         (opt.compiled_path == 0 && opt.samples_per_thread == 0 && opt.max_task_nodes == 0)) {
         const int rc = prepare_compiled(g, opt, dev, sms, t0, out_plan);
-        if (rc == SPN_OK || opt.compiled_path == 2 || rc == SPN_E_ARG || rc == SPN_E_OOM) return rc;
+        if (rc == SPN_OK || opt.compiled_path == 2 || opt.value_space == 2 || rc == SPN_E_ARG ||
+            rc == SPN_E_OOM)
+            return rc;
         // SPN_E_UNSUPPORTED / SPN_E_CUDA from the compiler or loader: the
         // interpreter kernel (also sm_100a, not a CPU path) serves the graph
     }
@@ -1004,7 +1013,17 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     }
     P->grid_max = sms * bps;
     if (P->n_gslots > 0) {
-        const size_t bytes = (size_t)P->grid_max * (block / 32) * P->n_gslots * WT * 4;
+        // per-warp scratch for values crossing tasks: a multi-task plan of a
+        // very large SPN (C5 at <= 10k ops per task) keeps tens of thousands
+        // of cut values live per sample, so the persistent grid is capped to
+        // keep the scratch within 1/4 of free device memory (8 GiB at most);
+        // the kernel's grid-stride loop covers any n with fewer warps
+        size_t free_b = 0, total_b = 0;
+        cudaMemGetInfo(&free_b, &total_b);
+        const size_t budget = std::min<size_t>((size_t)8 << 30, free_b / 4);
+        const size_t per_cta = (size_t)(block / 32) * P->n_gslots * WT * 4;
+        P->grid_max = (int)std::max<size_t>(1, std::min<size_t>((size_t)P->grid_max, budget / per_cta));
+        const size_t bytes = (size_t)P->grid_max * per_cta;
         if ((e = cudaMalloc(&P->d_gslots, bytes)) != cudaSuccess) {
             free_plan(P);
             return set_err(SPN_E_OOM, "scratch slots");
@@ -1195,6 +1214,9 @@ int spn_codegen(const spn_handle *graph, int32_t task, int32_t lang, char *src, 
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
     if (const char *e = getenv("SPNB_JIT_BAR")) jo.bar_every = std::max(0, atoi(e));
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
+    // value space of the generated code: bits 8..9 of lang (0 auto, 1 log2, 2 linear)
+    jo.space = (lang >> 8) & 3;
+    lang &= 0xff;
     JitProgram jp;
     std::string msg;
     int rc = generate_jit(*graph->graph, jo, jp, msg);

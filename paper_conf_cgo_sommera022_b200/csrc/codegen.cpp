@@ -73,7 +73,8 @@ enum IrOp {
     I_LG2,     // d = log2(a)     (MUFU lg2.approx.ftz)
     I_SELNAN,  // d = isnan(a) ? b : c
     I_SELINF,  // d = isinf(a) ? b : c
-    I_DISC,    // d = a in [lo, lo+K) ? tab[floor(a) - lo] : -inf;  isnan(a): joint a, marginal 0
+    I_DISC,    // d = a in [lo, lo+K) ? tab[floor(a) - lo] : b;  isnan(a): joint a, marginal c
+               // (log2 space: b = -inf, c = 0; linear space: b = 0, c = 1)
     I_OUT,     // out[aux] = a * ln2
     I_ARGMAX,  // argmax over out[roots] (lowest index of the largest non-NaN; -1 if none)
     I_MOV,     // d = a (immediate)
@@ -179,6 +180,8 @@ struct TaskGen {
         i.op = I_DISC;
         i.d = ir.nreg++;
         i.a = Ir::R(F.x);
+        i.b = ir.imm(-INFINITY);
+        i.c = ir.imm(0.0);
         i.aux = L.tab;
         i.lo = L.lo;
         i.K = L.K;
@@ -323,8 +326,11 @@ std::string emit_cpp(const Ir &ir, const std::string &fn) {
             case I_SELNAN: snprintf(b, sizeof(b), "const float %s = (%s != %s) ? %s : %s;", d.c_str(), a.c_str(), a.c_str(), bb.c_str(), cc.c_str()); break;
             case I_SELINF: snprintf(b, sizeof(b), "const float %s = (fabsf(%s) == INFINITY) ? %s : %s;", d.c_str(), a.c_str(), bb.c_str(), cc.c_str()); break;
             case I_DISC:
-                snprintf(b, sizeof(b), "const float %s = spnb_disc(%s, %lld, %lld, tab + %lld, %d);",
-                         d.c_str(), a.c_str(), (long long)i.lo, (long long)i.K, (long long)i.aux, ir.marg ? 1 : 0);
+                snprintf(b, sizeof(b),
+                         "const float %s = spnb_disc(%s, %lld, %lld, tab + %lld, %d, spnb_f(0x%08xu), "
+                         "spnb_f(0x%08xu));",
+                         d.c_str(), a.c_str(), (long long)i.lo, (long long)i.K, (long long)i.aux,
+                         ir.marg ? 1 : 0, fbits(i.b.imm), fbits(i.c.imm));
                 break;
             case I_OUT: snprintf(b, sizeof(b), "o[%lld] = %s * spnb_f(0x3f317218u);", (long long)i.aux, a.c_str()); break;
             case I_ARGMAX: {
@@ -353,10 +359,11 @@ const char *kCppPrelude = R"PRE(// generated by libspnb codegen.cpp (compiled pa
 #include <string.h>
 static inline float spnb_f(unsigned u) { float f; memcpy(&f, &u, 4); return f; }
 static inline float spnb_maxn(float a, float b) { return (a != a || b != b) ? NAN : (a > b ? a : b); }
-static inline float spnb_disc(float x, long long lo, long long K, const float *t, int marg) {
+static inline float spnb_disc(float x, long long lo, long long K, const float *t, int marg,
+                              float outside, float missing) {
     const int ok = (x >= (float)lo) && (x < (float)(lo + K));
-    float v = ok ? t[(long long)floorf(x) - lo] : -INFINITY;
-    if (x != x) v = marg ? 0.f : x;
+    float v = ok ? t[(long long)floorf(x) - lo] : outside;
+    if (x != x) v = marg ? missing : x;
     return v;
 }
 )PRE";
@@ -421,6 +428,8 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
                 break;
             }
             case I_DISC: {
+                char mval[16];
+                snprintf(mval, sizeof(mval), "0f%08X", fbits(i.c.imm));
                 const int p0 = np, r0 = nr, q0 = nd;
                 np += 3;
                 nr += 1;
@@ -432,12 +441,12 @@ std::string emit_ptx_entry(const Ir &ir, const std::string &name, int block, int
                          "setp.ge.f32 %%p%d, %s, %s; setp.lt.and.f32 %%p%d, %s, %s, %%p%d; "
                          "cvt.rmi.s32.f32 %%r%d, %s; sub.s32 %%r%d, %%r%d, %lld; "
                          "mul.wide.s32 %%rd%d, %%r%d, 4; add.s64 %%rd%d, %%tab, %%rd%d; "
-                         "mov.f32 %s, 0fFF800000; @%%p%d ld.global.nc.f32 %s, [%%rd%d+%lld]; "
+                         "mov.f32 %s, 0f%08X; @%%p%d ld.global.nc.f32 %s, [%%rd%d+%lld]; "
                          "setp.nan.f32 %%p%d, %s, %s; selp.f32 %s, %s, %s, %%p%d;",
                          p0, a.c_str(), lo, p0 + 1, a.c_str(), hi, p0, r0, a.c_str(), r0, r0,
-                         (long long)i.lo, q0, r0, q0, q0, d.c_str(), p0 + 1, d.c_str(), q0,
-                         (long long)i.aux * 4, p0 + 2, a.c_str(), a.c_str(), d.c_str(),
-                         ir.marg ? "0f00000000" : a.c_str(), d.c_str(), p0 + 2);
+                         (long long)i.lo, q0, r0, q0, q0, d.c_str(), fbits(i.b.imm), p0 + 1,
+                         d.c_str(), q0, (long long)i.aux * 4, p0 + 2, a.c_str(), a.c_str(),
+                         d.c_str(), ir.marg ? mval : a.c_str(), d.c_str(), p0 + 2);
                 break;
             }
             case I_OUT: {
@@ -581,6 +590,64 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
     const int64_t n = c.n;
     out = JitProgram();
 
+    // ---- value space (the `probability` type is chosen by
+    // the compiler, e.g. from the graph depth): linear fp32 when every leaf
+    // is discrete and interval bounds on the non-zero values any node can
+    // take (marginalised leaves count as 1) stay inside [2^-100, 2^100] --
+    // then no value can underflow or overflow fp32's normal range, sums are
+    // plain FFMA chains and the only MUFU op is one lg2 per root
+    {
+        bool disc_only = true;
+        std::vector<double> vlo(n, 1.0), vhi(n, 1.0);
+        double gmin = 1.0, gmax = 1.0;
+        for (int64_t u = 0; u < n && disc_only; ++u) {  // children before parents
+            const int64_t o = c.orig[u];
+            if (c.kind[u] == SPN_GAUSSIAN) {
+                disc_only = false;
+            } else if (c.kind[u] == SPN_CATEGORICAL || c.kind[u] == SPN_HISTOGRAM) {
+                const double *p = g.params.data() + g.param_begin[o];
+                const int64_t np = g.n_params[o];
+                double lo = 1.0, hi = 1.0;  // 1: a marginalised (missing) leaf
+                for (int64_t i = c.kind[u] == SPN_CATEGORICAL ? 0 : 2; i < np;
+                     i += c.kind[u] == SPN_CATEGORICAL ? 1 : 3)
+                    if (p[i] > 0.0) {
+                        lo = std::min(lo, p[i]);
+                        hi = std::max(hi, p[i]);
+                    }
+                vlo[u] = lo;
+                vhi[u] = hi;
+            } else if (c.kind[u] == SPN_PRODUCT) {
+                double lo = 1.0, hi = 1.0;
+                for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e) {
+                    lo *= vlo[c.ch[e]];
+                    hi *= vhi[c.ch[e]];
+                }
+                vlo[u] = lo;
+                vhi[u] = hi;
+            } else {
+                double lo = INFINITY, hi = 0.0;
+                for (int64_t e = c.cb[u]; e < c.cb[u + 1]; ++e)
+                    if (c.w[e] > 0.0) {
+                        lo = std::min(lo, c.w[e] * vlo[c.ch[e]]);
+                        hi += c.w[e] * vhi[c.ch[e]];
+                    }
+                vlo[u] = std::isfinite(lo) ? lo : 1.0;
+                vhi[u] = hi > 0.0 ? hi : 1.0;
+            }
+            gmin = std::min(gmin, vlo[u]);
+            gmax = std::max(gmax, vhi[u]);
+        }
+        const bool in_range = disc_only && gmin >= std::ldexp(1.0, -100) && gmax <= std::ldexp(1.0, 100);
+        if (opt.space == 2 && !in_range) {
+            msg = disc_only ? "linear space: value range outside [2^-100, 2^100]"
+                            : "linear space needs discrete leaves only";
+            return SPN_E_UNSUPPORTED;
+        }
+        out.linear = opt.space == 2 || (opt.space == 0 && in_range);
+        out.lin_min = gmin;
+        out.lin_max = gmax;
+    }
+
     // ---- leaves: parameters in the log2 domain --------------------------
     std::vector<LeafInfo> leaf(n);
     std::vector<double> msum(g.F, 0.0);
@@ -614,17 +681,18 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
             L.lo = 0;
             L.K = np;
             L.tab = (int64_t)out.tables.size();
-            for (int64_t i = 0; i < np; ++i) out.tables.push_back((float)std::log2(p[i]));
+            for (int64_t i = 0; i < np; ++i)
+                out.tables.push_back(out.linear ? (float)p[i] : (float)std::log2(p[i]));
         } else {
             int64_t lo = INT64_MAX, hi = INT64_MIN;
             for (int64_t b = 0; b < np; b += 3) {
                 lo = std::min(lo, (int64_t)p[b]);
                 hi = std::max(hi, (int64_t)p[b + 1]);
             }
-            std::vector<float> tab((size_t)(hi - lo), -INFINITY);
+            std::vector<float> tab((size_t)(hi - lo), out.linear ? 0.f : -INFINITY);
             for (int64_t b = 0; b < np; b += 3)
                 for (int64_t v = (int64_t)p[b]; v < (int64_t)p[b + 1]; ++v)
-                    tab[v - lo] = (float)std::log2(p[b + 2]);
+                    tab[v - lo] = out.linear ? (float)p[b + 2] : (float)std::log2(p[b + 2]);
             L.lo = lo;
             L.K = hi - lo;
             L.tab = (int64_t)out.tables.size();
@@ -670,6 +738,12 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
         }
     }
     out.n_nodes = n;
+    if (out.linear) {  // one lg2 per root; an FMUL per product edge, an FFMA per sum edge
+        out.mufu_per_sample = out.mufu_exec_per_sample = (int64_t)g.roots.size();
+        out.fma_per_sample = 0;
+        for (int64_t u = 0; u < n; ++u)
+            if (!is_leaf(c.kind[u])) out.fma_per_sample += c.cb[u + 1] - c.cb[u];
+    }
 
     // ---- tasks: connected components packed up to task_cap_nodes --------
     std::vector<int64_t> uf(n);
@@ -755,13 +829,47 @@ int generate_jit(const GraphData &g, const JitOptions &opt, JitProgram &out, std
                 if (use_d[f]) F.d = ir.marg ? ir.emit(I_SELNAN, R(F.x), ir.imm(0.0), R(xm)) : xm;
             }
             ir.n_prologue = ir.ins.size();
-            for (int64_t u : tnodes[t]) {
-                if (c.kind[u] == SPN_PRODUCT) tg.product(u);
-                else if (c.kind[u] == SPN_SUM) tg.sum(u);
+            if (out.linear) {
+                // linear space: leaf = p (0 outside the support, 1 if missing
+                // in a marginal query); product = FMUL chain; sum = FFMA chain
+                // with the weights as immediates
+                for (int64_t u : tnodes[t]) {
+                    if (is_leaf(c.kind[u])) {
+                        const LeafInfo &L = leaf[u];
+                        Ins i;
+                        i.op = I_DISC;
+                        i.d = ir.nreg++;
+                        i.a = R(fr[L.f].x);
+                        i.b = ir.imm(0.0);
+                        i.c = ir.imm(1.0);
+                        i.aux = L.tab;
+                        i.lo = L.lo;
+                        i.K = L.K;
+                        ir.ins.push_back(i);
+                        val[u] = i.d;
+                    } else if (c.kind[u] == SPN_PRODUCT) {
+                        int32_t acc = val[c.ch[c.cb[u]]];
+                        for (int64_t e = c.cb[u] + 1; e < c.cb[u + 1]; ++e)
+                            acc = ir.emit(I_MUL, R(acc), R(val[c.ch[e]]));
+                        val[u] = acc;
+                    } else {
+                        int32_t acc = ir.emit(I_MUL, R(val[c.ch[c.cb[u]]]), ir.imm(c.w[c.cb[u]]));
+                        for (int64_t e = c.cb[u] + 1; e < c.cb[u + 1]; ++e)
+                            acc = ir.emit(I_FMA, R(val[c.ch[e]]), ir.imm(c.w[e]), R(acc));
+                        val[u] = acc;
+                    }
+                }
+            } else {
+                for (int64_t u : tnodes[t]) {
+                    if (c.kind[u] == SPN_PRODUCT) tg.product(u);
+                    else if (c.kind[u] == SPN_SUM) tg.sum(u);
+                }
             }
             for (auto &rr : troots[t]) {
                 const int64_t u = rr.second;
-                const int32_t v = is_leaf(c.kind[u]) ? tg.inline_leaf(u, 0.0) : val[u];
+                int32_t v;
+                if (out.linear) v = ir.emit(I_LG2, R(val[u]));
+                else v = is_leaf(c.kind[u]) ? tg.inline_leaf(u, 0.0) : val[u];
                 Ins o;
                 o.op = I_OUT;
                 o.a = R(v);

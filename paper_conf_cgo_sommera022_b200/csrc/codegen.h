@@ -34,6 +34,9 @@ struct JitOptions {
     int64_t max_live_auto = 64;     // auto selection: larger ir_max_live stays on the
                                     // interpreter (RAT-SPN cross products: hundreds of live
                                     // values, ptxas takes minutes and the kernel spills)
+    int space = 0;                  // value space (the deferred `probability`
+                                    // type): 0 auto, 1 log2, 2 linear fp32 (discrete
+                                    // leaves only, value range inside fp32's normal range)
 };
 
 struct JitTask {
@@ -52,6 +55,8 @@ struct JitProgram {
     std::vector<JitTask> tasks;
     std::vector<float> tables;   // discrete leaf tables (log2), read via `tab`
     bool fused_argmax = false;   // one task covers every root: argmax in-kernel
+    bool linear = false;         // values are probabilities (linear fp32), tables hold p
+    double lin_min = 0, lin_max = 0;  // linear: bounds of the non-zero values reachable
     // statistics (same definitions as PlanProgram)
     int64_t n_nodes = 0, n_leaves = 0, n_sums = 0, n_products = 0, n_sum_edges = 0;
     int64_t mufu_per_sample = 0, fma_per_sample = 0;

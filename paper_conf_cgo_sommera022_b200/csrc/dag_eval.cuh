@@ -575,7 +575,7 @@ __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
     }
 #define SPN_BODY_9(S)                                                            \
     {                                                                            \
-        const uint32_t a = cx >> CASE_BITS;                                      \
+        const uint32_t a = cz; /* global slot byte offset (32 bits) */           \
         const float b = __uint_as_float(cy);                                     \
         SPN_NEXT(pc + 16)                                                        \
         GIO<K>::ld(reinterpret_cast<const float *>(e.gs + a), r[SPN_SS(S)]);     \
@@ -589,7 +589,7 @@ __host__ __device__ constexpr bool op_valid(int op, int sp, int D) {
     }
 #define SPN_BODY_11(S)                                                           \
     {                                                                            \
-        const uint32_t a = cx >> CASE_BITS;                                      \
+        const uint32_t a = cz; /* global slot byte offset (32 bits) */           \
         SPN_NEXT(pc + 16)                                                        \
         GIO<K>::st(reinterpret_cast<float *>(e.gs + a), r[S - 1]);               \
     }

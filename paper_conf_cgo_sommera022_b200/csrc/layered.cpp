@@ -529,11 +529,16 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
     p.I = I;
     p.S = S;
     p.D = D;
+    // TMEM: two accumulators of R2_COLS_A + R2_COLS_B columns (tcgen05.mma
+    // costs ~170 cycles per dependent step almost independently of N, so the
+    // widest groups minimise the MMA count; the two chains interleave), then
+    // the D activation slots and the C root accumulators
     const int32_t fixed_cols = D * S + p.C;
-    int32_t gc = std::min<int32_t>(256, (512 - fixed_cols) / 2) / 16 * 16;
     const int32_t na_max = std::max(I, S);
-    if (gc < na_max) return fail("TMEM budget: " + std::to_string(fixed_cols) + " fixed columns");
-    p.gcols = gc;
+    if (R2_COLS_A + R2_COLS_B + fixed_cols > 512)
+        return fail("TMEM budget: " + std::to_string(fixed_cols) + " activation/root columns");
+    if (na_max > R2_COLS_B) return fail("region wider than an accumulator buffer");
+    p.gcols = R2_COLS_A + R2_COLS_B;
     p.ea_max = (na_max + 7) / 8 * 8;
     p.kpad_bot = (I + 15) / 16 * 16;
     p.kpad_up = S > 0 ? (S + 15) / 16 * 16 : 16;
@@ -578,12 +583,28 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
             r.slot_a = slot[lp.child_a[t]];
             r.slot_b = slot[lp.child_b[t]];
         }
-        int32_t spg = std::max(1, gc / na);
-        int32_t ng = (n_out + spg - 1) / spg;
-        spg = (n_out + ng - 1) / ng;  // balanced groups
-        r.n_groups = ng;
-        r.s_per_group = spg;
-        r.n_group = (spg * na + 15) / 16 * 16;
+        // sums per group: the most whose columns (x16) fit the buffer
+        auto cap = [&](int32_t cols) {
+            int32_t c = cols / na;
+            while (c > 1 && (c * na + 15) / 16 * 16 > cols) --c;
+            return std::max(1, c);
+        };
+        const int32_t cap_a = cap(R2_COLS_A), cap_b = cap(R2_COLS_B);
+        int32_t spg_a = cap_a, spg_b = cap_b;
+        if (n_out <= cap_a + cap_b) {  // one pair: split in proportion to the buffers
+            spg_a = std::min(cap_a, (n_out * cap_a + cap_a + cap_b - 1) / (cap_a + cap_b));
+            spg_b = n_out - spg_a;
+            if (spg_b > cap_b) {
+                spg_b = cap_b;
+                spg_a = n_out - cap_b;
+            }
+        }
+        const int32_t n_pairs = (n_out + spg_a + spg_b - 1) / (spg_a + spg_b);
+        r.n_groups = 2 * n_pairs;
+        r.spg_a = spg_a;
+        r.spg_b = spg_b;
+        r.ncol_a = std::max(16, (spg_a * na + 15) / 16 * 16);
+        r.ncol_b = std::max(16, (spg_b * na + 15) / 16 * 16);
         // per-sum scale exponents: w' = w 2^k with max_ij w' in [1, 2)
         const std::vector<double> &W = lp.raw[t];
         while (p.fparams.size() % 4) p.fparams.push_back(0.f);
@@ -597,14 +618,18 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
             p.fparams.push_back((float)k);
         }
         while (p.fparams.size() % 4) p.fparams.push_back(0.f);
-        r.w_group_bytes = (int64_t)r.n_group * r.kpad * 2;
+        r.wbytes_a = (int64_t)r.ncol_a * r.kpad * 2;
+        r.wbytes_b = (int64_t)r.ncol_b * r.kpad * 2;
         while (p.wimg.size() % 64) p.wimg.push_back(0);  // 128-byte aligned images
         r.w_off = (int64_t)p.wimg.size() * 2;
-        const size_t gel = (size_t)r.n_group * r.kpad;
-        for (int32_t gi = 0; gi < ng; ++gi) {
+        for (int32_t gi = 0; gi < r.n_groups; ++gi) {
+            const bool gb = gi & 1;
+            const int32_t ncol = gb ? r.ncol_b : r.ncol_a, spg = gb ? spg_b : spg_a;
+            const int32_t s_first = (gi / 2) * (spg_a + spg_b) + (gb ? spg_a : 0);
+            const size_t gel = (size_t)ncol * r.kpad;
             std::vector<uint16_t> hi(gel, 0), lo(gel, 0);
             for (int32_t sl = 0; sl < spg; ++sl) {
-                const int32_t s2 = gi * spg + sl;
+                const int32_t s2 = s_first + sl;
                 if (s2 >= n_out) break;
                 for (int32_t i = 0; i < na; ++i)
                     for (int32_t j = 0; j < nb; ++j) {
@@ -612,7 +637,7 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
                         const double w = W[(size_t)s2 * na * nb + (size_t)i * nb + j] * scale[s2];
                         const uint16_t h = f32_to_f16((float)w);
                         const uint16_t l = f32_to_f16((float)(w - (double)f16_to_f32(h)));
-                        const size_t idx = (size_t)(j / 8) * ((size_t)r.n_group / 8) * 64 +
+                        const size_t idx = (size_t)(j / 8) * ((size_t)ncol / 8) * 64 +
                                            (size_t)(row / 8) * 64 + (size_t)(row % 8) * 8 +
                                            (size_t)(j % 8);
                         hi[idx] = h;
@@ -622,7 +647,7 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
             p.wimg.insert(p.wimg.end(), hi.begin(), hi.end());
             p.wimg.insert(p.wimg.end(), lo.begin(), lo.end());
         }
-        p.max_wgroup = std::max<int32_t>(p.max_wgroup, (int32_t)r.w_group_bytes);
+        p.max_wgroup = std::max<int32_t>(p.max_wgroup, (int32_t)std::max(r.wbytes_a, r.wbytes_b));
         p.n_sum++;
         p.steps.push_back(r);
     }

@@ -79,16 +79,21 @@ struct R2Step {
     int32_t type;        // 0 LEAF, 1 BOT (children: two leaf regions), 2 UP (two sum regions)
     int32_t root;        // 1: the outputs are root (class) values, accumulated over repetitions
     int32_t n_out, na, nb, kpad;
-    int32_t n_groups, s_per_group, n_group;  // N groups: sums per group, columns (x16)
+    // N groups alternate between the two TMEM accumulators: even groups
+    // (buffer A, R2_COLS_A columns) hold spg_a sums, odd groups (buffer B)
+    // spg_b; the last pair may be partial (a group may be empty); n_groups
+    // is even.  ncol_*: MMA N (sums x na rounded up to 16)
+    int32_t n_groups, spg_a, ncol_a, spg_b, ncol_b;
     int32_t slot_a, slot_b, slot_out;        // TMEM activation slots (1-based; UP inputs, output)
     int32_t n_vars;      // LEAF: variables of the region
     int32_t pad_;
     int64_t vars_off;    // LEAF: int32 offset into vars
     int64_t blk_off;     // LEAF: float offset of the block (a,b)[v][I], C[I]; SUM: kscale[n_out]
     int64_t blk_floats;  // LEAF: block size in floats (multiple of 4)
-    int64_t w_off;       // SUM: byte offset of the group images (group-major, [hi, lo] per group)
-    int64_t w_group_bytes;  // bytes of one (group, part) image
+    int64_t w_off;       // SUM: byte offset of the images: per group pair [A hi, A lo, B hi, B lo]
+    int64_t wbytes_a, wbytes_b;  // bytes of one part image of an A / B group
 };
+constexpr int R2_COLS_A = 240, R2_COLS_B = 160;  // TMEM accumulator buffers (columns)
 
 struct Rat2Plan {
     bool ok = false;
@@ -97,7 +102,7 @@ struct Rat2Plan {
     int32_t max_vars = 0, max_blk = 0;          // largest leaf region / parameter block (floats)
     int32_t kpad_bot = 0, kpad_up = 0;          // K of the BOT / UP contractions (x16)
     int32_t max_wgroup = 0;                     // bytes of the largest (group, part) image
-    int32_t gcols = 0;                          // TMEM columns per accumulator buffer
+    int32_t gcols = 0;                          // TMEM columns of both accumulators (A + B)
     int32_t ea_max = 0;                         // max(I, S) rounded up to 8
     std::vector<R2Step> steps;
     std::vector<int32_t> vars;

@@ -878,7 +878,9 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
         const int64_t u = f.node;
         if (slot_of[u] < 0) return fail(msg, SPN_E_UNSUPPORTED, "internal: node %lld has no slot", u);
         const uint64_t off = (uint64_t)slot_of[u] * slot_bytes;
-        if (off > ARG_MAX || off >= SLOT_GLOBAL)
+        // shared slots: byte offset in the 23-bit record argument; global
+        // slots: in the record's z word / the edge ref (31 bits)
+        if ((!in_global[u] && off > ARG_MAX) || off >= SLOT_GLOBAL)
             return fail(msg, SPN_E_UNSUPPORTED, "too many scratch slots (%lld)", slot_of[u]);
         if (f.kind <= 1) {
             Rec &r = prog[f.idx];
@@ -886,7 +888,8 @@ int build_program(const GraphData &g, const CodegenConfig &cfg, PlanProgram &out
             uint32_t op;
             if (f.kind == 0) op = in_global[u] ? OP_LDG : OP_LDS;
             else op = in_global[u] ? OP_STG : OP_STS;
-            r = make_rec(op, sp, (uint32_t)off, r.y, r.z, r.w);
+            if (in_global[u]) r = make_rec(op, sp, 0u, r.y, (uint32_t)off, r.w);
+            else r = make_rec(op, sp, (uint32_t)off, r.y, r.z, r.w);
         } else {
             const uint32_t ref = (uint32_t)off | (in_global[u] ? SLOT_GLOBAL : 0u);
             if (f.kind == 2) out.edges[f.idx].a = ref;

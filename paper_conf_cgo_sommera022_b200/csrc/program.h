@@ -35,7 +35,8 @@
 //   LSE1..4  | bias          r[sp-n] = LSE_i(r[sp-n+i]) + bias   weighted sum: the
 //                            largest input is the shift m, so its ex2(0)=1 needs no
 //                            MUFU: n-1 ex2 + 1 lg2 per sum
-//   LDS/LDG s | bias         r[sp]   = slot_s + bias   (shared / global scratch)
+//   LDS/LDG s | bias         r[sp]   = slot_s + bias   (shared / global scratch;
+//                            LDG/STG carry the slot's byte offset in z, 32 bits)
 //   STS/STG s                slot_s  = r[sp-1]  (the next record's sp pops)
 //   GLSE     | off_lo, off_hi, n   r[sp] = LSE over edge terms slot(a)[+slot(b)]+lw
 //   OUT    r                 out[., r] = ln2 * r[sp-1]

@@ -45,6 +45,8 @@ constexpr int RT = 128;           // samples per tile = UMMA M = TMEM lanes
 constexpr int NTHREADS = 16 * 32;
 constexpr int W_EPI0 = 8, W_PROD = 12, W_MMA = 13, W_WPROD = 14;
 constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
+// TMEM accumulators: A = columns [0, R2_COLS_A), B = [R2_COLS_A, +R2_COLS_B);
+// the groups of a step alternate A, B (layered.h R2Step)
 
 __device__ __forceinline__ float ex2(float x) {
     float y;
@@ -142,6 +144,18 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float *v) {
 #pragma unroll
     for (int k = 0; k < 8; ++k) v[k] = __uint_as_float(r[k]);
 }
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float *v) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
+        "%12, %13, %14, %15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+          "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(r[k]);
+}
 __device__ __forceinline__ void tmem_ld4(uint32_t taddr, float *v) {
     uint32_t r[4];
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
@@ -213,11 +227,11 @@ enum {
     B_B_EMPTY = 14,   // [2]
     B_U_FULL = 16,
     B_U_EMPTY = 17,
-    B_W_FULL = 18,    // [4]
-    B_W_EMPTY = 22,   // [4]
-    B_T_FULL = 26,    // [2]
-    B_T_EMPTY = 28,   // [2]
-    B_COUNT = 30
+    B_W_FULL = 18,    // [8]
+    B_W_EMPTY = 26,   // [8]
+    B_T_FULL = 34,    // [2]
+    B_T_EMPTY = 36,   // [2]
+    B_COUNT = 38
 };
 
 struct Smem {
@@ -423,30 +437,54 @@ __device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int3
     pf.mark(7);
 }
 
+// group gi of a sum step: first sum, number of sums (0: empty), MMA columns,
+// image byte offset relative to w_off and bytes of one part image
+struct GroupInfo {
+    int s0, ns, ncol;
+    int64_t off, bytes;
+};
+__device__ __forceinline__ GroupInfo group_info(const R2Step &st, int gi) {
+    const bool b = gi & 1;
+    const int pair = gi >> 1;
+    GroupInfo g;
+    g.s0 = pair * (st.spg_a + st.spg_b) + (b ? st.spg_a : 0);
+    g.ns = max(0, min(b ? st.spg_b : st.spg_a, st.n_out - g.s0));
+    g.ncol = b ? st.ncol_b : st.ncol_a;
+    g.bytes = b ? st.wbytes_b : st.wbytes_a;
+    g.off = (int64_t)pair * 2 * (st.wbytes_a + st.wbytes_b) + (b ? 2 * st.wbytes_a : 0);
+    return g;
+}
+
 __device__ void weight_producer_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps,
                                      int n_sum, int lane) {
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    uint32_t wi = 0;
+    uint32_t w_idx = 0, w_ph = 0;
+    const uint32_t n_w = (uint32_t)p.n_w;
     const int parts = p.prec == 3 ? 2 : 1;
     Prof pf(sm.prof(3), p.prof != nullptr);  // 2 wait weight slot, 7 issue
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         for (int si = 0; si < n_sum; ++si) {
-            const R2Step &st = p.steps[sum_steps[si]];
-            const uint32_t gb = (uint32_t)st.w_group_bytes;
-            for (int gi = 0; gi < st.n_groups; ++gi, ++wi) {
-                const int s = (int)(wi % (uint32_t)p.n_w);
+            const R2Step &st = p.steps[__ldg(sum_steps + si)];
+            for (int gi = 0; gi < st.n_groups; ++gi) {
+                const GroupInfo gr = group_info(st, gi);
+                if (gr.ns == 0) continue;  // empty group: no weights (the MMA skips it too)
                 pf.mark(7);
-                bar_wait(sm.bar(B_W_EMPTY + s), ((wi / (uint32_t)p.n_w) & 1u) ^ 1u);
+                bar_wait(sm.bar(B_W_EMPTY) + 8u * w_idx, w_ph ^ 1u);
                 pf.mark(2);
-                const uint32_t full = sm.bar(B_W_FULL + s);
+                const uint32_t full = sm.bar(B_W_FULL) + 8u * w_idx;
                 if (lane == 0) {
+                    const uint32_t gb = (uint32_t)gr.bytes;
                     bar_expect_tx(full, gb * parts);
-                    const uint8_t *src = p.wimg + st.w_off + (size_t)2 * gb * gi;
+                    const uint8_t *src = p.wimg + st.w_off + gr.off;
                     for (int pt = 0; pt < parts; ++pt)
-                        bulk_g2s(smem_u32(sm.wbuf(s)) + pt * (uint32_t)p.max_wgroup,
+                        bulk_g2s(smem_u32(sm.wbuf((int)w_idx)) + pt * (uint32_t)p.max_wgroup,
                                  src + (size_t)pt * gb, gb, full);
                 }
                 __syncwarp();
+                if (++w_idx == n_w) {
+                    w_idx = 0;
+                    w_ph ^= 1u;
+                }
             }
         }
     }
@@ -454,55 +492,97 @@ __device__ void weight_producer_role(const R2Params &p, const Smem &sm, const in
 }
 
 // ============================================================== MMA issuer
+// Per pair of groups (A, B) the K-steps of the two accumulators are
+// interleaved (consecutive MMAs into one accumulator serialise on its
+// latency, ~170 cycles per step on B200 whatever N; two chains overlap).
+// Ring positions advance incrementally (no runtime division); descriptors
+// are built once per group and advanced along K by adding byte offset >> 4
+// to the start-address field (shared addresses < 256 KB never carry).
+__device__ __forceinline__ uint64_t desc_hi(uint32_t lbo, uint32_t sbo) {
+    return ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
+           ((uint64_t)1 << 46);
+}
 __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps, int n_sum,
                          uint32_t tmem, int lane) {
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    uint32_t kb = 0, ku = 0, wi = 0, ti = 0;
+    uint32_t kb = 0, ku = 0, tp = 0;  // BOT / UP operand counters, accumulator-pair counter
+    uint32_t w_idx = 0, w_ph = 0;     // next weight-ring slot and its phase
+    const uint32_t n_w = (uint32_t)p.n_w;
     const uint32_t lbo_a = RT * 16;
-    Prof pf(sm.prof(2), p.prof != nullptr);  // 0 wait A operand, 1 wait weights, 2 wait TMEM buffer, 3 issue
+    const uint64_t a_hi_bits = desc_hi(lbo_a, 128);
+    const uint32_t wbase = smem_u32(sm.wbuf(0)), wstride = (uint32_t)p.w_bytes;
+    const uint32_t bar_wfull = sm.bar(B_W_FULL), bar_wempty = sm.bar(B_W_EMPTY);
+    const uint32_t bar_tfull = sm.bar(B_T_FULL), bar_tempty = sm.bar(B_T_EMPTY);
+    const bool split = p.prec == 3;
+    const uint32_t wlo_d = (uint32_t)p.max_wgroup >> 4;
+    Prof pf(sm.prof(2), p.prof != nullptr);  // 0 wait A operand, 1 wait weights, 2 wait TMEM, 3 issue
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         for (int si = 0; si < n_sum; ++si) {
-            const R2Step &st = p.steps[sum_steps[si]];
+            const R2Step &st = p.steps[__ldg(sum_steps + si)];
             const bool bot = st.type == 1;
-            uint32_t a_hi;
+            const int G = st.n_groups, ksteps = st.kpad / 16;
+            uint32_t a_addr;
             if (bot) {
                 const int ab = (int)(kb & 1u);
                 bar_wait(sm.bar(B_B_FULL + ab), (kb >> 1) & 1u);
-                a_hi = smem_u32(sm.bimg(ab));
+                a_addr = smem_u32(sm.bimg(ab));
             } else {
                 bar_wait(sm.bar(B_U_FULL), ku & 1u);
-                a_hi = smem_u32(sm.uimg());
+                a_addr = smem_u32(sm.uimg());
             }
             pf.mark(0);
-            const uint32_t a_lo = a_hi + (uint32_t)(bot ? p.bimg_bytes : p.uimg_bytes) / 2;
-            const uint32_t lbo_b = (uint32_t)st.n_group * 16;
-            const uint32_t idesc = (1u << 4) | ((uint32_t)(st.n_group >> 3) << 17) |
-                                   ((uint32_t)(RT >> 4) << 24);
-            for (int gi = 0; gi < st.n_groups; ++gi, ++wi, ++ti) {
-                const int ws = (int)(wi % (uint32_t)p.n_w);
-                const int tb = (int)(ti & 1u);
+            const uint64_t a_desc = a_hi_bits | (uint64_t)((a_addr >> 4) & 0x3FFFu);
+            const uint32_t a_lo_d = ((uint32_t)(bot ? p.bimg_bytes : p.uimg_bytes) / 2) >> 4;
+            const uint32_t ka_d = (2 * lbo_a) >> 4;
+            for (int gp = 0; gp < G; gp += 2, ++tp) {
+                GroupInfo gr[2] = {group_info(st, gp), group_info(st, gp + 1)};
+                uint32_t wsl[2] = {0, 0};
                 pf.mark(3);
-                bar_wait(sm.bar(B_W_FULL + ws), (wi / (uint32_t)p.n_w) & 1u);
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    if (gr[b].ns > 0) {
+                        wsl[b] = w_idx;
+                        bar_wait(bar_wfull + 8u * w_idx, w_ph);
+                        if (++w_idx == n_w) {
+                            w_idx = 0;
+                            w_ph ^= 1u;
+                        }
+                    }
+                }
                 pf.mark(1);
-                bar_wait(sm.bar(B_T_EMPTY + tb), ((ti >> 1) & 1u) ^ 1u);
+                bar_wait(bar_tempty, (tp & 1u) ^ 1u);
+                bar_wait(bar_tempty + 8u, (tp & 1u) ^ 1u);
                 pf.mark(2);
                 tc_fence_after();
                 if (lane == 0) {
-                    const uint32_t w_hi = smem_u32(sm.wbuf(ws)), w_lo = w_hi + (uint32_t)p.max_wgroup;
-                    const uint32_t d = tmem + (uint32_t)(tb * p.gcols);
-                    for (int kk = 0; kk < st.kpad / 16; ++kk) {
-                        const uint32_t ka = kk * 2 * lbo_a, kw = kk * 2 * lbo_b;
-                        umma_f16(d, umma_desc(a_hi + ka, lbo_a, 128), umma_desc(w_hi + kw, lbo_b, 128),
-                                 idesc, kk > 0);
-                        if (p.prec == 3) {
-                            umma_f16(d, umma_desc(a_lo + ka, lbo_a, 128),
-                                     umma_desc(w_hi + kw, lbo_b, 128), idesc, 1);
-                            umma_f16(d, umma_desc(a_hi + ka, lbo_a, 128),
-                                     umma_desc(w_lo + kw, lbo_b, 128), idesc, 1);
+                    uint64_t w_desc[2];
+                    uint32_t idesc[2], kw_d[2];
+#pragma unroll
+                    for (int b = 0; b < 2; ++b) {
+                        const uint32_t lbo_b = (uint32_t)gr[b].ncol * 16;
+                        w_desc[b] = desc_hi(lbo_b, 128) | (uint64_t)(((wbase + wsl[b] * wstride) >> 4) & 0x3FFFu);
+                        kw_d[b] = (2 * lbo_b) >> 4;
+                        idesc[b] = (1u << 4) | ((uint32_t)(gr[b].ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
+                    }
+                    for (int kk = 0; kk < ksteps; ++kk) {
+#pragma unroll
+                        for (int b = 0; b < 2; ++b) {
+                            if (gr[b].ns > 0) {
+                                const uint32_t d = tmem + (b ? (uint32_t)R2_COLS_A : 0u);
+                                const uint64_t ad = a_desc + kk * ka_d, wd = w_desc[b] + kk * kw_d[b];
+                                umma_f16(d, ad, wd, idesc[b], kk > 0);
+                                if (split) {
+                                    umma_f16(d, ad + a_lo_d, wd, idesc[b], 1);
+                                    umma_f16(d, ad, wd + wlo_d, idesc[b], 1);
+                                }
+                            }
                         }
                     }
-                    umma_commit(sm.bar(B_T_FULL + tb));
-                    umma_commit(sm.bar(B_W_EMPTY + ws));
+                    umma_commit(bar_tfull);
+                    umma_commit(bar_tfull + 8u);
+#pragma unroll
+                    for (int b = 0; b < 2; ++b)
+                        if (gr[b].ns > 0) umma_commit(bar_wempty + 8u * wsl[b]);
                 }
                 __syncwarp();
             }
@@ -516,107 +596,95 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
 }
 
 // ============================================================== EPILOGUE
-// Thread = sample m = TMEM lane.  TMEM columns: [0, 2 gcols) accumulators,
+// Thread = sample m = TMEM lane.  TMEM columns: [0, NACC GC) accumulators,
 // then D activation slots of S columns, then C root accumulators.  Widths
 // are template parameters (I: leaf regions, S: sum regions), so a sum's
-// stage-2 contraction is straight-line code: its columns are read in units
-// of U <= 24 columns, double-buffered (the next unit's tcgen05.ld is in
-// flight while this unit's FFMA2s run; tcgen05.wait::ld waits for both).
+// stage-2 contraction is straight-line code.
 
-// descriptor fields the epilogue needs, prefetched one step ahead
-struct EStep {
-    int type, root, n_out, n_groups, spg, slot_a, slot_b, slot_out;
-    int64_t ks_off;
-};
-__device__ __forceinline__ EStep load_estep(const R2Step *steps, const int32_t *idx, int si) {
-    const R2Step &st = steps[__ldg(idx + si)];
-    return EStep{st.type, st.root, st.n_out, st.n_groups, st.s_per_group,
-                 st.slot_a, st.slot_b, st.slot_out, st.blk_off};
-}
-
-template <int U>
-__device__ __forceinline__ void ld_unit(uint32_t taddr, float (&t)[U]) {
-#pragma unroll
-    for (int c = 0; c + 8 <= U; c += 8) tmem_ld8(taddr + c, t + c);
-    if constexpr (U % 8) tmem_ld4(taddr + (U / 8) * 8, t + (U / 8) * 8);
-}
 template <int W>
 __device__ __forceinline__ void ld_unit_any(uint32_t taddr, float (&t)[W]) {
 #pragma unroll
     for (int c = 0; c + 8 <= W; c += 8) tmem_ld8(taddr + c, t + c);
     if constexpr (W % 8) tmem_ld4(taddr + (W / 8) * 8, t + (W / 8) * 8);
 }
-template <int U>
-__device__ __forceinline__ float dot_unit(const float *ea, const float (&t)[U]) {
+// One sum step's groups: out_s = shift + lg2(sum_i ea_i T[s, i]) - k_s.
+// Group gi lives in accumulator gi & 1; its sums are read one at a time,
+// double-buffered (the next sum's tcgen05.ld is in flight while this sum's
+// FFMA2s run; tcgen05.wait::ld then covers it).
+// partial dot product of U columns against ea[off .. off + U)
+template <int U, int NA>
+__device__ __forceinline__ float dot_part(const float (&ea)[NA], int off, const float (&t)[U]) {
     float2 p0 = make_float2(0.f, 0.f), p1 = make_float2(0.f, 0.f);
 #pragma unroll
     for (int i = 0; i + 4 <= U; i += 4) {
-        p0 = __ffma2_rn(make_float2(ea[i], ea[i + 1]), make_float2(t[i], t[i + 1]), p0);
-        p1 = __ffma2_rn(make_float2(ea[i + 2], ea[i + 3]), make_float2(t[i + 2], t[i + 3]), p1);
+        p0 = __ffma2_rn(make_float2(ea[off + i], ea[off + i + 1]), make_float2(t[i], t[i + 1]), p0);
+        p1 = __ffma2_rn(make_float2(ea[off + i + 2], ea[off + i + 3]), make_float2(t[i + 2], t[i + 3]),
+                        p1);
     }
     return (p0.x + p0.y) + (p1.x + p1.y);
 }
-
-// One sum step's groups: out_s = shift + lg2(sum_i ea_i T[s, i]) - k_s.
 template <int NA, bool ROOT>
-__device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const EStep &es,
+__device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const R2Step &st,
                                            const float (&ear)[NA], float shift, uint32_t lane_base,
-                                           uint32_t out_col, uint32_t col_root, uint32_t &ti,
+                                           uint32_t out_col, uint32_t col_root, uint32_t &tp,
                                            Prof &pf) {
-    constexpr int U = NA > 24 ? NA / 2 : NA;  // columns per load unit
-    constexpr int UPS = NA / U;               // units per sum (1 or 2)
-    static_assert(U % 4 == 0 && U <= 24 && UPS * U == NA, "unit width");
-    const float *ks = p.fparams + es.ks_off;
-    for (int gi = 0; gi < es.n_groups; ++gi, ++ti) {
-        const int tb = (int)(ti & 1u);
-        const int s0 = gi * es.spg;
-        const int s1 = min(es.n_out, s0 + es.spg);
+    static_assert(NA % 4 == 0, "region width");
+    const float *ks = p.fparams + st.blk_off;
+    auto fin = [&](int s, float a) {
+        const float val = shift + lg2(a) - __ldg(ks + s);
+        if constexpr (ROOT) {
+            const uint32_t c = col_root + (uint32_t)__ldg(p.root_map + s);
+            float r;
+            tmem_ld1(lane_base + c, r);
+            tmem_wait_ld();
+            tmem_st1(lane_base + c, lse2(r, val));
+        } else {
+            tmem_st1(lane_base + out_col + s, val);
+        }
+    };
+    for (int gi = 0; gi < st.n_groups; ++gi) {
+        const int b = gi & 1;
+        const GroupInfo gr = group_info(st, gi);
         pf.mark(3);
-        bar_wait(sm.bar(B_T_FULL + tb), (ti >> 1) & 1u);
+        bar_wait(sm.bar(B_T_FULL + b), (tp & 1u));
         pf.mark(2);
         tc_fence_after();
-        const uint32_t acc0 = lane_base + (uint32_t)(tb * p.gcols);
+        const uint32_t acc = lane_base + (b ? (uint32_t)R2_COLS_A : 0u);
+        const int ns = gr.ns;
+        // load units of U <= 24 columns (half a sum when NA > 24), two buffers
+        constexpr int U = NA > 24 ? NA / 2 : NA;
         float b0[U], b1[U];
-        auto fin = [&](int s, float a) {
-            const float val = shift + lg2(a) - __ldg(ks + s);
-            if constexpr (ROOT) {
-                const uint32_t c = col_root + (uint32_t)__ldg(p.root_map + s);
-                float r;
-                tmem_ld1(lane_base + c, r);
+        if (ns > 0) {
+            ld_unit_any<U>(acc, b0);
+            tmem_wait_ld();
+        }
+        if constexpr (NA > 24) {
+            for (int sl = 0; sl < ns; ++sl) {
+                const uint32_t row = acc + (uint32_t)(sl * NA);
+                ld_unit_any<U>(row + U, b1);              // second half of this sum
+                float a = dot_part<U>(ear, 0, b0);
                 tmem_wait_ld();
-                tmem_st1(lane_base + c, lse2(r, val));
-            } else {
-                tmem_st1(lane_base + out_col + s, val);
-            }
-        };
-        ld_unit<U>(acc0, b0);
-        tmem_wait_ld();
-        if constexpr (UPS == 2) {
-            for (int s = s0; s < s1; ++s) {
-                const uint32_t row = acc0 + (uint32_t)((s - s0) * NA);
-                ld_unit<U>(row + U, b1);                  // second half of s
-                float a = dot_unit<U>(ear, b0);
-                tmem_wait_ld();
-                if (s + 1 < s1) ld_unit<U>(row + NA, b0);  // first half of s + 1
-                a += dot_unit<U>(ear + U, b1);
-                fin(s, a);
-                if (s + 1 < s1) tmem_wait_ld();
+                if (sl + 1 < ns) ld_unit_any<U>(row + NA, b0);  // first half of the next
+                a += dot_part<U>(ear, U, b1);
+                fin(gr.s0 + sl, a);
+                if (sl + 1 < ns) tmem_wait_ld();
             }
         } else {
-            for (int s = s0; s < s1; s += 2) {
-                const uint32_t row = acc0 + (uint32_t)((s - s0) * NA);
-                if (s + 1 < s1) ld_unit<U>(row + NA, b1);
-                fin(s, dot_unit<U>(ear, b0));
-                if (s + 1 < s1) {
+            for (int sl = 0; sl < ns; sl += 2) {
+                const uint32_t row = acc + (uint32_t)(sl * NA);
+                if (sl + 1 < ns) ld_unit_any<U>(row + NA, b1);
+                fin(gr.s0 + sl, dot_part<U>(ear, 0, b0));
+                if (sl + 1 < ns) {
                     tmem_wait_ld();
-                    if (s + 2 < s1) ld_unit<U>(row + 2 * NA, b0);
-                    fin(s + 1, dot_unit<U>(ear, b1));
-                    if (s + 2 < s1) tmem_wait_ld();
+                    if (sl + 2 < ns) ld_unit_any<U>(row + 2 * NA, b0);
+                    fin(gr.s0 + sl + 1, dot_part<U>(ear, 0, b1));
+                    if (sl + 2 < ns) tmem_wait_ld();
                 }
             }
         }
         tc_fence_before();
-        bar_arrive(sm.bar(B_T_EMPTY + tb));
+        bar_arrive(sm.bar(B_T_EMPTY + b));
+        if (b) ++tp;
     }
 }
 
@@ -626,20 +694,18 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
     const int qd = warp & 3;
     const int m = qd * 32 + lane;
     const uint32_t lane_base = tmem + ((uint32_t)(qd * 32) << 16);
-    const uint32_t col_slots = 2u * (uint32_t)p.gcols;
+    const uint32_t col_slots = (uint32_t)(R2_COLS_A + R2_COLS_B);
     const uint32_t col_root = col_slots + (uint32_t)(p.D * S);
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    uint32_t kb = 0, ku = 0, ti = 0;
+    uint32_t kb = 0, ku = 0, tp = 0;
     const int part_u = p.uimg_bytes / 2;
     constexpr int SU = S > 0 ? S : 4;
     Prof pf(sm.prof(1), p.prof != nullptr);  // 0 wait leaf outputs, 1 UP phase 1, 2 wait TMEM full, 3 sums, 4 tile I/O, 5 step setup
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         for (int c = 0; c < p.C; ++c) tmem_st1(lane_base + col_root + c, -CUDART_INF_F);
         tmem_wait_st();
-        EStep nx = load_estep(p.steps, sum_steps, 0);
         for (int si = 0; si < n_sum; ++si) {
-            const EStep es = nx;
-            if (si + 1 < n_sum) nx = load_estep(p.steps, sum_steps, si + 1);
+            const R2Step &es = p.steps[__ldg(sum_steps + si)];
             pf.mark(5);
             const uint32_t out_col = col_slots + (uint32_t)((es.slot_out - 1) * S);
             if (es.type == 1) {
@@ -656,8 +722,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 const float shift = sm.ha(ab)[m] + sm.hb(ab)[m];
                 bar_arrive(sm.bar(B_A_EMPTY + ab));
                 ++kb;
-                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
-                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
+                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
             } else {
                 // UP: children in activation slots; B side -> f16 image, A side -> registers
                 float vb[SU], ear[SU];
@@ -694,8 +760,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 for (int i = 0; i < SU; ++i) ear[i] = ex2(ear[i] - hac);
                 const float shift = ha + hb - EB_SHIFT;
                 pf.mark(1);
-                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
-                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, ti, pf);
+                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
+                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
             }
             tmem_wait_st();
         }
@@ -725,7 +791,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     rat2_kernel(const R2Params p, const int32_t *__restrict__ leaf_steps, int n_leaf,
                 const int32_t *__restrict__ sum_steps, int n_sum) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t *base = reinterpret_cast<uint8_t *>(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    // realign with pointer arithmetic on the __shared__ array (a round trip
+    // through uintptr_t would make every access a generic LD/ST)
+    uint8_t *base = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const Smem sm(base, p);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(base + p.off_bar + 8 * B_COUNT);
@@ -738,6 +806,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         for (int i = 0; i < 4; ++i) {
             bar_init(sm.bar(B_IN_FULL + i), 1);
             bar_init(sm.bar(B_IN_EMPTY + i), 4);
+        }
+        for (int i = 0; i < 8; ++i) {
             bar_init(sm.bar(B_W_FULL + i), 1);
             bar_init(sm.bar(B_W_EMPTY + i), 1);
         }
@@ -746,6 +816,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             bar_init(sm.bar(B_A_EMPTY + i), 128);
             bar_init(sm.bar(B_B_FULL + i), 128);
             bar_init(sm.bar(B_B_EMPTY + i), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
             bar_init(sm.bar(B_T_FULL + i), 1);
             bar_init(sm.bar(B_T_EMPTY + i), 128);
         }

@@ -25,23 +25,31 @@ def _f16_split(v, prec):
 
 
 def _decode_weights(plan, st, prec):
+    """W[s, i, j] from the group images: groups alternate between the A and
+    B accumulator sizes (spg_a / spg_b sums, ncol_a / ncol_b columns), each
+    stored as [hi, lo]."""
     na, nb, S = int(st["na"]), int(st["nb"]), int(st["n_out"])
-    ng, kpad, spg = int(st["n_group"]), int(st["kpad"]), int(st["s_per_group"])
-    gel = ng * kpad
-    base = int(st["w_off"]) // 2
+    kpad = int(st["kpad"])
     wimg = plan["wimg"]
     W = np.zeros((S, na, nb))
+    off = int(st["w_off"]) // 2
     for g in range(int(st["n_groups"])):
-        hi = wimg[base + 2 * g * gel: base + 2 * g * gel + gel].astype(np.float64)
-        lo = wimg[base + 2 * g * gel + gel: base + 2 * (g + 1) * gel].astype(np.float64)
+        b = g & 1
+        ncol = int(st["ncol_b"] if b else st["ncol_a"])
+        spg = int(st["spg_b"] if b else st["spg_a"])
+        s_first = (g // 2) * int(st["spg_a"] + st["spg_b"]) + (int(st["spg_a"]) if b else 0)
+        gel = ncol * kpad
+        hi = wimg[off:off + gel].astype(np.float64)
+        lo = wimg[off + gel:off + 2 * gel].astype(np.float64)
+        off += 2 * gel
         wg = hi + (lo if prec == 3 else 0.0)
         for sl in range(spg):
-            s = g * spg + sl
+            s = s_first + sl
             if s >= S:
                 break
             for i in range(na):
                 row = sl * na + i
-                idx = [_img_index(row, j, ng) for j in range(nb)]
+                idx = [_img_index(row, j, ncol) for j in range(nb)]
                 W[s, i, :] = wg[idx]
     return W
 

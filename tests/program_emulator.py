@@ -138,12 +138,12 @@ def emulate(prog: dict, x: np.ndarray, n_roots: int, marginal: bool, K: int,
                     stack[sp - n] = _lse([stack[sp - n + i] for i in range(n)]) + bias
             elif op == "LDS":
                 stack[sp] = sslots[arg // slot_bytes] + _f32(r["y"])
-            elif op == "LDG":
-                stack[sp] = gslots[arg // slot_bytes] + _f32(r["y"])
+            elif op == "LDG":  # global slot offsets ride in z (32 bits)
+                stack[sp] = gslots[int(r["z"]) // slot_bytes] + _f32(r["y"])
             elif op == "STS":
                 sslots[arg // slot_bytes] = stack[sp - 1].copy()
             elif op == "STG":
-                gslots[arg // slot_bytes] = stack[sp - 1].copy()
+                gslots[int(r["z"]) // slot_bytes] = stack[sp - 1].copy()
             elif op == "GLSE":
                 off = int(r["y"]) | (int(r["z"]) << 32)
                 n = int(r["w"])

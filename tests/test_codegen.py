@@ -38,16 +38,16 @@ _tmp = tempfile.mkdtemp(prefix="spnb_cg_")
 _count = itertools.count()   # unique .so names: dlopen caches by path
 
 
-def host_eval(g, x, marginal):
+def host_eval(g, x, marginal, space=0):
     """Run every generated task's C++ form over x; returns (out, argmax or None)."""
     G = spnb.Graph(g)
-    first = spnb.codegen(G, 0)
+    first = spnb.codegen(G, 0, space=space)
     R = g.n_roots
     out = np.full((len(x), R), np.nan, np.float32)
     am = np.zeros(len(x), np.int32)
     xx = np.ascontiguousarray(x, np.float32)
     for t in range(first["n_tasks"]):
-        cg = spnb.codegen(G, t)
+        cg = spnb.codegen(G, t, space=space)
         base = os.path.join(_tmp, f"t{os.getpid()}_{next(_count)}")
         with open(base + ".cpp", "w") as f:
             f.write(cg["source"])
@@ -72,8 +72,8 @@ def _cmp(got, ref, tol=TOL):
     assert ok.all(), f"{(~ok).sum()} mismatches: got {got[~ok][:3]} ref {ref[~ok][:3]}"
 
 
-def _check(g, x, marginal=False):
-    out, am, nt = host_eval(g, x, marginal)
+def _check(g, x, marginal=False, space=0):
+    out, am, nt = host_eval(g, x, marginal, space)
     ref, am_ref = oracle_eval(g, x, marginal=marginal)
     _cmp(out, ref)
     if am is not None and g.n_roots > 1:
@@ -161,9 +161,42 @@ def test_tiny_gaussian():
 
 
 def test_ptx_assembles_for_sm100a():
-    for g in (toy_spn(), speaker_spn(2001)):
+    for g, space in ((toy_spn(), 1), (toy_spn(), 2), (speaker_spn(2001), 0)):
         G = spnb.Graph(g)
-        cg = spnb.codegen(G, 0, lang="ptx", compile=True)
+        cg = spnb.codegen(G, 0, lang="ptx", compile=True, space=space)
         src = cg["source"]
-        assert ".target sm_100a" in src and "ex2.approx.ftz.f32" in src
+        assert ".target sm_100a" in src and "lg2.approx.ftz.f32" in src
+        assert ("ex2.approx.ftz.f32" in src) == (space != 2)
         assert cg["name"] + "_j" in src and cg["name"] + "_m" in src
+
+
+# ---------------------------------------------------------------- value spaces (f4)
+@pytest.mark.parametrize("space", [1, 2])
+def test_codegen_value_spaces_discrete(space):
+    """Log2 space and linear fp32 space give the oracle's values on the toy
+    SPN (joint + marginal, out-of-support values) and on exhaustive inputs
+    of tiny discrete SPNs (the `probability` type)."""
+    g = toy_spn()
+    x = toy_data(3000, seed=15)
+    _check(g, x, False, space)
+    _check(g, nan_mask(x, 0.3, 16), True, space)
+    for seed in range(4):
+        g = tiny_discrete_spn(seed)
+        doms = g.meta["domains"]
+        x = np.array(list(itertools.product(*[range(-1, k + 1) for k in doms])), np.float32)
+        _check(g, x, False, space)
+        _check(g, nan_mask(x, 0.3, seed), True, space)
+
+
+def test_codegen_value_space_auto_rule():
+    """Auto: linear for discrete SPNs inside the range bound (one lg2 per
+    root, no ex2 in the generated code), log2 for Gaussian SPNs; forcing
+    linear space on a Gaussian SPN is refused."""
+    lin = spnb.codegen(spnb.Graph(toy_spn()), 0, lang="ptx")["source"]
+    assert "ex2.approx" not in lin and lin.count("lg2.approx") == 2   # 1 root x (joint, marginal)
+    log = spnb.codegen(spnb.Graph(toy_spn()), 0, lang="ptx", space=1)["source"]
+    assert "ex2.approx" in log
+    gauss = spnb.codegen(spnb.Graph(speaker_spn(2001)), 0, lang="ptx")["source"]
+    assert "ex2.approx" in gauss
+    with pytest.raises(spnb.SPNError):
+        spnb.codegen(spnb.Graph(speaker_spn(2001)), 0, space=2)

@@ -219,15 +219,20 @@ def test_tiny_discrete_exact():
 
 
 # ----------------------------------------------------------------- layered tensor-core path (a5)
+@pytest.mark.parametrize("kernel", [1, 2])
 @pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (24, 1, 1, 4, 8, 2),
                                    (128, 3, 2, 20, 40, 10)])
-def test_layered_rat_small_matches_oracle(shape):
+def test_layered_rat_small_matches_oracle(shape, kernel):
+    """Both layered kernels (v1 rat_eval.cu, v2 rat2.cu), hi/lo and single
+    f16 passes, joint and marginal."""
     F, D, R, S, I, C = shape
     g = rat_spn(11, F=F, D=D, R=R, S=S, I=I, C=C)
     x, _ = ancestral_sample(g, 1000, 12)
-    err, P = _parity(g, x, layered_path=2, tc_precision=2)
-    assert P.info()["path"] == 1
-    _parity(g, nan_mask(x, 0.2, 13), marginal=True, layered_path=2, tc_precision=2)
+    for prec in ((2, 1) if kernel == 2 else (2,)):
+        err, P = _parity(g, x, layered_path=2, tc_precision=prec, layered_kernel=kernel)
+        assert P.info()["path"] == 1 and P.info()["layered_kernel"] == kernel
+        _parity(g, nan_mask(x, 0.2, 13), marginal=True, layered_path=2, tc_precision=prec,
+                layered_kernel=kernel)
 
 
 def test_layered_matches_generic_path():
@@ -257,9 +262,25 @@ def test_layered_ragged_and_chunked():
     g = rat_spn(31, F=256, D=3, R=2, S=8, I=8, C=3)
     x = np.random.default_rng(32).uniform(0, 1, size=(80_001, 256)).astype(np.float32)
     out, am, P = _run(g, x, layered_path=2)     # > one transposed chunk, ragged tail
+    assert P.info()["layered_kernel"] == 1      # (I, S) = (8, 8): no v2 instance
     idx = np.concatenate([np.arange(0, 50), np.arange(37_850, 37_950), np.arange(79_950, 80_001)])
     ref, _ = oracle_eval(g, x[idx])
     _cmp(out[idx], ref)
+
+
+def test_layered_v2_ragged_and_chunked():
+    """v2 kernel over two transposed chunks (148 x 128 x 8 samples each) with
+    a ragged tail; rows from both chunk edges against the oracle."""
+    g = rat_spn(33, F=128, D=3, R=2, S=4, I=8, C=3)
+    x = np.random.default_rng(34).uniform(0, 1, size=(160_001, 128)).astype(np.float32)
+    out, am, P = _run(g, x, layered_path=2)
+    info = P.info()
+    assert info["layered_kernel"] == 2 and info["chunk_samples"] < len(x)
+    c = info["chunk_samples"]
+    idx = np.concatenate([np.arange(0, 64), np.arange(c - 64, c + 64), np.arange(len(x) - 65, len(x))])
+    ref, am_ref = oracle_eval(g, x[idx])
+    _cmp(out[idx], ref)
+    _cmp_argmax(am[idx], ref, am_ref)
 
 
 # ----------------------------------------------------------------- compiled path (KS)
@@ -368,15 +389,80 @@ def test_c4_layered_marginal_full_graph_sampled():
 
 
 def test_c5_layered_full_graph_sampled():
-    """Config 5 graph (3,242,010 nodes) on the layered path, counter-based
-    U[0,1] inputs (the bench recipe) over two transposed chunks with a ragged
-    tail; oracle on rows from the start, the chunk boundary and the end."""
+    """Config 5 graph (3,242,010 nodes) on the layered path in the bench's
+    launch configuration (default plan, counter-based U[0,1] inputs) over two
+    transposed chunks with a ragged tail; oracle on rows from the start, the
+    chunk boundary and the end."""
     from spn_inputs import config_graph, uniform_chunked
     g = config_graph("C5")
-    x = uniform_chunked(40_001, g.n_features, 5002)
-    out, am, P = _run(g, x, layered_path=2)
-    assert P.info()["path"] == 1
-    idx = np.concatenate([np.arange(0, 16), np.arange(18_936, 18_952), np.arange(39_985, 40_001)])
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    c = P.info()["chunk_samples"]
+    n = c + 10_001
+    x = uniform_chunked(n, g.n_features, 5002)
+    out, am = P.infer(torch.from_numpy(x).cuda())
+    torch.cuda.synchronize()
+    out, am = out.cpu().numpy(), am.cpu().numpy()
+    assert P.info()["path"] == 1 and P.info()["layered_kernel"] == 2
+    idx = np.concatenate([np.arange(0, 16), np.arange(c - 16, c + 16), np.arange(n - 16, n)])
+    ref, am_ref = oracle_eval(g, x[idx])
+    _cmp(out[idx], ref)
+    _cmp_argmax(am[idx], ref, am_ref)
+
+
+def test_c5_partitioned_generic_vs_layered_vs_oracle():
+    """BASELINE configs[4] "partitioned into tasks": the C5 graph through the
+    generic interpreter with the paper's <= 10k-operation tasks (PAPER.md
+    L336-346, L481-485; several thousand tasks, cut values in global
+    scratch) on 10k ancestral samples, against the layered tensor-core path
+    on all 10k rows and both against the fp64 oracle on 1k rows."""
+    from spn_inputs import config_graph
+    g = config_graph("C5")
+    x, _ = ancestral_sample(g, 10_000, 5003)
+    G = spnb.Graph(g)
+    Pg = spnb.Plan(G, layered_path=1, compiled_path=1, max_task_nodes=10_000)
+    ig = Pg.info()
+    assert ig["path"] == 0 and ig["n_tasks"] > 1000 and ig["n_global_slots"] > 0, ig
+    xt = torch.from_numpy(x).cuda()
+    og, amg = Pg.infer(xt)
+    Pl = spnb.Plan(G)
+    assert Pl.info()["path"] == 1
+    ol, aml = Pl.infer(xt)
+    torch.cuda.synchronize()
+    og, amg, ol, aml = og.cpu().numpy(), amg.cpu().numpy(), ol.cpu().numpy(), aml.cpu().numpy()
+    _cmp(og, ol.astype(np.float64))
+    idx = np.random.default_rng(7).choice(len(x), 1000, replace=False)
+    ref, am_ref = oracle_eval(g, x[idx])
+    _cmp(og[idx], ref)
+    _cmp(ol[idx], ref)
+    _cmp_argmax(amg[idx], ref, am_ref)
+    _cmp_argmax(aml[idx], ref, am_ref)
+
+
+@pytest.mark.parametrize("which", ["compiled", "interpreter", "layered"])
+def test_host_api_matches_oracle(which):
+    """spn_infer_*_host (pinned host buffers, chunked copies overlapped with
+    compute on two streams) over more than two host
+    chunks: bitwise equal to the device-buffer call and within tolerance of
+    the oracle on rows from every chunk."""
+    from spn_inputs import config_graph
+    if which == "compiled":
+        g, n, opt = speaker_spn(2001), 2_600_000, {}
+    elif which == "interpreter":
+        g, n, opt = rat_spn(41, F=256, D=3, R=3, S=6, I=8, C=4), 70_000, {"layered_path": 1,
+                                                                           "compiled_path": 1,
+                                                                           "max_task_nodes": 400}
+    else:
+        g, n, opt = config_graph("C4"), 20_000, {}
+    x, _ = ancestral_sample(g, n, 42)
+    G = spnb.Graph(g)
+    P = spnb.Plan(G, **opt)
+    dev, amd = P.infer(torch.from_numpy(x).cuda())
+    xh = torch.from_numpy(x).pin_memory()
+    out, am = P.infer_host(xh)
+    assert np.array_equal(out, dev.cpu().numpy())
+    assert np.array_equal(am, amd.cpu().numpy())
+    idx = np.linspace(0, n - 1, 240).astype(np.int64)
     ref, am_ref = oracle_eval(g, x[idx])
     _cmp(out[idx], ref)
     _cmp_argmax(am[idx], ref, am_ref)

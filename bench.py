@@ -37,9 +37,14 @@ METRIC = "SPN inference samples/sec (joint & marginal) at 1/2/4/8 B200; % of HBM
 UNIT = "samples/s"
 
 
+_N_OVERRIDE = {}
+
+
 def CONFIGS_N(cfg: str) -> int:
+    """Samples of a config (BASELINE.json sizes; --samples overrides, e.g. C1
+    at 1e8 where the toy SPN becomes HBM-bound)."""
     from spn_inputs import CONFIGS
-    return CONFIGS[cfg]["n_samples"]
+    return _N_OVERRIDE.get(cfg, CONFIGS[cfg]["n_samples"])
 
 
 def _peaks():
@@ -56,7 +61,7 @@ def samples_per_rank(cfg: str, world: int) -> tuple[int, str]:
     BASELINE.json configs[4]); the others are weak (a full batch per GPU)."""
     from spn_inputs import CONFIGS
     from paper_conf_cgo_sommera022_b200.parallel import shard_sizes
-    n = CONFIGS[cfg]["n_samples"]
+    n = CONFIGS_N(cfg)
     if cfg == "C5":
         return max(shard_sizes(n, world)), "strong"
     return n, "weak"
@@ -87,7 +92,7 @@ def make_workload(cfg: str, rank: int, marginal: bool, n_max: int | None = None)
                             toy_data, uniform_chunked)
     c = CONFIGS[cfg]
     g = config_graph(cfg)
-    n = c["n_samples"]
+    n = CONFIGS_N(cfg)
     if cfg == "C1":
         x = toy_data(n, seed=1001 + rank)
         if marginal:
@@ -228,14 +233,17 @@ def run_reference(args):
 def _config_dict(args, g, n, world=1, scaling="weak"):
     from spn_inputs import CONFIGS
     c = g.counts()
-    d = {"workload": f"{args.config}: {CONFIGS[args.config]['desc']}",
+    desc = CONFIGS[args.config]["desc"]
+    if args.config in _N_OVERRIDE:
+        desc += f" [--samples {_N_OVERRIDE[args.config]}]"
+    d = {"workload": f"{args.config}: {desc}",
          "query": "marginal" if args.marginal else "joint",
          "samples_per_gpu": n, "n_features": g.n_features, "n_roots": g.n_roots,
          "graph_nodes": c["nodes"], "sum_edges": c["sum_edges"],
          "l2": "flushed between timed steps (256 MiB write)",
          "parallelism": f"dp{world} (sample sharding)"}
     if scaling == "strong":
-        d["samples_total"] = CONFIGS[args.config]["n_samples"]
+        d["samples_total"] = CONFIGS_N(args.config)
         d["l2"] = ("inputs larger than L2 (31 GB / N) and L2 flushed between timed steps "
                    "(256 MiB write)")
     return d
@@ -276,7 +284,7 @@ def run_ours(args):
         from paper_conf_cgo_sommera022_b200.parallel import shard_range
         g = config_graph(args.config)
         n = n_rank
-        lo = shard_range(CONFIGS[args.config]["n_samples"], rank, world)[0] if scaling == "strong" \
+        lo = shard_range(CONFIGS_N(args.config), rank, world)[0] if scaling == "strong" \
             else rank * n
         xd = device_uniform(n, g.n_features, CONFIGS[args.config]["data_seed"], lo, dev)
         x = xd[:min(n, 1 << 20)].cpu().numpy()   # host copy of a bounded subset (e2e, oracle)
@@ -467,7 +475,11 @@ def main():
     ap.add_argument("--block", type=int, default=0, help="threads per CTA (0 = auto)")
     ap.add_argument("--tc-precision", type=int, default=0,
                     help="layered path: 0 auto, 1 single f16 pass, 2 f16 hi/lo split")
+    ap.add_argument("--samples", type=int, default=0,
+                    help="override the config's sample count (e.g. C1 at 100000000)")
     args = ap.parse_args()
+    if args.samples > 0:
+        _N_OVERRIDE[args.config] = args.samples
     if args.impl == "reference":
         run_reference(args)
     else:

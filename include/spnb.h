@@ -80,8 +80,12 @@ typedef struct spn_prepare_options {
                                    the DAG is not a layered region graph)    */
     int64_t max_task_nodes;     /* partition cap in LoSPN ops;
                                    0 = auto (shared-memory budget), -1 = none  */
-    int32_t tc_precision;       /* layered path: 0 auto (= 2), 1 f16 single
-                                   pass, 2 f16 hi/lo split (3 MMAs, ~fp32)    */
+    int32_t tc_precision;       /* layered path: 0 auto, 1 f16 single pass, 2
+                                   f16 hi/lo split (3 MMAs, ~fp32; v1 kernel).
+                                   Auto: the v2 kernel's single pass with
+                                   per-sample certification (spn_plan_stats
+                                   cert_err); samples failing it are
+                                   recomputed in hi/lo within the same call  */
     int32_t ctas_per_sm;        /* 0 = auto; compiled path: the kernels'
                                    __launch_bounds__ minimum CTAs per SM     */
     int32_t compiled_path;      /* 0 auto, 1 off (interpreter), 2 force: one
@@ -151,7 +155,17 @@ typedef struct spn_plan_stats {
     int32_t layered_kernel;     /* layered path: 1 v1, 2 v2 (0 other paths)   */
     int32_t tc_passes;          /* layered path: f16 MMA passes (1 or 3)      */
     int32_t value_space;        /* 1 log2 space, 2 linear fp32 (compiled path) */
-    int32_t reserved_;
+    int32_t certified;          /* layered v2, tc_precision auto: 1 when every
+                                   sample's single-pass result is checked
+                                   against cert_err and failures recomputed in
+                                   hi/lo precision (v1 kernel)                */
+    double  cert_err;           /* layered v2: a-priori bound (nats) on the
+                                   single f16 pass's deviation from the exact
+                                   contraction, for every root; a sample is
+                                   kept when cert_err <= 0.9e-4 max(1, |ln p|
+                                   - cert_err) for all its roots (the other
+                                   0.1e-4 of the tolerance covers the fp32
+                                   arithmetic both precisions share)          */
 } spn_plan_stats;
 
 /* Fill *opt with defaults (all auto). */
@@ -271,10 +285,12 @@ int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, i
  *   sizes[2] fparams (float), sizes[3] weight-image bytes, sizes[4] roots;
  *   dims[11] = {F, C, I, S, D, gcols, kpad_bot, kpad_up, max_wgroup,
  *   max_vars, max_blk}.  NULL buffers: sizes and dims only.
+ *   *tc_err_1pass (nullable) receives the plan's a-priori bound (nats) on
+ *   the single f16 pass's deviation from the exact contraction.
  */
 int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
                        int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
-                       void *wimg, int32_t *root_map);
+                       void *wimg, int32_t *root_map, double *tc_err_1pass);
 int spn_partition_graph(const spn_handle *graph, int64_t max_task_ops, int32_t *task_of_node,
                         int32_t *n_tasks, int64_t *cost, int64_t *cut_values);
 int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32_t x_in_smem,

@@ -70,7 +70,8 @@ class _Stats(ctypes.Structure):
         ("ctas_per_sm", ctypes.c_int32), ("mufu_exec_per_sample", ctypes.c_int64),
         ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64),
         ("layered_kernel", ctypes.c_int32), ("tc_passes", ctypes.c_int32),
-        ("value_space", ctypes.c_int32), ("reserved_", ctypes.c_int32)]
+        ("value_space", ctypes.c_int32), ("certified", ctypes.c_int32),
+        ("cert_err", ctypes.c_double)]
 
 
 _lib = None
@@ -100,7 +101,7 @@ def load_library(path: str | None = None):
     lib.spn_partition_graph.argtypes = [P, I64, P, P, P, P]
     lib.spn_build_program.argtypes = [P, I32, I32, I64, I64, P, P, P, P, P, P, P, P, P]
     lib.spn_build_layered.argtypes = [P, P, P, I64, P, P, P, P, P, P]
-    lib.spn_build_layered2.argtypes = [P, P, P, I64, P, P, P, P, P, P, P]
+    lib.spn_build_layered2.argtypes = [P, P, P, I64, P, P, P, P, P, P, P, P]
     lib.spn_codegen.argtypes = [P, I32, I32, P, P, P, P, P, P, P, P, I32, ctypes.c_char_p]
     for name in ("spn_load_graph", "spn_prepare", "spn_infer_joint", "spn_infer_marginal",
                  "spn_infer_joint_host", "spn_infer_marginal_host", "spn_plan_info",
@@ -349,8 +350,9 @@ def build_layered2(graph: Graph):
     why = ctypes.create_string_buffer(256)
     sizes = np.zeros(6, dtype=np.int64)
     dims = np.zeros(11, dtype=np.int32)
+    err = ctypes.c_double()
     _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
-                                  _ptr(dims), None, None, None, None, None))
+                                  _ptr(dims), None, None, None, None, None, ctypes.byref(err)))
     if not ok.value:
         return None, why.value.decode()
     assert sizes[5] == R2STEP_DTYPE.itemsize, (sizes[5], R2STEP_DTYPE.itemsize)
@@ -361,11 +363,11 @@ def build_layered2(graph: Graph):
     rm = np.zeros(sizes[4], dtype=np.int32)
     _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
                                   _ptr(dims), _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w),
-                                  _ptr(rm)))
+                                  _ptr(rm), None))
     keys = ("F", "C", "I", "S", "D", "gcols", "kpad_bot", "kpad_up", "max_wgroup", "max_vars",
             "max_blk")
     return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
-            **{k: int(v) for k, v in zip(keys, dims)}}, ""
+            "tc_err_1pass": float(err.value), **{k: int(v) for k, v in zip(keys, dims)}}, ""
 
 
 def codegen(graph: Graph, task: int = 0, lang: str = "cpp", compile: bool = False,

@@ -43,6 +43,12 @@ cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float
 bool rat2_supported_shape(int I, int S);
 int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int kpad_up,
                 int max_wgroup, int prec, int n_in, int n_w);
+cudaError_t cert_gather_launch(const float *x, int64_t ld, int F, const int64_t *idx,
+                               const int32_t *count, int64_t off, int64_t cap, float *xT,
+                               int64_t ldT, cudaStream_t st);
+cudaError_t cert_scatter_launch(const float *tmp, const int32_t *am_tmp, const int64_t *idx,
+                                const int32_t *count, int64_t off, int64_t cap, int C, float *out,
+                                int32_t *am, cudaStream_t st);
 cudaError_t rat2_launch(const R2Params &p, const int32_t *leaf_steps, int n_leaf,
                         const int32_t *sum_steps, int n_sum, bool marg, int grid, cudaStream_t st);
 cudaError_t argmax_rows_launch(const float *out, int64_t n, int R, int32_t *argmax, cudaStream_t st);
@@ -121,6 +127,15 @@ struct DevicePlan {
     float *d_r2fp = nullptr;
     uint8_t *d_r2w = nullptr;
     int32_t n_r2leaf = 0, n_r2sum = 0;
+    // certified single pass (tc_precision auto): samples whose a-priori
+    // error bound does not fit the tolerance are recomputed by v1 in hi/lo
+    bool cert = false;
+    float cert_err = 0.f;
+    int32_t *d_flag_count = nullptr;
+    int64_t *d_flag_idx = nullptr;  // grown (stream-ordered) to the largest n seen
+    int64_t flag_cap = 0;
+    float *d_cert_out = nullptr;
+    int32_t *d_cert_am = nullptr;
     // compiled (per-SPN generated kernel) path
     std::vector<JitKernel> jk;
     std::vector<int32_t> jgrid_max;         // per task: SMs x CTAs/SM (joint kernel)
@@ -191,6 +206,10 @@ void free_plan(DevicePlan *p) {
     cudaFree(p->d_r2sum);
     cudaFree(p->d_r2fp);
     cudaFree(p->d_r2w);
+    cudaFree(p->d_flag_count);
+    if (p->d_flag_idx) cudaFreeAsync(p->d_flag_idx, 0);
+    cudaFree(p->d_cert_out);
+    cudaFree(p->d_cert_am);
     for (auto &k : p->jk) jit_unload(k);
     if (p->d_prof) {
         unsigned long long h[8];
@@ -285,6 +304,31 @@ int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *ou
     return SPN_OK;
 }
 
+// parameters of the v1 layered kernel (rat_eval.cu) of a plan
+RParams v1_params(const DevicePlan &P) {
+    RParams rp;
+    memset(&rp, 0, sizeof(rp));
+    rp.steps = P.d_steps;
+    rp.n_steps = P.n_steps;
+    rp.C = P.R;
+    rp.vars = P.d_vars;
+    rp.fparams = P.d_fparams;
+    rp.wimg = P.d_wimg;
+    rp.root_map = P.d_root_map;
+    rp.prec = P.prec;
+    rp.smem_floats = P.smem_floats;
+    rp.max_kpad = P.max_kpad;
+    rp.max_ngroup = P.max_ngroup;
+    rp.max_na = P.max_na;
+    rp.max_vars = P.max_vars;
+    rp.first_leaf = P.first_leaf;
+    rp.max_leaf_params = P.max_leaf_params;
+    rp.wbufs = P.wbufs;
+    rp.overlap = P.tmem_overlap;
+    rp.prof = P.r2 ? nullptr : P.d_prof;
+    return rp;
+}
+
 int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                       int32_t *argmax, void *stream, bool marg) {
     if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
@@ -316,7 +360,28 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
         R2Params rp = P.r2p;
         rp.xT = P.d_xT;
         rp.ldT = P.chunk;
+        cudaError_t e;
+        if (P.cert) {
+            if (n > P.flag_cap) {  // room for every sample of this call
+                if (P.d_flag_idx) cudaFreeAsync(P.d_flag_idx, (cudaStream_t)stream);
+                P.d_flag_idx = nullptr;
+                P.flag_cap = 0;
+                if ((e = cudaMallocAsync((void **)&P.d_flag_idx, (size_t)n * 8, (cudaStream_t)stream)) !=
+                    cudaSuccess)
+                    return set_err(SPN_E_OOM, "certification index list");
+                P.flag_cap = n;
+            }
+            if ((e = cudaMemsetAsync(P.d_flag_count, 0, sizeof(int32_t), (cudaStream_t)stream)) != cudaSuccess)
+                return cuda_err(e, "cudaMemsetAsync");
+            rp.flag_count = P.d_flag_count;
+            rp.flag_idx = P.d_flag_idx;
+            rp.cert_err = P.cert_err;
+            // 0.9 of the north-star tolerance (1e-4): the remaining 0.1 covers the fp32
+            // arithmetic both precisions share (measured 2.2e-7 relative on C4, hi/lo vs oracle)
+            rp.cert_tol = 0.9e-4f;
+        }
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
+            rp.row0 = c0;
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
             cudaError_t e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
@@ -330,31 +395,35 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
                             (cudaStream_t)stream);
             if (e != cudaSuccess) return cuda_err(e, "rat2 launch");
         }
+        if (P.cert) {
+            // flagged samples (count on the device): gather their rows into the
+            // transposed scratch, v1 kernel in hi/lo precision, scatter back;
+            // one round per chunk of capacity, each a no-op when nothing is left
+            RParams vp = v1_params(P);
+            vp.xT = P.d_xT;
+            vp.ldT = P.chunk;
+            vp.out = P.d_cert_out;
+            vp.argmax = P.d_cert_am;
+            vp.n = P.chunk;
+            vp.n_count = P.d_flag_count;
+            for (int64_t off = 0; off < n; off += P.chunk) {
+                vp.n_off = off;
+                if ((e = cert_gather_launch(x, ld, P.F, P.d_flag_idx, P.d_flag_count, off, P.chunk, P.d_xT,
+                                            P.chunk, (cudaStream_t)stream)) != cudaSuccess)
+                    return cuda_err(e, "certification gather");
+                if ((e = rat_launch(vp, marg, P.grid_max, P.smem, (cudaStream_t)stream)) != cudaSuccess)
+                    return cuda_err(e, "certification recompute");
+                if ((e = cert_scatter_launch(P.d_cert_out, P.d_cert_am, P.d_flag_idx, P.d_flag_count, off,
+                                             P.chunk, P.R, out, argmax, (cudaStream_t)stream)) != cudaSuccess)
+                    return cuda_err(e, "certification scatter");
+            }
+        }
         return SPN_OK;
     }
     if (P.path == 1) {
-        RParams rp;
-        memset(&rp, 0, sizeof(rp));
-        rp.steps = P.d_steps;
-        rp.n_steps = P.n_steps;
-        rp.C = P.R;
-        rp.vars = P.d_vars;
-        rp.fparams = P.d_fparams;
-        rp.wimg = P.d_wimg;
-        rp.root_map = P.d_root_map;
+        RParams rp = v1_params(P);
         rp.xT = P.d_xT;
         rp.ldT = P.chunk;
-        rp.prec = P.prec;
-        rp.smem_floats = P.smem_floats;
-        rp.max_kpad = P.max_kpad;
-        rp.max_ngroup = P.max_ngroup;
-        rp.max_na = P.max_na;
-        rp.max_vars = P.max_vars;
-        rp.first_leaf = P.first_leaf;
-        rp.max_leaf_params = P.max_leaf_params;
-        rp.wbufs = P.wbufs;
-        rp.overlap = P.tmem_overlap;
-        rp.prof = P.d_prof;
         for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
@@ -514,9 +583,15 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         // deepest rings that fit: leaf inputs 3..2 (3 lets both leaf groups
         // prefetch), weight groups 4..2 (the MMA warp holds a pair at once)
         static const int kRings[][2] = {{3, 4}, {3, 3}, {3, 2}, {2, 4}, {2, 2}};
+        // v2 runs the single f16 pass (hi/lo operands do not fit its shared
+        // memory on C4/C5-sized regions): tc_precision 2 keeps v1
+        if (r2.ok && opt.tc_precision == 2) {
+            r2.ok = false;
+            r2.why = "tc_precision 2 (hi/lo) runs on the v1 kernel";
+        }
         for (int a = 0; r2.ok && a < 5 && !fits; ++a)
             fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
-                               r2.max_wgroup, P->prec, kRings[a][0], kRings[a][1]) <= smem_optin;
+                               r2.max_wgroup, 1, kRings[a][0], kRings[a][1]) <= smem_optin;
         if (r2.ok && fits) {
             std::vector<int32_t> leaf_idx, sum_idx;
             for (int32_t t = 0; t < (int32_t)r2.steps.size(); ++t)
@@ -539,7 +614,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
             rp.fparams = P->d_r2fp;
             rp.wimg = P->d_r2w;
             rp.root_map = P->d_r2rm;
-            rp.prec = P->prec;
+            rp.prec = 1;
             rp.max_vars = r2.max_vars;
             rp.max_blk = r2.max_blk;
             rp.kpad_bot = r2.kpad_bot;
@@ -550,12 +625,22 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
             rp.prof = P->d_prof;
             P->r2p = rp;
             P->r2 = true;
+            // auto precision: certify every sample's single-pass result against
+            // the a-priori bound; failures are recomputed by v1 in hi/lo
+            P->cert = opt.tc_precision == 0 && std::isfinite(r2.tc_err_1pass);
+            P->cert_err = (float)r2.tc_err_1pass;
             P->n_r2leaf = (int32_t)leaf_idx.size();
             P->n_r2sum = (int32_t)sum_idx.size();
-            P->smem = rp.smem_bytes;
+            // (P->smem stays the v1 kernel's: it serves the certification fallback)
             // persistent kernel over many tiles per launch: 8 tiles per CTA
             chunk = (int64_t)sms * 128 * 8;
             P->chunk = chunk;
+            if (P->cert && (cudaMalloc(&P->d_flag_count, sizeof(int32_t)) != cudaSuccess ||
+                            cudaMalloc(&P->d_cert_out, (size_t)4 * chunk * lp.C) != cudaSuccess ||
+                            cudaMalloc(&P->d_cert_am, (size_t)4 * chunk) != cudaSuccess)) {
+                free_plan(P);
+                return set_err(SPN_E_OOM, "certification buffers");
+            }
         } else if (want_r2 == 2) {
             free_plan(P);
             return set_err(SPN_E_UNSUPPORTED, "layered v2 kernel not applicable: " +
@@ -600,10 +685,12 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     s.block_threads = P->r2 ? 512 : (lp.max_na > 48 ? 256 : 512);
     s.samples_per_thread = 0;
     s.grid = P->grid_max;
-    s.smem_bytes = (int32_t)P->smem;
+    s.smem_bytes = (int32_t)(P->r2 ? P->r2p.smem_bytes : P->smem);
     s.x_in_smem = 0;
     s.layered_kernel = P->r2 ? 2 : 1;
-    s.tc_passes = P->prec == 3 ? 3 : 1;
+    s.tc_passes = P->r2 ? 1 : (P->prec == 3 ? 3 : 1);
+    s.cert_err = P->r2 ? P->cert_err : 0.0;
+    s.certified = P->cert ? 1 : 0;
     s.prepare_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     spn_handle *h = new (std::nothrow) spn_handle();
@@ -1151,7 +1238,7 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
 
 int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
                        int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
-                       void *wimg, int32_t *root_map) {
+                       void *wimg, int32_t *root_map, double *tc_err_1pass) {
     if (!valid_graph_handle(graph) || !ok || !sizes || !dims) return set_err(SPN_E_ARG, "bad arguments");
     LayeredPlan lp;
     detect_layered(*graph->graph, lp);
@@ -1171,6 +1258,7 @@ int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t 
     const int32_t d[11] = {p.F, p.C, p.I, p.S, p.D, p.gcols, p.kpad_bot, p.kpad_up,
                            p.max_wgroup, p.max_vars, p.max_blk};
     memcpy(dims, d, sizeof(d));
+    if (tc_err_1pass) *tc_err_1pass = p.tc_err_1pass;
     if (steps) memcpy(steps, p.steps.data(), p.steps.size() * sizeof(R2Step));
     if (vars) memcpy(vars, p.vars.data(), p.vars.size() * 4);
     if (fparams) memcpy(fparams, p.fparams.data(), p.fparams.size() * 4);

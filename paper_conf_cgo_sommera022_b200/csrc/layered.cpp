@@ -542,7 +542,9 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
     p.ea_max = (na_max + 7) / 8 * 8;
     p.kpad_bot = (I + 15) / 16 * 16;
     p.kpad_up = S > 0 ? (S + 15) / 16 * 16 : 16;
-    // ---- steps
+    // ---- steps (and the single-pass error bound, log2 units, per step)
+    std::vector<double> err(ns, 0.0);
+    double err_root = 0.0;
     for (int32_t t = 0; t < ns; ++t) {
         const LStep &st = lp.steps[t];
         R2Step r;
@@ -610,13 +612,31 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
         while (p.fparams.size() % 4) p.fparams.push_back(0.f);
         r.blk_off = (int64_t)p.fparams.size();
         std::vector<double> scale(n_out, 1.0);
+        double eps_step = 0.0;  // largest relative error of one of this step's sums
         for (int32_t s2 = 0; s2 < n_out; ++s2) {
-            double mx = 0.0;
-            for (int64_t c = 0; c < (int64_t)na * nb; ++c) mx = std::max(mx, W[(size_t)s2 * na * nb + c]);
+            double mx = 0.0, mn = INFINITY, tot = 0.0;
+            for (int64_t c = 0; c < (int64_t)na * nb; ++c) {
+                const double w = W[(size_t)s2 * na * nb + c];
+                mx = std::max(mx, w);
+                mn = std::min(mn, w);
+                tot += w;
+            }
             const int k = mx > 0.0 ? -(int)std::floor(std::log2(mx)) : 0;
             scale[s2] = std::ldexp(1.0, k);
             p.fparams.push_back((float)k);
+            double ew = 0.0;  // exact relative rounding of the f16 weights of this sum
+            for (int64_t c = 0; c < (int64_t)na * nb; ++c) {
+                const double w = W[(size_t)s2 * na * nb + c] * scale[s2];
+                if (w > 0.0) ew = std::max(ew, std::fabs((double)f16_to_f32(f32_to_f16((float)w)) - w) / w);
+            }
+            const double rho = mn > 0.0 ? tot / mn : INFINITY;
+            const double u16 = std::ldexp(1.0, -11), u32 = std::ldexp(1.0, -24);
+            const double delta = (1.0 + ew) * (1.0 + u16) - 1.0 + std::ldexp(rho, -29) +
+                                 (double)(nb + na + 8) * u32;
+            eps_step = std::max(eps_step, delta < 0.5 ? -std::log1p(-delta) / M_LN2 : INFINITY);
         }
+        err[t] = eps_step + err[lp.child_a[t]] + err[lp.child_b[t]];
+        if (st.type == 2) err_root = std::max(err_root, err[t]);
         while (p.fparams.size() % 4) p.fparams.push_back(0.f);
         r.wbytes_a = (int64_t)r.ncol_a * r.kpad * 2;
         r.wbytes_b = (int64_t)r.ncol_b * r.kpad * 2;
@@ -652,6 +672,7 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
         p.steps.push_back(r);
     }
     p.root_map = lp.root_map;
+    p.tc_err_1pass = err_root * M_LN2;
     p.ok = true;
 }
 

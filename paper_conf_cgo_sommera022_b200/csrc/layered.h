@@ -110,6 +110,14 @@ struct Rat2Plan {
     std::vector<uint16_t> wimg;                 // f16 images
     std::vector<int32_t> root_map;
     int64_t n_leaf = 0, n_sum = 0;
+    // a-priori bound (natural log units) on |ln p(1 f16 pass) - ln p(exact
+    // contraction)| for every root: per sum, the exact relative rounding of
+    // its f16 weights, the f16 rounding of the B-side exps (2^-11, normal
+    // range by the 2^15 shift), the flushed exps below 2^-29 (2^-29 times
+    // sum/min weight) and fp32 accumulation; propagated bottom-up (a
+    // product adds its children's bounds, a sum adds its own, LSE being
+    // 1-Lipschitz in the max norm).  Infinite if a sum has a zero weight.
+    double tc_err_1pass = 0.0;
 };
 
 // Builds the v2 plan from a detected layered plan; fails (ok = false, why)
@@ -138,6 +146,14 @@ struct R2Params {
         off_w, w_bytes, off_bar;
     int32_t smem_bytes;
     unsigned long long *prof;  // optional: per-role phase cycles [4 roles][8] (SPNB_PROFILE)
+    // certification of the single f16 pass (tc_precision auto): a sample
+    // whose roots do not all satisfy cert_err <= cert_tol * max(1, |ln p| -
+    // cert_err) is appended to flag_idx (global row = row0 + tile row) for
+    // the hi/lo recomputation; flag_count == nullptr: no certification
+    float cert_err, cert_tol;
+    int32_t *flag_count;
+    int64_t *flag_idx;
+    int64_t row0;
 };
 
 // Detects the structure; on success fills plan (ok = true).
@@ -169,6 +185,10 @@ struct RParams {
                         // on C4: 5.78e6 vs 5.45e6 samples/s with 16 warps (TMEM reads
                         // under a running MMA are slower, but the MMA is hidden)
     unsigned long long *prof;  // optional phase-cycle counters (thread 0 of each CTA)
+    // optional device-side sample count (the certification fallback): when
+    // set, n = clamp(*n_count - n_off, 0, n) is read by the kernel itself
+    const int32_t *n_count;
+    int64_t n_off;
 };
 
 }  // namespace spnb

@@ -40,8 +40,8 @@ namespace r2 {
 constexpr int RT = 128;           // samples per tile = UMMA M = TMEM lanes
 // 16 warps = 4 warpgroups: leaf group 0, leaf group 1, epilogue, and
 // {leaf producer, MMA, weight producer, idle}.  setmaxnreg moves registers
-// from the last warpgroup (40 each) to the epilogue (216 each); the leaf
-// warpgroups keep the launch's 128: 2*128 + 216 + 40 = 512 per SMSP lane.
+// from the last warpgroup (56 each) to the epilogue (200 each); the leaf
+// warpgroups keep the launch's 128: 2*128 + 200 + 56 = 512 per SMSP lane.
 constexpr int NTHREADS = 16 * 32;
 constexpr int W_EPI0 = 8, W_PROD = 12, W_MMA = 13, W_WPROD = 14;
 constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
@@ -76,14 +76,18 @@ __device__ __forceinline__ uint32_t smem_u32(const void *p) {
 __device__ __forceinline__ void bar_init(uint32_t b, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(b), "r"(count));
 }
+// try_wait with a suspend-time hint: a waiting warp is parked by the
+// hardware until the phase completes (or the hint expires) instead of
+// spinning -- spinning producer / MMA warps (the highest warp ids, which the
+// scheduler favours) would otherwise take issue slots from the epilogue
 __device__ __forceinline__ void bar_wait(uint32_t b, uint32_t parity) {
     uint32_t done = 0;
     while (!done) {
         asm volatile(
-            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
             "selp.u32 %0, 1, 0, p;\n\t}\n"
             : "=r"(done)
-            : "r"(b), "r"(parity)
+            : "r"(b), "r"(parity), "r"(0x989680u)
             : "memory");
     }
 }
@@ -437,13 +441,44 @@ __device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int3
     pf.mark(7);
 }
 
+// the fields of a sum step the MMA / epilogue / weight roles use, loaded once
+// per step into registers (held by reference, every use in a loop would be a
+// dependent global load on the role's critical path)
+struct SumStep {
+    int type, root, n_out, na, kpad, n_groups, spg_a, ncol_a, spg_b, ncol_b, slot_a, slot_b,
+        slot_out;
+    int64_t blk_off, w_off, wbytes_a, wbytes_b;
+};
+__device__ __forceinline__ SumStep load_sum_step(const R2Step *steps, const int32_t *idx, int si) {
+    const R2Step *q = steps + __ldg(idx + si);
+    SumStep r;
+    r.type = __ldg(&q->type);
+    r.root = __ldg(&q->root);
+    r.n_out = __ldg(&q->n_out);
+    r.na = __ldg(&q->na);
+    r.kpad = __ldg(&q->kpad);
+    r.n_groups = __ldg(&q->n_groups);
+    r.spg_a = __ldg(&q->spg_a);
+    r.ncol_a = __ldg(&q->ncol_a);
+    r.spg_b = __ldg(&q->spg_b);
+    r.ncol_b = __ldg(&q->ncol_b);
+    r.slot_a = __ldg(&q->slot_a);
+    r.slot_b = __ldg(&q->slot_b);
+    r.slot_out = __ldg(&q->slot_out);
+    r.blk_off = __ldg(&q->blk_off);
+    r.w_off = __ldg(&q->w_off);
+    r.wbytes_a = __ldg(&q->wbytes_a);
+    r.wbytes_b = __ldg(&q->wbytes_b);
+    return r;
+}
+
 // group gi of a sum step: first sum, number of sums (0: empty), MMA columns,
 // image byte offset relative to w_off and bytes of one part image
 struct GroupInfo {
     int s0, ns, ncol;
     int64_t off, bytes;
 };
-__device__ __forceinline__ GroupInfo group_info(const R2Step &st, int gi) {
+__device__ __forceinline__ GroupInfo group_info(const SumStep &st, int gi) {
     const bool b = gi & 1;
     const int pair = gi >> 1;
     GroupInfo g;
@@ -464,7 +499,7 @@ __device__ void weight_producer_role(const R2Params &p, const Smem &sm, const in
     Prof pf(sm.prof(3), p.prof != nullptr);  // 2 wait weight slot, 7 issue
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         for (int si = 0; si < n_sum; ++si) {
-            const R2Step &st = p.steps[__ldg(sum_steps + si)];
+            const SumStep st = load_sum_step(p.steps, sum_steps, si);
             for (int gi = 0; gi < st.n_groups; ++gi) {
                 const GroupInfo gr = group_info(st, gi);
                 if (gr.ns == 0) continue;  // empty group: no weights (the MMA skips it too)
@@ -517,8 +552,10 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
     const uint32_t wlo_d = (uint32_t)p.max_wgroup >> 4;
     Prof pf(sm.prof(2), p.prof != nullptr);  // 0 wait A operand, 1 wait weights, 2 wait TMEM, 3 issue
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        SumStep nx = load_sum_step(p.steps, sum_steps, 0);
         for (int si = 0; si < n_sum; ++si) {
-            const R2Step &st = p.steps[__ldg(sum_steps + si)];
+            const SumStep st = nx;
+            if (si + 1 < n_sum) nx = load_sum_step(p.steps, sum_steps, si + 1);
             const bool bot = st.type == 1;
             const int G = st.n_groups, ksteps = st.kpad / 16;
             uint32_t a_addr;
@@ -623,15 +660,35 @@ __device__ __forceinline__ float dot_part(const float (&ea)[NA], int off, const 
     }
     return (p0.x + p0.y) + (p1.x + p1.y);
 }
+// W columns of one TMEM lane (W a multiple of 4): x16 / x8 / x4 loads
+template <int W>
+__device__ __forceinline__ void ld_cols(uint32_t taddr, float *t) {
+#pragma unroll
+    for (int c = 0; c + 16 <= W; c += 16) tmem_ld16(taddr + c, t + c);
+    if constexpr (W % 16 >= 8) tmem_ld8(taddr + (W / 16) * 16, t + (W / 16) * 16);
+    if constexpr (W % 8) tmem_ld4(taddr + (W / 8) * 8, t + (W / 8) * 8);
+}
+// sum_i ea_i t_i with four FFMA2 chains (eight partial sums)
+template <int NA>
+__device__ __forceinline__ float dot4(const float (&ea)[NA], const float *t) {
+    float2 q[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f),
+                   make_float2(0.f, 0.f)};
+#pragma unroll
+    for (int i = 0; i + 2 <= NA; i += 2)
+        q[(i / 2) & 3] = __ffma2_rn(make_float2(ea[i], ea[i + 1]), make_float2(t[i], t[i + 1]), q[(i / 2) & 3]);
+    return ((q[0].x + q[0].y) + (q[1].x + q[1].y)) + ((q[2].x + q[2].y) + (q[3].x + q[3].y));
+}
+
 template <int NA, bool ROOT>
-__device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const R2Step &st,
+__device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const SumStep &st,
                                            const float (&ear)[NA], float shift, uint32_t lane_base,
                                            uint32_t out_col, uint32_t col_root, uint32_t &tp,
                                            Prof &pf) {
     static_assert(NA % 4 == 0, "region width");
+    constexpr int PB = NA >= 80 ? 1 : 80 / NA;  // sums per TMEM batch
     const float *ks = p.fparams + st.blk_off;
-    auto fin = [&](int s, float a) {
-        const float val = shift + lg2(a) - __ldg(ks + s);
+    auto fin = [&](int s, float a, float k) {
+        const float val = shift + lg2(a) - k;
         if constexpr (ROOT) {
             const uint32_t c = col_root + (uint32_t)__ldg(p.root_map + s);
             float r;
@@ -642,7 +699,8 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
             tmem_st1(lane_base + out_col + s, val);
         }
     };
-    for (int gi = 0; gi < st.n_groups; ++gi) {
+    const int G = st.n_groups;
+    for (int gi = 0; gi < G; ++gi) {
         const int b = gi & 1;
         const GroupInfo gr = group_info(st, gi);
         pf.mark(3);
@@ -651,39 +709,32 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         tc_fence_after();
         const uint32_t acc = lane_base + (b ? (uint32_t)R2_COLS_A : 0u);
         const int ns = gr.ns;
-        // load units of U <= 24 columns (half a sum when NA > 24), two buffers
-        constexpr int U = NA > 24 ? NA / 2 : NA;
-        float b0[U], b1[U];
-        if (ns > 0) {
-            ld_unit_any<U>(acc, b0);
+        // batches of PB sums (one tcgen05.ld of PB * NA <= 80 columns, one
+        // wait): the sums' dot products are independent chains the scheduler
+        // interleaves (a lone warp's per-sum chain -- FFMA2s, reduction, lg2,
+        // subtract, store -- measured ~190 cycles; scripts/micro/epi_sum.cu)
+        for (int sl = 0; sl < ns; sl += PB) {
+            float t[PB * NA], kv[PB];
+            ld_cols<PB * NA>(acc + (uint32_t)(sl * NA), t);
+#pragma unroll
+            for (int k = 0; k < PB; ++k)  // the sums' scale exponents, in flight with the TMEM batch
+                kv[k] = sl + k < ns ? __ldg(ks + gr.s0 + sl + k) : 0.f;
             tmem_wait_ld();
-        }
-        if constexpr (NA > 24) {
-            for (int sl = 0; sl < ns; ++sl) {
-                const uint32_t row = acc + (uint32_t)(sl * NA);
-                ld_unit_any<U>(row + U, b1);              // second half of this sum
-                float a = dot_part<U>(ear, 0, b0);
-                tmem_wait_ld();
-                if (sl + 1 < ns) ld_unit_any<U>(row + NA, b0);  // first half of the next
-                a += dot_part<U>(ear, U, b1);
-                fin(gr.s0 + sl, a);
-                if (sl + 1 < ns) tmem_wait_ld();
+            if (sl + PB >= ns) {
+                tc_fence_before();
+                bar_arrive(sm.bar(B_T_EMPTY + b));  // all of this group's columns are in registers
             }
-        } else {
-            for (int sl = 0; sl < ns; sl += 2) {
-                const uint32_t row = acc + (uint32_t)(sl * NA);
-                if (sl + 1 < ns) ld_unit_any<U>(row + NA, b1);
-                fin(gr.s0 + sl, dot_part<U>(ear, 0, b0));
-                if (sl + 1 < ns) {
-                    tmem_wait_ld();
-                    if (sl + 2 < ns) ld_unit_any<U>(row + 2 * NA, b0);
-                    fin(gr.s0 + sl + 1, dot_part<U>(ear, 0, b1));
-                    if (sl + 2 < ns) tmem_wait_ld();
-                }
-            }
+            float val[PB];
+#pragma unroll
+            for (int k = 0; k < PB; ++k) val[k] = dot4(ear, t + k * NA);
+#pragma unroll
+            for (int k = 0; k < PB; ++k)
+                if (sl + k < ns) fin(gr.s0 + sl + k, val[k], kv[k]);
         }
-        tc_fence_before();
-        bar_arrive(sm.bar(B_T_EMPTY + b));
+        if (ns == 0) {
+            tc_fence_before();
+            bar_arrive(sm.bar(B_T_EMPTY + b));
+        }
         if (b) ++tp;
     }
 }
@@ -704,8 +755,10 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         for (int c = 0; c < p.C; ++c) tmem_st1(lane_base + col_root + c, -CUDART_INF_F);
         tmem_wait_st();
+        SumStep nx = load_sum_step(p.steps, sum_steps, 0);
         for (int si = 0; si < n_sum; ++si) {
-            const R2Step &es = p.steps[__ldg(sum_steps + si)];
+            const SumStep es = nx;
+            if (si + 1 < n_sum) nx = load_sum_step(p.steps, sum_steps, si + 1);
             pf.mark(5);
             const uint32_t out_col = col_slots + (uint32_t)((es.slot_out - 1) * S);
             if (es.type == 1) {
@@ -770,6 +823,7 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
         const int64_t row = tile * RT + m;
         int best = -1;
         float bv = -CUDART_INF_F;
+        bool cert = true;
         for (int c = 0; c < p.C; ++c) {
             float r;
             tmem_ld1(lane_base + col_root + c, r);
@@ -780,8 +834,14 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 best = c;
                 bv = v;
             }
+            // single-pass error bound inside the tolerance? (NaN / inf
+            // results are the same in both precisions)
+            const float av = fabsf(v);
+            if (av < CUDART_INF_F && !(p.cert_err <= p.cert_tol * fmaxf(1.f, av - p.cert_err)))
+                cert = false;
         }
         if (row < p.n && p.argmax) p.argmax[row] = best;
+        if (row < p.n && p.flag_count && !cert) p.flag_idx[atomicAdd(p.flag_count, 1)] = p.row0 + row;
         pf.mark(4);
     }
 }
@@ -835,8 +895,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
 
-    if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 40;");
-    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 216;");
+    if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 200;");
     if (warp < W_EPI0) {
         leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
     } else if (warp < W_PROD) {

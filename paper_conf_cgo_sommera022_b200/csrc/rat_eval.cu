@@ -311,6 +311,10 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
     constexpr int SPS = NTH == 512 ? 1 : EPI_SPS;  // sums per TMEM wait in the epilogue
     extern __shared__ __align__(1024) uint8_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    // samples: from the launch, or counted on the device (certification fallback)
+    int64_t n = p.n;
+    if (p.n_count) n = max((int64_t)0, min(n, (int64_t)*p.n_count - p.n_off));
+    if (n <= 0) return;
     // ---- shared-memory carve-up (mirrored by rat_smem_bytes) ----
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);  // 0 mma, 1-3 w, 4/5 x
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + 64);
@@ -398,7 +402,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
         }
     };
 
-    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    const int64_t n_tiles = (n + RT - 1) / RT;
     // optional profiling: cycles per phase measured by thread 0
     unsigned long long pc_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     unsigned long long t_mark = clock64();
@@ -608,7 +612,7 @@ __global__ void __launch_bounds__(NTH, 1) rat_eval_kernel(const RParams p) {
         // ---------------- outputs -------------------------------------------
         if (tid < RT) {
             const int64_t srow = base + tid;
-            if (srow < p.n) {
+            if (srow < n) {
                 int best = -1;
                 float bv = -CUDART_INF_F;
                 for (int c = 0; c < p.C; ++c) {
@@ -649,6 +653,57 @@ __global__ void transpose_x_kernel(const float *__restrict__ x, int64_t n, int64
         const int64_t f = f0 + k, s = s0 + tx;
         if (f < F && s < rows_pad) xT[f * ldT + s] = t[tx][k];
     }
+}
+
+// certification fallback: xT[f][k] = x[idx[off + k]][f] for the flagged rows
+// k < min(*count - off, cap) (zero for the rest of each 32-row block)
+__global__ void gather_transpose_kernel(const float *__restrict__ x, int64_t ld, int F,
+                                        const int64_t *__restrict__ idx, const int32_t *count,
+                                        int64_t off, int64_t cap, float *__restrict__ xT,
+                                        int64_t ldT) {
+    const int64_t m = max((int64_t)0, min(cap, (int64_t)*count - off));
+    const int64_t s0 = (int64_t)blockIdx.x * 32, f0 = (int64_t)blockIdx.y * 32;
+    if (s0 >= m) return;
+    __shared__ float t[32][33];
+    const int tx = threadIdx.x, ty = threadIdx.y;
+    for (int k = ty; k < 32; k += 8) {
+        const int64_t s = s0 + k, f = f0 + tx;
+        t[k][tx] = (s < m && f < F) ? __ldg(x + __ldg(idx + off + s) * ld + f) : 0.f;
+    }
+    __syncthreads();
+    for (int k = ty; k < 32; k += 8) {
+        const int64_t f = f0 + k, s = s0 + tx;
+        if (f < F) xT[f * ldT + s] = t[tx][k];
+    }
+}
+
+// certification fallback: out[idx[off + k]] = tmp[k] (and argmax) for the flagged rows
+__global__ void scatter_rows_kernel(const float *__restrict__ tmp, const int32_t *__restrict__ am_tmp,
+                                    const int64_t *__restrict__ idx, const int32_t *count,
+                                    int64_t off, int64_t cap, int C, float *__restrict__ out,
+                                    int32_t *__restrict__ am) {
+    const int64_t m = max((int64_t)0, min(cap, (int64_t)*count - off));
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < m;
+         k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = __ldg(idx + off + k);
+        for (int c = 0; c < C; ++c) out[r * C + c] = tmp[k * C + c];
+        if (am) am[r] = am_tmp[k];
+    }
+}
+
+cudaError_t cert_gather_launch(const float *x, int64_t ld, int F, const int64_t *idx,
+                               const int32_t *count, int64_t off, int64_t cap, float *xT,
+                               int64_t ldT, cudaStream_t st) {
+    dim3 grid((unsigned)((cap + 31) / 32), (unsigned)((F + 31) / 32));
+    gather_transpose_kernel<<<grid, dim3(32, 8), 0, st>>>(x, ld, F, idx, count, off, cap, xT, ldT);
+    return cudaGetLastError();
+}
+
+cudaError_t cert_scatter_launch(const float *tmp, const int32_t *am_tmp, const int64_t *idx,
+                                const int32_t *count, int64_t off, int64_t cap, int C, float *out,
+                                int32_t *am, cudaStream_t st) {
+    scatter_rows_kernel<<<148, 256, 0, st>>>(tmp, am_tmp, idx, count, off, cap, C, out, am);
+    return cudaGetLastError();
 }
 
 size_t rat_smem_bytes(int smem_floats, int C, int max_na, int max_kpad, int max_ngroup,

@@ -3,7 +3,9 @@ import os
 import sys
 import time
 
-os.environ["SPNB_PROFILE"] = "1"
+os.environ.setdefault("SPNB_PROFILE", "1")   # SPNB_PROFILE=0 for clean ncu captures
+if os.environ["SPNB_PROFILE"] == "0":
+    del os.environ["SPNB_PROFILE"]
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 

@@ -31,19 +31,20 @@ if what in ("parity", "all"):
         x, _ = ancestral_sample(g, 1000, 3)
         ref, _ = oracle_eval(g, x)
         refm, _ = oracle_eval(g, nan_mask(x, 0.2, 4), marginal=True)
-        for prec in (2, 1):
+        for prec in (0, 1):
             P = spnb.Plan(spnb.Graph(g), layered_path=2, tc_precision=prec, layered_kernel=2)
             xd = torch.from_numpy(x).cuda()
             out, am = P.infer(xd)
             outm, _ = P.infer(torch.from_numpy(nan_mask(x, 0.2, 4)).cuda(), marginal=True)
             torch.cuda.synchronize()
             print("shape", shape, "prec", prec, "info", P.info()["layered_kernel"],
+                  "cert", P.info()["certified"], round(P.info()["cert_err"], 5),
                   "err", err(out.cpu().numpy(), ref), "marg err", err(outm.cpu().numpy(), refm),
                   flush=True)
     g = config_graph("C4")
     x, _ = ancestral_sample(g, 300, 4002)
     ref, _ = oracle_eval(g, x)
-    for prec in (2, 1):
+    for prec in (0, 1):
         P = spnb.Plan(spnb.Graph(g), tc_precision=prec, layered_kernel=2)
         out, am = P.infer(torch.from_numpy(x).cuda())
         torch.cuda.synchronize()
@@ -55,7 +56,7 @@ if what in ("time", "all"):
         g = config_graph(cfg)
         G = spnb.Graph(g)
         xd = bench.device_uniform(n, g.n_features, 4002, 0, torch.device("cuda"))
-        for kern, prec in ((2, 1), (2, 2), (1, 2)):
+        for kern, prec in ((2, 0), (2, 1), (1, 2)):
             P = spnb.Plan(G, tc_precision=prec, layered_kernel=kern)
             out, am = P.infer(xd)
             torch.cuda.synchronize()

@@ -81,6 +81,30 @@ def test_c1_toy_100k_joint_and_marginal():
     _parity(g, nan_mask(x, 0.2, 1002), marginal=True)
 
 
+@pytest.mark.parametrize("space", [1, 2])
+def test_value_space_selection(space):
+    """f4: the toy and tiny discrete SPNs in log2 space and in
+    linear fp32 space through the compiled path; auto picks linear for them
+    and log2 for Gaussian SPNs; linear is refused for a Gaussian SPN."""
+    import itertools
+    g = toy_spn()
+    x = toy_data(200_000, seed=1003)
+    err, P = _parity(g, x, value_space=space)
+    assert P.info()["path"] == 2 and P.info()["value_space"] == space
+    _parity(g, nan_mask(x, 0.2, 1004), marginal=True, value_space=space)
+    for seed in range(3):
+        gd = tiny_discrete_spn(seed)
+        doms = gd.meta["domains"]
+        xd = np.array(list(itertools.product(*[range(-1, k + 1) for k in doms])), np.float32)
+        _parity(gd, xd, value_space=space)
+        _parity(gd, nan_mask(xd, 0.3, seed), marginal=True, value_space=space)
+    if space == 2:
+        assert spnb.Plan(spnb.Graph(toy_spn())).info()["value_space"] == 2       # auto
+        assert spnb.Plan(spnb.Graph(speaker_spn(2001))).info()["value_space"] == 1
+        with pytest.raises(spnb.SPNError):
+            spnb.Plan(spnb.Graph(speaker_spn(2001)), value_space=2)
+
+
 # ----------------------------------------------------------------- config 2
 @pytest.mark.parametrize("n", [1, 31, 128, 129, 1000, 4099])
 def test_c2_ragged_sizes(n):

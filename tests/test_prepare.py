@@ -299,3 +299,25 @@ def test_layered2_rejects_outside_constraints():
     assert p is None and "multiple of 8" in why
     p, why = spnb.build_layered2(spnb.Graph(speaker_spn(2001)))
     assert p is None and why
+
+
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (96, 4, 2, 20, 40, 10)])
+def test_layered2_single_pass_error_bound_holds(shape):
+    """The certification bound of the single f16 pass (layered.h
+    Rat2Plan::tc_err_1pass) is an upper bound of the emulated single pass's
+    deviation from the hi/lo (exact-contraction) emulation, on ancestral and
+    adversarial (far out-of-distribution) inputs."""
+    from spn_inputs import rat_spn
+    from tests.layered2_emulator import emulate_layered2
+    F, D, R, S, I, C = shape
+    g = rat_spn(9, F=F, D=D, R=R, S=S, I=I, C=C)
+    plan, why = spnb.build_layered2(spnb.Graph(g))
+    E = plan["tc_err_1pass"]
+    assert 0 < E < 0.1, E
+    x, _ = ancestral_sample(g, 200, 5)
+    xo = np.random.default_rng(6).uniform(-3, 4, size=(200, F)).astype(np.float32)
+    for xx in (x, xo):
+        e1 = emulate_layered2(plan, xx, prec=1)
+        e3 = emulate_layered2(plan, xx, prec=3)
+        fin = np.isfinite(e3)
+        assert np.abs(e1 - e3)[fin].max() <= E, (np.abs(e1 - e3)[fin].max(), E)

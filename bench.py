@@ -255,7 +255,10 @@ def launches_per_step(info: dict, n: int, want_am: bool) -> int:
         return info["n_tasks"] + (1 if want_am and info["n_tasks"] > 1 else 0)
     if info["path"] == 1:   # per transposed chunk: transpose + layered kernel
         chunk = max(1, info["chunk_samples"])
-        return 2 * ((n + chunk - 1) // chunk)
+        rounds = (n + chunk - 1) // chunk
+        # certified single pass: per round a gather, a hi/lo recompute and a
+        # scatter (no-ops when every sample is certified)
+        return 2 * rounds + (3 * rounds if info.get("certified") else 0)
     return 1
 
 
@@ -316,9 +319,10 @@ def run_ours(args):
 
     def collect():
         # equal shards (10M / {1,2,4,8}): one all_gather_into_tensor each (NCCL)
-        dist.all_gather_into_tensor(full_out, out)
+        from paper_conf_cgo_sommera022_b200.parallel import gather_into
+        gather_into(full_out, out)
         if want_am:
-            dist.all_gather_into_tensor(full_am, am)
+            gather_into(full_am, am)
 
     for _ in range(max(3, args.warmup)):
         flush.fill_(1)

@@ -485,6 +485,9 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
         // chunk sized to ~32 MB of features: big enough to amortise launches,
         // small enough to overlap H2D / kernel / D2H across the two streams
         P.host_chunk = std::max<int64_t>(4096, ((int64_t)(32 << 20) / (4 * P.F)) & ~int64_t(4095));
+        // the layered path launches one persistent wave per transposed chunk:
+        // host chunks of that size keep every SM busy (C5: 151,552 samples)
+        if (P.path == 1) P.host_chunk = std::max<int64_t>(P.host_chunk, P.chunk);
         for (int i = 0; i < 2; ++i) {
             if ((e = cudaStreamCreateWithFlags(&P.hs[i], cudaStreamNonBlocking)) != cudaSuccess)
                 return cuda_err(e, "cudaStreamCreate");

@@ -38,12 +38,15 @@ namespace spnb {
 namespace r2 {
 
 constexpr int RT = 128;           // samples per tile = UMMA M = TMEM lanes
-// 16 warps = 4 warpgroups: leaf group 0, leaf group 1, epilogue, and
-// {leaf producer, MMA, weight producer, idle}.  setmaxnreg moves registers
-// from the last warpgroup (56 each) to the epilogue (200 each); the leaf
-// warpgroups keep the launch's 128: 2*128 + 200 + 56 = 512 per SMSP lane.
+// 16 warps = 4 warpgroups: leaf, epilogue (accumulator A), epilogue
+// (accumulator B), {leaf producer, MMA, weight producer, idle}.  setmaxnreg
+// moves registers from the last warpgroup (56 each) to the epilogue ones
+// (160 each); the leaf warpgroup keeps the launch's 128: 128 + 2*160 + 56
+// = 504 <= 512 per SMSP lane.
 constexpr int NTHREADS = 16 * 32;
-constexpr int W_EPI0 = 8, W_PROD = 12, W_MMA = 13, W_WPROD = 14;
+constexpr int NLG = 1;            // leaf groups of 4 warps (each evaluates whole regions)
+constexpr int W_EPI0 = 4 * NLG;   // epilogue warps: two per TMEM lane quarter
+constexpr int W_PROD = 12, W_MMA = 13, W_WPROD = 14;
 constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
 // TMEM accumulators: A = columns [0, R2_COLS_A), B = [R2_COLS_A, +R2_COLS_B);
 // the groups of a step alternate A, B (layered.h R2Step)
@@ -189,9 +192,11 @@ __device__ __forceinline__ void tmem_wait_st() {
 __device__ __forceinline__ uint32_t img_off(int row, int k) {
     return (uint32_t)((k >> 3) * (RT * 16) + (row >> 3) * 128 + (row & 7) * 16 + (k & 7) * 2);
 }
+// two floats -> packed f16x2 with one cvt.rn.f16x2.f32 (a in the low half)
 __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
-    const __half ha = __float2half_rn(a), hb = __float2half_rn(b);
-    return (uint32_t)__half_as_ushort(ha) | ((uint32_t)__half_as_ushort(hb) << 16);
+    uint32_t r;
+    asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+    return r;
 }
 // hi/lo split of a pair: hi = f16(v), lo = f16(v - hi)
 __device__ __forceinline__ void split_h2(float a, float b, uint32_t &hi, uint32_t &lo) {
@@ -281,20 +286,29 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
     const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi): c_v = log2(a) + K0
     const float4 *ab4 = reinterpret_cast<const float4 *>(prm + 2 * d0);
     const int vstride = I / 2;  // float4 per variable
-#pragma unroll 4
+    // operands of variable v + 1 are loaded while v's FFMA2s run (a leaf warp
+    // is alone on its SMSP: the shared-memory latency must come from ILP)
+    float4 x4 = *reinterpret_cast<const float4 *>(xs + m0);
+    float4 qn[DPB / 2];
+#pragma unroll
+    for (int k = 0; k < DPB / 2; ++k) qn[k] = ab4[k];
     for (int v = 0; v < V; ++v) {
-        const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + m0);
         float2 q[DPB];
 #pragma unroll
         for (int k = 0; k < DPB / 2; ++k) {
-            const float4 t = ab4[v * vstride + k];
-            q[2 * k] = make_float2(t.x, t.y);
-            q[2 * k + 1] = make_float2(t.z, t.w);
+            q[2 * k] = make_float2(qn[k].x, qn[k].y);
+            q[2 * k + 1] = make_float2(qn[k].z, qn[k].w);
+        }
+        const float4 xc = x4;
+        if (v + 1 < V) {
+            x4 = *reinterpret_cast<const float4 *>(xs + (v + 1) * RT + m0);
+#pragma unroll
+            for (int k = 0; k < DPB / 2; ++k) qn[k] = ab4[(v + 1) * vstride + k];
         }
         bool anynan = false;
-        if constexpr (MARG) anynan = (x4.x != x4.x) | (x4.y != x4.y) | (x4.z != x4.z) | (x4.w != x4.w);
+        if constexpr (MARG) anynan = (xc.x != xc.x) | (xc.y != xc.y) | (xc.z != xc.z) | (xc.w != xc.w);
         if (MARG && anynan) {
-            const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
+            const float xv[4] = {xc.x, xc.y, xc.z, xc.w};
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float cc = lg2(q[d].x) + K0;
@@ -306,7 +320,7 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
                 }
             }
         } else {
-            const float2 x01 = make_float2(x4.x, x4.y), x23 = make_float2(x4.z, x4.w);
+            const float2 x01 = make_float2(xc.x, xc.y), x23 = make_float2(xc.z, xc.w);
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float2 a2 = make_float2(q[d].x, q[d].x), nb2 = make_float2(-q[d].y, -q[d].y);
@@ -325,16 +339,17 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
 template <int DPB, bool MARG>
 __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
                           int n_leaf, int warp, int lane) {
-    const int g = warp >> 2, gw = warp & 3;
+    const int g = warp >> 2, gw = warp & 3;  // leaf group, warp in group (= lane quarter)
     const int q = lane >> 2, b = lane & 3;
     const int m0 = gw * 32 + q * 4, d0 = b * DPB;
     const int I = p.I;
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    uint32_t li = (uint32_t)g;  // global leaf-region counter of this group (step 2)
-    uint32_t j = 0;             // this group's region count = bottom-partition counter
+    uint32_t li = (uint32_t)g;  // global leaf-region counter (step NLG); even: A side, odd: B side
     Prof pf(sm.prof(0), p.prof != nullptr);  // 0 wait input, 1 compute, 2 shifts, 3 wait output slot, 4 exps + write
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-        for (int l = g; l < n_leaf; l += 2, li += 2, ++j) {
+        for (int l = g; l < n_leaf; l += NLG, li += NLG) {
+            const bool side_b = (l & 1) != 0;  // leaf regions alternate left (A) / right (B)
+            const uint32_t j = li >> 1;         // bottom partition
             const R2Step &st = p.steps[leaf_steps[l]];
             const int s = (int)(li % (uint32_t)p.n_in);
             bar_wait(sm.bar(B_IN_FULL + s), (li / (uint32_t)p.n_in) & 1u);
@@ -361,9 +376,9 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
             pf.mark(2);
             // both sides wait for the A slot (it also carries hb)
             bar_wait(sm.bar(B_A_EMPTY + ab), ph ^ 1u);
-            if (g == 1) bar_wait(sm.bar(B_B_EMPTY + ab), ph ^ 1u);
+            if (side_b) bar_wait(sm.bar(B_B_EMPTY + ab), ph ^ 1u);
             pf.mark(3);
-            if (g == 0) {
+            if (!side_b) {
                 float *ea = sm.ea(ab);
 #pragma unroll
                 for (int d = 0; d < DPB; ++d) {
@@ -683,7 +698,7 @@ template <int NA, bool ROOT>
 __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const SumStep &st,
                                            const float (&ear)[NA], float shift, uint32_t lane_base,
                                            uint32_t out_col, uint32_t col_root, uint32_t &tp,
-                                           Prof &pf) {
+                                           Prof &pf, int h) {
     static_assert(NA % 4 == 0, "region width");
     constexpr int PB = NA >= 80 ? 1 : 80 / NA;  // sums per TMEM batch
     const float *ks = p.fparams + st.blk_off;
@@ -700,7 +715,7 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         }
     };
     const int G = st.n_groups;
-    for (int gi = 0; gi < G; ++gi) {
+    for (int gi = h; gi < G; gi += 2) {  // this warp's accumulator: groups of parity h
         const int b = gi & 1;
         const GroupInfo gr = group_info(st, gi);
         pf.mark(3);
@@ -735,7 +750,7 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
             tc_fence_before();
             bar_arrive(sm.bar(B_T_EMPTY + b));
         }
-        if (b) ++tp;
+        ++tp;
     }
 }
 
@@ -743,9 +758,18 @@ template <int I, int S, bool MARG>
 __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps,
                               int n_sum, uint32_t tmem, int warp, int lane) {
     const int qd = warp & 3;
+    const int h = (warp - W_EPI0) >> 2;  // 0: groups in accumulator A, 1: in accumulator B
     const int m = qd * 32 + lane;
     const uint32_t lane_base = tmem + ((uint32_t)(qd * 32) << 16);
     const uint32_t col_slots = (uint32_t)(R2_COLS_A + R2_COLS_B);
+    // the two warps of a lane quarter exchange activation slots / root
+    // columns through TMEM: wait for own stores, then a 64-thread barrier
+    auto pair_sync = [&]() {
+        tmem_wait_st();
+        tc_fence_before();
+        asm volatile("bar.sync %0, 64;" ::"r"(1 + qd) : "memory");
+        tc_fence_after();
+    };
     const uint32_t col_root = col_slots + (uint32_t)(p.D * S);
     const int64_t n_tiles = (p.n + RT - 1) / RT;
     uint32_t kb = 0, ku = 0, tp = 0;
@@ -753,8 +777,9 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
     constexpr int SU = S > 0 ? S : 4;
     Prof pf(sm.prof(1), p.prof != nullptr);  // 0 wait leaf outputs, 1 UP phase 1, 2 wait TMEM full, 3 sums, 4 tile I/O, 5 step setup
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-        for (int c = 0; c < p.C; ++c) tmem_st1(lane_base + col_root + c, -CUDART_INF_F);
-        tmem_wait_st();
+        if (h == 0)
+            for (int c = 0; c < p.C; ++c) tmem_st1(lane_base + col_root + c, -CUDART_INF_F);
+        pair_sync();
         SumStep nx = load_sum_step(p.steps, sum_steps, 0);
         for (int si = 0; si < n_sum; ++si) {
             const SumStep es = nx;
@@ -775,11 +800,12 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 const float shift = sm.ha(ab)[m] + sm.hb(ab)[m];
                 bar_arrive(sm.bar(B_A_EMPTY + ab));
                 ++kb;
-                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
-                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
+                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
             } else {
                 // UP: children in activation slots; B side -> f16 image, A side -> registers
                 float vb[SU], ear[SU];
+                pair_sync();  // the children's sums were written by both warps
                 ld_unit_any<SU>(lane_base + col_slots + (uint32_t)((es.slot_b - 1) * S), vb);
                 ld_unit_any<SU>(lane_base + col_slots + (uint32_t)((es.slot_a - 1) * S), ear);
                 tmem_wait_ld();
@@ -789,36 +815,40 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                     hb = maxnan(hb, vb[i]);
                     ha = maxnan(ha, ear[i]);
                 }
-                bar_wait(sm.bar(B_U_EMPTY), (ku & 1u) ^ 1u);
-                uint8_t *img = sm.uimg();
-                const float hc = fmaxf(hb, -1e30f) - EB_SHIFT;
+                if (h == 0) {  // one warp of the pair writes the B-side operand image
+                    bar_wait(sm.bar(B_U_EMPTY), (ku & 1u) ^ 1u);
+                    uint8_t *img = sm.uimg();
+                    const float hc = fmaxf(hb, -1e30f) - EB_SHIFT;
 #pragma unroll
-                for (int i = 0; i < SU; i += 2) {
-                    const float e0 = ex2(vb[i] - hc), e1 = i + 1 < SU ? ex2(vb[i + 1] - hc) : 0.f;
-                    const uint32_t o = img_off(m, i);
-                    if (p.prec == 3) {
-                        uint32_t hi, lo;
-                        split_h2(e0, e1, hi, lo);
-                        *reinterpret_cast<uint32_t *>(img + o) = hi;
-                        *reinterpret_cast<uint32_t *>(img + part_u + o) = lo;
-                    } else {
-                        *reinterpret_cast<uint32_t *>(img + o) = pack_h2(e0, e1);
+                    for (int i = 0; i < SU; i += 2) {
+                        const float e0 = ex2(vb[i] - hc), e1 = i + 1 < SU ? ex2(vb[i + 1] - hc) : 0.f;
+                        const uint32_t o = img_off(m, i);
+                        if (p.prec == 3) {
+                            uint32_t hi, lo;
+                            split_h2(e0, e1, hi, lo);
+                            *reinterpret_cast<uint32_t *>(img + o) = hi;
+                            *reinterpret_cast<uint32_t *>(img + part_u + o) = lo;
+                        } else {
+                            *reinterpret_cast<uint32_t *>(img + o) = pack_h2(e0, e1);
+                        }
                     }
+                    fence_async_smem();
+                    bar_arrive(sm.bar(B_U_FULL));
                 }
-                fence_async_smem();
-                bar_arrive(sm.bar(B_U_FULL));
                 ++ku;
                 const float hac = fmaxf(ha, -1e30f);
 #pragma unroll
                 for (int i = 0; i < SU; ++i) ear[i] = ex2(ear[i] - hac);
                 const float shift = ha + hb - EB_SHIFT;
                 pf.mark(1);
-                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
-                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf);
+                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
             }
             tmem_wait_st();
         }
         pf.mark(3);
+        pair_sync();  // root columns were accumulated by both warps
+        if (h == 1) continue;
         // ---- outputs of the tile (the TMEM loads stay warp-converged)
         const int64_t row = tile * RT + m;
         int best = -1;
@@ -873,7 +903,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         for (int i = 0; i < 2; ++i) {
             bar_init(sm.bar(B_A_FULL + i), 128);
-            bar_init(sm.bar(B_A_EMPTY + i), 128);
+            bar_init(sm.bar(B_A_EMPTY + i), 256);  // both epilogue warps of each quarter
             bar_init(sm.bar(B_B_FULL + i), 128);
             bar_init(sm.bar(B_B_EMPTY + i), 1);
         }
@@ -896,7 +926,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const uint32_t tmem = *tmem_slot;
 
     if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
-    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 200;");
+    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 160;");
     if (warp < W_EPI0) {
         leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
     } else if (warp < W_PROD) {

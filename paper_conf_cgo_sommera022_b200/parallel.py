@@ -45,6 +45,18 @@ def gather_results(local: torch.Tensor, n_total: int, group=None) -> torch.Tenso
     return torch.cat(parts, dim=0)
 
 
+def gather_into(full: torch.Tensor, local: torch.Tensor, group=None) -> torch.Tensor:
+    """Gather equal shards ([n/P, ...] per rank) into a preallocated
+    [n, ...] tensor on every rank with one all_gather_into_tensor (NCCL over
+    NVLink on GPUs).  The bench calls this inside the timed step for the
+    strong-scaling config (10M samples split evenly over 1/2/4/8 ranks)."""
+    world = dist.get_world_size(group)
+    if full.shape[0] != local.shape[0] * world or full.shape[1:] != local.shape[1:]:
+        raise ValueError(f"gather_into: full {tuple(full.shape)} != {world} x {tuple(local.shape)}")
+    dist.all_gather_into_tensor(full, local.contiguous(), group=group)
+    return full
+
+
 def sharded_infer(plan, x_full: torch.Tensor, marginal: bool = False, gather: bool = True,
                   group=None):
     """Evaluate this rank's shard of x_full with `plan` (a Plan on this

@@ -10,7 +10,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 from paper_conf_cgo_sommera022_b200.parallel import (shard_range, shard_sizes, gather_results,
-                                                     sharded_infer)
+                                                     gather_into, sharded_infer)
 
 
 def test_shard_ranges_cover_exactly_once():
@@ -54,6 +54,16 @@ def _worker(rank, world, port, n, q):
         loc = torch.arange(lo, hi, dtype=torch.int64)
         full = gather_results(loc, n)
         ok = ok and torch.equal(full, torch.arange(n, dtype=torch.int64))
+        # the bench's strong-scaling gather: equal shards into a preallocated buffer
+        m = n - n % world
+        a, b = shard_range(m, rank, world)
+        logp = torch.stack([torch.arange(a, b, dtype=torch.float32)] * 3, dim=1)
+        buf = torch.empty((m, 3), dtype=torch.float32)
+        gather_into(buf, logp)
+        ok = ok and torch.equal(buf[:, 0], torch.arange(m, dtype=torch.float32))
+        am_buf = torch.empty((m,), dtype=torch.int32)
+        gather_into(am_buf, torch.arange(a, b, dtype=torch.int32))
+        ok = ok and torch.equal(am_buf, torch.arange(m, dtype=torch.int32))
         q.put((rank, bool(ok)))
     finally:
         dist.destroy_process_group()

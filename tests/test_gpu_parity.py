@@ -252,7 +252,7 @@ def test_layered_rat_small_matches_oracle(shape, kernel):
     F, D, R, S, I, C = shape
     g = rat_spn(11, F=F, D=D, R=R, S=S, I=I, C=C)
     x, _ = ancestral_sample(g, 1000, 12)
-    for prec in ((2, 1) if kernel == 2 else (2,)):
+    for prec in ((0, 1) if kernel == 2 else (2,)):
         err, P = _parity(g, x, layered_path=2, tc_precision=prec, layered_kernel=kernel)
         assert P.info()["path"] == 1 and P.info()["layered_kernel"] == kernel
         _parity(g, nan_mask(x, 0.2, 13), marginal=True, layered_path=2, tc_precision=prec,

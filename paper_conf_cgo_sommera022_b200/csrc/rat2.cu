@@ -40,13 +40,31 @@ namespace r2 {
 constexpr int RT = 128;           // samples per tile = UMMA M = TMEM lanes
 // 16 warps = 4 warpgroups: leaf, epilogue (accumulator A), epilogue
 // (accumulator B), {leaf producer, MMA, weight producer, idle}.  setmaxnreg
-// moves registers from the last warpgroup (56 each) to the epilogue ones
-// (160 each); the leaf warpgroup keeps the launch's 128: 128 + 2*160 + 56
-// = 504 <= 512 per SMSP lane.
-constexpr int NTHREADS = 16 * 32;
-constexpr int NLG = 1;            // leaf groups of 4 warps (each evaluates whole regions)
+// moves registers from the last warpgroup (56 each) to the other three
+// (152 each): 3*152 + 56 = 512 per SMSP lane.
+#ifndef R2_WARPS
+#define R2_WARPS 16
+#endif
+#if R2_WARPS == 20
+// 20 warps: two leaf groups (left / right regions), 8 epilogue warps, producers
+// setmaxnreg moves registers only within the CTA's launch allocation
+// (640 threads x 96): 8*96 + 8*120 + 4*40 = 1888 <= 20*96 per lane
+constexpr int NLG = 2, EPI_COLS = 40;
+constexpr int REG_LEAF = 96, REG_EPI = 120, REG_PROD = 40;
+#else
+// launch allocation 512 threads x 128: 4*152 + 8*152 + 4*56 = 2048 = 16*128 per lane
+constexpr int NLG = 1, EPI_COLS = 80;
+constexpr int REG_LEAF = 152, REG_EPI = 152, REG_PROD = 56;
+#endif
+constexpr int NTHREADS = (4 * NLG + 12) * 32;
+// registers per thread of the launch (65536 / NTHREADS rounded down to 8):
+// the pool setmaxnreg redistributes; rat2_launch refuses a build whose
+// register count differs (an unbalanced budget would block setmaxnreg.inc)
+constexpr int LAUNCH_REGS = (65536 / NTHREADS) / 8 * 8;
+static_assert(4 * NLG * REG_LEAF + 8 * REG_EPI + 4 * REG_PROD <= (4 * NLG + 12) * LAUNCH_REGS,
+              "setmaxnreg budget exceeds the launch allocation");
 constexpr int W_EPI0 = 4 * NLG;   // epilogue warps: two per TMEM lane quarter
-constexpr int W_PROD = 12, W_MMA = 13, W_WPROD = 14;
+constexpr int W_PROD = W_EPI0 + 8, W_MMA = W_PROD + 1, W_WPROD = W_PROD + 2;
 constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
 // TMEM accumulators: A = columns [0, R2_COLS_A), B = [R2_COLS_A, +R2_COLS_B);
 // the groups of a step alternate A, B (layered.h R2Step)
@@ -286,29 +304,20 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
     const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi): c_v = log2(a) + K0
     const float4 *ab4 = reinterpret_cast<const float4 *>(prm + 2 * d0);
     const int vstride = I / 2;  // float4 per variable
-    // operands of variable v + 1 are loaded while v's FFMA2s run (a leaf warp
-    // is alone on its SMSP: the shared-memory latency must come from ILP)
-    float4 x4 = *reinterpret_cast<const float4 *>(xs + m0);
-    float4 qn[DPB / 2];
-#pragma unroll
-    for (int k = 0; k < DPB / 2; ++k) qn[k] = ab4[k];
+#pragma unroll 4
     for (int v = 0; v < V; ++v) {
+        const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + m0);
         float2 q[DPB];
 #pragma unroll
         for (int k = 0; k < DPB / 2; ++k) {
-            q[2 * k] = make_float2(qn[k].x, qn[k].y);
-            q[2 * k + 1] = make_float2(qn[k].z, qn[k].w);
-        }
-        const float4 xc = x4;
-        if (v + 1 < V) {
-            x4 = *reinterpret_cast<const float4 *>(xs + (v + 1) * RT + m0);
-#pragma unroll
-            for (int k = 0; k < DPB / 2; ++k) qn[k] = ab4[(v + 1) * vstride + k];
+            const float4 t = ab4[v * vstride + k];
+            q[2 * k] = make_float2(t.x, t.y);
+            q[2 * k + 1] = make_float2(t.z, t.w);
         }
         bool anynan = false;
-        if constexpr (MARG) anynan = (xc.x != xc.x) | (xc.y != xc.y) | (xc.z != xc.z) | (xc.w != xc.w);
+        if constexpr (MARG) anynan = (x4.x != x4.x) | (x4.y != x4.y) | (x4.z != x4.z) | (x4.w != x4.w);
         if (MARG && anynan) {
-            const float xv[4] = {xc.x, xc.y, xc.z, xc.w};
+            const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float cc = lg2(q[d].x) + K0;
@@ -320,7 +329,7 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
                 }
             }
         } else {
-            const float2 x01 = make_float2(xc.x, xc.y), x23 = make_float2(xc.z, xc.w);
+            const float2 x01 = make_float2(x4.x, x4.y), x23 = make_float2(x4.z, x4.w);
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float2 a2 = make_float2(q[d].x, q[d].x), nb2 = make_float2(-q[d].y, -q[d].y);
@@ -700,7 +709,7 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
                                            uint32_t out_col, uint32_t col_root, uint32_t &tp,
                                            Prof &pf, int h) {
     static_assert(NA % 4 == 0, "region width");
-    constexpr int PB = NA >= 80 ? 1 : 80 / NA;  // sums per TMEM batch
+    constexpr int PB = NA >= EPI_COLS ? 1 : EPI_COLS / NA;  // sums per TMEM batch
     const float *ks = p.fparams + st.blk_off;
     auto fin = [&](int s, float a, float k) {
         const float val = shift + lg2(a) - k;
@@ -925,8 +934,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
 
-    if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
-    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 160;");
+    // launch: 128 registers per thread (16 warps); leaf 152, epilogue 152,
+    // producers / MMA 56: 152 + 2 * 152 + 56 = 512 per SMSP lane
+    if (warp >= W_PROD) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(REG_PROD));
+    else if (warp >= W_EPI0) asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(REG_EPI));
+    else if (REG_LEAF > LAUNCH_REGS)
+        asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(REG_LEAF));
     if (warp < W_EPI0) {
         leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
     } else if (warp < W_PROD) {
@@ -998,7 +1011,11 @@ cudaError_t rat2_launch(const R2Params &p, const int32_t *leaf_steps, int n_leaf
     R2_CASE(8, 4) R2_CASE(16, 8) R2_CASE(40, 20) R2_CASE(32, 16) R2_CASE(16, 16) R2_CASE(48, 24)
 #undef R2_CASE
     if (!fn) return cudaErrorInvalidConfiguration;
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, fn);
+    if (e != cudaSuccess) return e;
+    if (fa.numRegs != r2::LAUNCH_REGS) return cudaErrorInvalidConfiguration;  // setmaxnreg budget
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
     if (e != cudaSuccess) return e;
     fn<<<grid, r2::NTHREADS, p.smem_bytes, st>>>(p, leaf_steps, n_leaf, sum_steps, n_sum);
     return cudaGetLastError();

@@ -1,5 +1,5 @@
 """Build an experimental variant of libspnb.so with extra -D flags on the
-kernel translation units (A/B timing on the GPU box; load it with
+layered kernel translation units (A/B timing on the GPU box; load it with
 SPNB_LIB=<path>).  Usage: build_variant.py NAME [-DFOO ...]"""
 import os
 import subprocess
@@ -15,8 +15,8 @@ os.makedirs(out_dir, exist_ok=True)
 objs = []
 for s in B.CU_SOURCES + B.CXX_SOURCES:
     obj = os.path.join(B.BUILD, s + ".o")
-    if s == "rat_eval.cu" and defs:
-        vobj = os.path.join(out_dir, f"rat_eval_{name}.o")
+    if s in ("rat_eval.cu", "rat2.cu") and defs:
+        vobj = os.path.join(out_dir, f"{s[:-3]}_{name}.o")
         subprocess.run([B._nvcc()] + B.NVCC_FLAGS + defs + ["-c", os.path.join(B.CSRC, s), "-o", vobj],
                        check=True)
         obj = vobj

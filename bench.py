@@ -236,7 +236,8 @@ def _config_dict(args, g, n, world=1, scaling="weak"):
     desc = CONFIGS[args.config]["desc"]
     if args.config in _N_OVERRIDE:
         desc += f" [--samples {_N_OVERRIDE[args.config]}]"
-    d = {"workload": f"{args.config}: {desc}",
+    query = "marginal" if args.marginal else "joint"
+    d = {"workload": f"{args.config}: {desc}, {query}",
          "query": "marginal" if args.marginal else "joint",
          "samples_per_gpu": n, "n_features": g.n_features, "n_roots": g.n_roots,
          "graph_nodes": c["nodes"], "sum_edges": c["sum_edges"],

@@ -317,17 +317,17 @@ def rat_counts(F, D, R, S, I, C):
 # Named configs (BASELINE.json "configs")
 # --------------------------------------------------------------------------
 CONFIGS = {
-    "C1": dict(desc="toy SPN (Fig.1 stand-in), 100k samples, joint+marginal",
+    "C1": dict(desc="toy SPN (Fig.1 stand-in), 100k samples",
                n_samples=100_000),
-    "C2": dict(desc="speaker-ID SPN, 26 Gaussian features, ~2.5k nodes, 1M samples, joint",
+    "C2": dict(desc="speaker-ID SPN, 26 Gaussian features, ~2.5k nodes, 1M samples",
                n_samples=1_000_000, graph_seed=2001, data_seed=2002),
-    "C3": dict(desc="32 speaker SPNs, 20% NaN marginal + argmax, 1M samples",
+    "C3": dict(desc="32 speaker SPNs, 20% NaN, argmax, 1M samples",
                n_samples=1_000_000, graph_seeds=list(range(3001, 3033)),
                data_seed=3002, nan_seed=3100, nan_p=0.2),
     "C4": dict(desc="RAT-SPN D5 R8 S20 I40 C10 over 784 features, 100k samples",
                n_samples=100_000, graph_seed=4001, data_seed=4002,
                rat=dict(F=784, D=5, R=8, S=20, I=40, C=10)),
-    "C5": dict(desc="RAT-SPN D5 R50 S20 I40 C10 (3.24M nodes), 10M samples",
+    "C5": dict(desc="RAT-SPN D5 R50 S20 I40 C10 (3.24M nodes), 10M samples, argmax",
                n_samples=10_000_000, graph_seed=5001, data_seed=5002,
                rat=dict(F=784, D=5, R=50, S=20, I=40, C=10)),
 }

@@ -408,7 +408,14 @@ def run_ours(args):
         metric_roof = {"frac": hm, "binding": "hbm" if hbm_part["frac"] >= mufu_part["frac"]
                        else "mufu", "hbm": hbm_part, "mufu": mufu_part}
         peak_note = f"x 148 SMs x {clock_mhz:.0f} MHz (sm_max_mhz, {src})"
-        if info["path"] in (0, 2):
+        if info["path"] in (0, 2) and hbm_part["frac"] >= mufu_part["frac"]:
+            # e.g. C1 at 1e8 samples in linear space: one lg2 per sample, HBM binds
+            roof = {"bound": "hbm", "achieved": hbm, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                    "frac": hbm_part["frac"], "traffic": traffic,
+                    "peak_source": f"hbm_gbs ({src})", "bytes_per_sample": info["bytes_per_sample"],
+                    "value_space": "linear" if info.get("value_space") == 2 else "log2",
+                    "hbm_mufu": metric_roof, "mufu": mufu_part}
+        elif info["path"] in (0, 2):
             roof = {"bound": "alu", "pipe": "MUFU ex2/lg2 (16 op/clk/SM)",
                     "achieved": mufu / 1e9, "peak": mufu_peak / 1e9, "unit": "Gop/s",
                     "frac": mufu / mufu_peak, "traffic": traffic,

@@ -583,9 +583,10 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         R2Params rp;
         memset(&rp, 0, sizeof(rp));
         bool fits = false;
-        // deepest rings that fit: leaf inputs 3..2 (3 lets both leaf groups
-        // prefetch), weight groups 4..2 (the MMA warp holds a pair at once)
-        static const int kRings[][2] = {{3, 4}, {3, 3}, {3, 2}, {2, 4}, {2, 2}};
+        // deepest rings that fit: leaf inputs 3..2, weight groups 3..2 (the
+        // MMA warp holds a pair at once); the left/right leaf outputs have
+        // R2_NAB = 3 slots (the leaf warps' run-ahead past the epilogue)
+        static const int kRings[][2] = {{3, 3}, {3, 2}, {2, 3}, {2, 2}, {2, 2}};
         // v2 runs the single f16 pass (hi/lo operands do not fit its shared
         // memory on C4/C5-sized regions): tc_precision 2 keeps v1
         if (r2.ok && opt.tc_precision == 2) {
@@ -727,6 +728,11 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     // (spill fallback to 2 x 256) 2.12e9
     jo.min_blocks = opt.ctas_per_sm > 0 ? opt.ctas_per_sm : std::max(1, 768 / jo.block);
     if (const char *e = getenv("SPNB_JIT_MINB")) jo.min_blocks = std::max(1, atoi(e));
+    // tiny SPNs (C1's toy: 12 nodes) are bound by HBM, not by their few
+    // instructions: four interleaved samples per thread keep 4x the loads in
+    // flight (large SPNs stay at one: register pressure, SPNB_JIT_K=2 measured
+    // 1.42e9 vs 3.6e9 samples/s on C2)
+    if ((int64_t)g.kind.size() <= 64) jo.samples_per_thread = 4;
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
     if (const char *e = getenv("SPNB_JIT_BAR")) jo.bar_every = std::max(0, atoi(e));
     JitProgram jp;

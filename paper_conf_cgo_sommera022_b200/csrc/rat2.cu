@@ -56,6 +56,16 @@ constexpr int REG_LEAF = 96, REG_EPI = 120, REG_PROD = 40;
 constexpr int NLG = 1, EPI_COLS = 80;
 constexpr int REG_LEAF = 152, REG_EPI = 152, REG_PROD = 56;
 #endif
+#ifndef R2_NAB
+#define R2_NAB 3  // left / right leaf-output slots (the leaf warps' run-ahead)
+#endif
+constexpr int NAB = R2_NAB;
+#ifndef EPI_SHARE
+#define EPI_SHARE 0  // 1: both epilogue warps of a lane quarter drain every group (measured slower)
+#endif
+#ifndef LEAF_SPT
+#define LEAF_SPT 4  // samples per leaf thread (4: one region per 4 warps; 8: per 2 warps, measured no faster)
+#endif
 constexpr int NTHREADS = (4 * NLG + 12) * 32;
 // registers per thread of the launch (65536 / NTHREADS rounded down to 8):
 // the pool setmaxnreg redistributes; rat2_launch refuses a build whose
@@ -101,15 +111,29 @@ __device__ __forceinline__ void bar_init(uint32_t b, uint32_t count) {
 // hardware until the phase completes (or the hint expires) instead of
 // spinning -- spinning producer / MMA warps (the highest warp ids, which the
 // scheduler favours) would otherwise take issue slots from the epilogue
+// R2_WATCHDOG builds (development): a wait that has not completed after
+// 2^34 cycles (~9 s; a 128-sample tile takes ~6 ms on C5) is a protocol
+// deadlock -- trap so the launch fails instead of hanging the device.  Off
+// in the product build (the clock reads cost ~7% on C5).
 __device__ __forceinline__ void bar_wait(uint32_t b, uint32_t parity) {
     uint32_t done = 0;
-    while (!done) {
+#ifdef R2_WATCHDOG
+    long long t0 = 0;
+#endif
+    while (true) {
         asm volatile(
             "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
             "selp.u32 %0, 1, 0, p;\n\t}\n"
             : "=r"(done)
             : "r"(b), "r"(parity), "r"(0x989680u)
             : "memory");
+        if (done) break;
+#ifdef R2_WATCHDOG
+        long long t;
+        asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
+        if (t0 == 0) t0 = t;
+        else if (t - t0 > (1ll << 34)) __trap();
+#endif
     }
 }
 __device__ __forceinline__ void bar_arrive(uint32_t b) {
@@ -248,17 +272,17 @@ struct Prof {
 enum {
     B_IN_FULL = 0,    // [4]
     B_IN_EMPTY = 4,   // [4]
-    B_A_FULL = 8,     // [2]
-    B_A_EMPTY = 10,   // [2]
-    B_B_FULL = 12,    // [2]
-    B_B_EMPTY = 14,   // [2]
-    B_U_FULL = 16,
-    B_U_EMPTY = 17,
-    B_W_FULL = 18,    // [8]
-    B_W_EMPTY = 26,   // [8]
-    B_T_FULL = 34,    // [2]
-    B_T_EMPTY = 36,   // [2]
-    B_COUNT = 38
+    B_A_FULL = 8,     // [4] (NAB used)
+    B_A_EMPTY = 12,   // [4]
+    B_B_FULL = 16,    // [4]
+    B_B_EMPTY = 20,   // [4]
+    B_U_FULL = 24,
+    B_U_EMPTY = 25,
+    B_W_FULL = 26,    // [8]
+    B_W_EMPTY = 34,   // [8]
+    B_T_FULL = 42,    // [2]
+    B_T_EMPTY = 44,   // [2]
+    B_COUNT = 46
 };
 
 struct Smem {
@@ -292,21 +316,27 @@ struct Smem {
 // d0 = b DPB .. +DPB-1 (DPB = I / 4).  Per variable: one LDS.128 of the four
 // samples' features (a warp reads 128 contiguous bytes) and DPB/2 LDS.128 of
 // (a, b) pairs (4 distinct addresses per warp), then 2 DPB FFMA2.
-template <int DPB, bool MARG>
+template <int DPB, int SPT, bool MARG>
 __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, int V, int I,
-                                             int m0, int d0, float (&acc)[DPB][4]) {
+                                             int m0, int d0, float (&acc)[DPB][SPT]) {
     const float *C = prm + 2 * V * I;
 #pragma unroll
     for (int d = 0; d < DPB; ++d) {
         const float c = C[d0 + d];
-        acc[d][0] = c; acc[d][1] = c; acc[d][2] = c; acc[d][3] = c;
+#pragma unroll
+        for (int k = 0; k < SPT; ++k) acc[d][k] = c;
     }
     const float K0 = -1.0901312512f;  // 0.5 * log2(ln2 / pi): c_v = log2(a) + K0
     const float4 *ab4 = reinterpret_cast<const float4 *>(prm + 2 * d0);
     const int vstride = I / 2;  // float4 per variable
-#pragma unroll 4
+#pragma unroll 2
     for (int v = 0; v < V; ++v) {
-        const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + m0);
+        float xv[SPT];
+#pragma unroll
+        for (int c = 0; c < SPT; c += 4) {
+            const float4 x4 = *reinterpret_cast<const float4 *>(xs + v * RT + m0 + c);
+            xv[c] = x4.x; xv[c + 1] = x4.y; xv[c + 2] = x4.z; xv[c + 3] = x4.w;
+        }
         float2 q[DPB];
 #pragma unroll
         for (int k = 0; k < DPB / 2; ++k) {
@@ -315,64 +345,77 @@ __device__ __forceinline__ void leaf_compute(const float *xs, const float *prm, 
             q[2 * k + 1] = make_float2(t.z, t.w);
         }
         bool anynan = false;
-        if constexpr (MARG) anynan = (x4.x != x4.x) | (x4.y != x4.y) | (x4.z != x4.z) | (x4.w != x4.w);
+        if constexpr (MARG) {
+#pragma unroll
+            for (int k = 0; k < SPT; ++k) anynan |= xv[k] != xv[k];
+        }
         if (MARG && anynan) {
-            const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float cc = lg2(q[d].x) + K0;
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
+                for (int k = 0; k < SPT; ++k) {
                     const bool nan = xv[k] != xv[k];
                     const float t = fmaf(q[d].x, xv[k], -q[d].y);
                     acc[d][k] = fmaf(-(nan ? cc : t), nan ? 1.f : t, acc[d][k]);
                 }
             }
         } else {
-            const float2 x01 = make_float2(x4.x, x4.y), x23 = make_float2(x4.z, x4.w);
 #pragma unroll
             for (int d = 0; d < DPB; ++d) {
                 const float2 a2 = make_float2(q[d].x, q[d].x), nb2 = make_float2(-q[d].y, -q[d].y);
-                const float2 t01 = __ffma2_rn(x01, a2, nb2);
-                const float2 t23 = __ffma2_rn(x23, a2, nb2);
-                const float2 s01 = __ffma2_rn(make_float2(-t01.x, -t01.y), t01,
-                                              make_float2(acc[d][0], acc[d][1]));
-                const float2 s23 = __ffma2_rn(make_float2(-t23.x, -t23.y), t23,
-                                              make_float2(acc[d][2], acc[d][3]));
-                acc[d][0] = s01.x; acc[d][1] = s01.y; acc[d][2] = s23.x; acc[d][3] = s23.y;
+#pragma unroll
+                for (int k = 0; k < SPT; k += 2) {
+                    const float2 t = __ffma2_rn(make_float2(xv[k], xv[k + 1]), a2, nb2);
+                    const float2 r = __ffma2_rn(make_float2(-t.x, -t.y), t,
+                                                make_float2(acc[d][k], acc[d][k + 1]));
+                    acc[d][k] = r.x;
+                    acc[d][k + 1] = r.y;
+                }
             }
         }
     }
 }
 
+// leaf warps: LW = 4 NLG; a group of WPG = 16 / LEAF_SPT warps evaluates one
+// leaf region for the tile's 128 samples (thread = LEAF_SPT samples x I/4
+// distributions: lane = 8 sample groups x 4 distribution blocks); the LW /
+// WPG groups take consecutive regions (left A / right B alternate)
+constexpr int WPG = 16 / LEAF_SPT;
+constexpr int NGRP = 4 * NLG / WPG;
+
 template <int DPB, bool MARG>
 __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
                           int n_leaf, int warp, int lane) {
-    const int g = warp >> 2, gw = warp & 3;  // leaf group, warp in group (= lane quarter)
+    constexpr int SPT = LEAF_SPT;
+    const int g = warp / WPG, gw = warp % WPG;
     const int q = lane >> 2, b = lane & 3;
-    const int m0 = gw * 32 + q * 4, d0 = b * DPB;
+    const int m0 = gw * (RT / WPG) + q * SPT, d0 = b * DPB;
     const int I = p.I;
     const int64_t n_tiles = (p.n + RT - 1) / RT;
-    uint32_t li = (uint32_t)g;  // global leaf-region counter (step NLG); even: A side, odd: B side
+    uint32_t li = (uint32_t)g;  // global leaf-region counter (step NGRP); even: A side, odd: B side
     Prof pf(sm.prof(0), p.prof != nullptr);  // 0 wait input, 1 compute, 2 shifts, 3 wait output slot, 4 exps + write
     for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-        for (int l = g; l < n_leaf; l += NLG, li += NLG) {
+        for (int l = g; l < n_leaf; l += NGRP, li += NGRP) {
             const bool side_b = (l & 1) != 0;  // leaf regions alternate left (A) / right (B)
             const uint32_t j = li >> 1;         // bottom partition
             const R2Step &st = p.steps[leaf_steps[l]];
             const int s = (int)(li % (uint32_t)p.n_in);
             bar_wait(sm.bar(B_IN_FULL + s), (li / (uint32_t)p.n_in) & 1u);
             pf.mark(0);
-            float acc[DPB][4];
-            leaf_compute<DPB, MARG>(sm.in_x(s), sm.in_prm(s), st.n_vars, I, m0, d0, acc);
+            float acc[DPB][SPT];
+            leaf_compute<DPB, SPT, MARG>(sm.in_x(s), sm.in_prm(s), st.n_vars, I, m0, d0, acc);
+            // the slot's next fill is an async-proxy (TMA) write: order this
+            // warp's generic-proxy reads before the release of the slot
+            fence_async_smem();
             __syncwarp();
             if (lane == 0) bar_arrive(sm.bar(B_IN_EMPTY + s));
             pf.mark(1);
             // per-sample shift over the I distributions: local max over DPB,
-            // then across the 4 lanes of the sample quad (xor 1, 2)
-            float h[4];
+            // then across the 4 lanes of the sample group (xor 1, 2)
+            float h[SPT];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {
+            for (int k = 0; k < SPT; ++k) {
                 float v = acc[0][k];
 #pragma unroll
                 for (int d = 1; d < DPB; ++d) v = maxnan(v, acc[d][k]);
@@ -380,8 +423,8 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
                 v = maxnan(v, __shfl_xor_sync(0xffffffffu, v, 2));
                 h[k] = v;
             }
-            const int ab = (int)(j & 1u);
-            const uint32_t ph = (j >> 1) & 1u;
+            const int ab = (int)(j % NAB);
+            const uint32_t ph = (j / NAB) & 1u;
             pf.mark(2);
             // both sides wait for the A slot (it also carries hb)
             bar_wait(sm.bar(B_A_EMPTY + ab), ph ^ 1u);
@@ -391,20 +434,26 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
                 float *ea = sm.ea(ab);
 #pragma unroll
                 for (int d = 0; d < DPB; ++d) {
-                    float e[4];
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) e[k] = ex2(acc[d][k] - fmaxf(h[k], -1e30f));
-                    *reinterpret_cast<float4 *>(ea + (d0 + d) * RT + m0) =
-                        make_float4(e[0], e[1], e[2], e[3]);
+                    for (int c = 0; c < SPT; c += 4) {
+                        float e[4];
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) e[k] = ex2(acc[d][c + k] - fmaxf(h[c + k], -1e30f));
+                        *reinterpret_cast<float4 *>(ea + (d0 + d) * RT + m0 + c) =
+                            make_float4(e[0], e[1], e[2], e[3]);
+                    }
                 }
                 if (b == 0)
-                    *reinterpret_cast<float4 *>(sm.ha(ab) + m0) = make_float4(h[0], h[1], h[2], h[3]);
+#pragma unroll
+                    for (int c = 0; c < SPT; c += 4)
+                        *reinterpret_cast<float4 *>(sm.ha(ab) + m0 + c) =
+                            make_float4(h[c], h[c + 1], h[c + 2], h[c + 3]);
                 bar_arrive(sm.bar(B_A_FULL + ab));
             } else {
                 uint8_t *img = sm.bimg(ab);
                 const int part = p.bimg_bytes / 2;  // lo image after hi (prec 3)
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
+                for (int k = 0; k < SPT; ++k) {
                     const float hc = fmaxf(h[k], -1e30f) - EB_SHIFT;
 #pragma unroll
                     for (int d = 0; d < DPB; d += 2) {
@@ -421,8 +470,11 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
                     }
                 }
                 if (b == 0)
-                    *reinterpret_cast<float4 *>(sm.hb(ab) + m0) =
-                        make_float4(h[0] - EB_SHIFT, h[1] - EB_SHIFT, h[2] - EB_SHIFT, h[3] - EB_SHIFT);
+#pragma unroll
+                    for (int c = 0; c < SPT; c += 4)
+                        *reinterpret_cast<float4 *>(sm.hb(ab) + m0 + c) =
+                            make_float4(h[c] - EB_SHIFT, h[c + 1] - EB_SHIFT, h[c + 2] - EB_SHIFT,
+                                        h[c + 3] - EB_SHIFT);
                 fence_async_smem();
                 bar_arrive(sm.bar(B_B_FULL + ab));
             }
@@ -584,8 +636,8 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
             const int G = st.n_groups, ksteps = st.kpad / 16;
             uint32_t a_addr;
             if (bot) {
-                const int ab = (int)(kb & 1u);
-                bar_wait(sm.bar(B_B_FULL + ab), (kb >> 1) & 1u);
+                const int ab = (int)(kb % NAB);
+                bar_wait(sm.bar(B_B_FULL + ab), (kb / NAB) & 1u);
                 a_addr = smem_u32(sm.bimg(ab));
             } else {
                 bar_wait(sm.bar(B_U_FULL), ku & 1u);
@@ -595,6 +647,49 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
             const uint64_t a_desc = a_hi_bits | (uint64_t)((a_addr >> 4) & 0x3FFFu);
             const uint32_t a_lo_d = ((uint32_t)(bot ? p.bimg_bytes : p.uimg_bytes) / 2) >> 4;
             const uint32_t ka_d = (2 * lbo_a) >> 4;
+#if EPI_SHARE
+            // per group: wait only for this group's accumulator, so group g+1's
+            // chain starts while the epilogue still drains the other buffer
+            for (int gi = 0; gi < G; ++gi) {
+                const int b = gi & 1;
+                const GroupInfo gr = group_info(st, gi);
+                uint32_t wsl = 0;
+                pf.mark(3);
+                if (gr.ns > 0) {
+                    wsl = w_idx;
+                    bar_wait(bar_wfull + 8u * w_idx, w_ph);
+                    if (++w_idx == n_w) {
+                        w_idx = 0;
+                        w_ph ^= 1u;
+                    }
+                }
+                pf.mark(1);
+                bar_wait(bar_tempty + 8u * b, (tp & 1u) ^ 1u);
+                pf.mark(2);
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t lbo_b = (uint32_t)gr.ncol * 16;
+                    const uint64_t w_desc =
+                        desc_hi(lbo_b, 128) | (uint64_t)(((wbase + wsl * wstride) >> 4) & 0x3FFFu);
+                    const uint32_t kw_d = (2 * lbo_b) >> 4;
+                    const uint32_t idesc = (1u << 4) | ((uint32_t)(gr.ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
+                    const uint32_t d = tmem + (b ? (uint32_t)R2_COLS_A : 0u);
+                    if (gr.ns > 0)
+                        for (int kk = 0; kk < ksteps; ++kk) {
+                            const uint64_t ad = a_desc + kk * ka_d, wd = w_desc + kk * kw_d;
+                            umma_f16(d, ad, wd, idesc, kk > 0);
+                            if (split) {
+                                umma_f16(d, ad + a_lo_d, wd, idesc, 1);
+                                umma_f16(d, ad, wd + wlo_d, idesc, 1);
+                            }
+                        }
+                    umma_commit(bar_tfull + 8u * b);
+                    if (gr.ns > 0) umma_commit(bar_wempty + 8u * wsl);
+                }
+                __syncwarp();
+                if (b) ++tp;
+            }
+#else
             for (int gp = 0; gp < G; gp += 2, ++tp) {
                 GroupInfo gr[2] = {group_info(st, gp), group_info(st, gp + 1)};
                 uint32_t wsl[2] = {0, 0};
@@ -647,7 +742,8 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                 }
                 __syncwarp();
             }
-            if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb & 1u) : B_U_EMPTY));
+#endif
+            if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb % NAB) : B_U_EMPTY));
             __syncwarp();
             if (bot) ++kb;
             else ++ku;
@@ -724,6 +820,47 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         }
     };
     const int G = st.n_groups;
+#if EPI_SHARE
+    // both warps of the lane quarter take every group, alternating its sums
+    constexpr int QB = NA >= EPI_COLS / 2 ? 1 : EPI_COLS / 2 / NA;  // own sums per TMEM batch
+    for (int gi = 0; gi < G; ++gi) {
+        const int b = gi & 1;
+        const GroupInfo gr = group_info(st, gi);
+        pf.mark(3);
+        bar_wait(sm.bar(B_T_FULL + b), (tp & 1u));
+        pf.mark(2);
+        tc_fence_after();
+        const uint32_t acc = lane_base + (b ? (uint32_t)R2_COLS_A : 0u);
+        const int ns = gr.ns;
+        const int mine = ns > h ? (ns - h + 1) / 2 : 0;  // this warp's sums: h, h + 2, ...
+        for (int k0 = 0; k0 < mine; k0 += QB) {
+            float t[QB * NA], kv[QB];
+#pragma unroll
+            for (int k = 0; k < QB; ++k) {
+                const int sl = h + 2 * (k0 + k);
+                if (k0 + k < mine) ld_cols<NA>(acc + (uint32_t)(sl * NA), t + k * NA);
+                kv[k] = k0 + k < mine ? __ldg(ks + gr.s0 + sl) : 0.f;
+            }
+            tmem_wait_ld();
+            if (k0 + QB >= mine) {
+                tc_fence_before();
+                bar_arrive(sm.bar(B_T_EMPTY + b));
+            }
+            float val[QB];
+#pragma unroll
+            for (int k = 0; k < QB; ++k) val[k] = dot4(ear, t + k * NA);
+#pragma unroll
+            for (int k = 0; k < QB; ++k)
+                if (k0 + k < mine) fin(gr.s0 + h + 2 * (k0 + k), val[k], kv[k]);
+        }
+        if (mine == 0) {
+            tc_fence_before();
+            bar_arrive(sm.bar(B_T_EMPTY + b));
+        }
+        if (b) ++tp;
+    }
+    return;
+#endif
     for (int gi = h; gi < G; gi += 2) {  // this warp's accumulator: groups of parity h
         const int b = gi & 1;
         const GroupInfo gr = group_info(st, gi);
@@ -797,8 +934,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
             const uint32_t out_col = col_slots + (uint32_t)((es.slot_out - 1) * S);
             if (es.type == 1) {
                 // BOT: ea from leaf group 0, hb from leaf group 1
-                const int ab = (int)(kb & 1u);
-                const uint32_t ph = (kb >> 1) & 1u;
+                const int ab = (int)(kb % NAB);
+                const uint32_t ph = (kb / NAB) & 1u;
                 bar_wait(sm.bar(B_A_FULL + ab), ph);
                 bar_wait(sm.bar(B_B_FULL + ab), ph);
                 pf.mark(0);
@@ -904,21 +1041,21 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     if (tid == 0) {
         for (int i = 0; i < 4; ++i) {
             bar_init(sm.bar(B_IN_FULL + i), 1);
-            bar_init(sm.bar(B_IN_EMPTY + i), 4);
+            bar_init(sm.bar(B_IN_EMPTY + i), WPG);  // the warps of one leaf group
         }
         for (int i = 0; i < 8; ++i) {
             bar_init(sm.bar(B_W_FULL + i), 1);
             bar_init(sm.bar(B_W_EMPTY + i), 1);
         }
-        for (int i = 0; i < 2; ++i) {
-            bar_init(sm.bar(B_A_FULL + i), 128);
+        for (int i = 0; i < NAB; ++i) {
+            bar_init(sm.bar(B_A_FULL + i), WPG * 32);  // the threads of one leaf group
             bar_init(sm.bar(B_A_EMPTY + i), 256);  // both epilogue warps of each quarter
-            bar_init(sm.bar(B_B_FULL + i), 128);
+            bar_init(sm.bar(B_B_FULL + i), WPG * 32);
             bar_init(sm.bar(B_B_EMPTY + i), 1);
         }
         for (int i = 0; i < 2; ++i) {
             bar_init(sm.bar(B_T_FULL + i), 1);
-            bar_init(sm.bar(B_T_EMPTY + i), 128);
+            bar_init(sm.bar(B_T_EMPTY + i), EPI_SHARE ? 256 : 128);  // epilogue threads draining it
         }
         bar_init(sm.bar(B_U_FULL), 128);
         bar_init(sm.bar(B_U_EMPTY), 1);
@@ -926,7 +1063,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         for (int k = 0; k < 32; ++k) sm.prof(0)[k] = 0;
     }
     // zero the operand images once (the K padding columns stay zero)
-    for (int i = tid * 16; i < 2 * p.bimg_bytes + p.uimg_bytes; i += NTHREADS * 16)
+    for (int i = tid * 16; i < NAB * p.bimg_bytes + p.uimg_bytes; i += NTHREADS * 16)
         *reinterpret_cast<uint4 *>(base + p.off_bimg + i) = make_uint4(0, 0, 0, 0);
     fence_async_smem();
     tc_fence_before();
@@ -985,11 +1122,11 @@ int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int
     off += n_in * p.in_bytes;
     p.ea_bytes = up((I + 2) * r2::RT * 4, 128);
     p.off_ea = off;
-    off += 2 * p.ea_bytes;
+    off += r2::NAB * p.ea_bytes;
     off = up(off, 1024);
     p.bimg_bytes = r2::RT * kpad_bot * 2 * parts;
     p.off_bimg = off;
-    off += 2 * p.bimg_bytes;
+    off += r2::NAB * p.bimg_bytes;
     p.uimg_bytes = r2::RT * kpad_up * 2 * parts;
     p.off_uimg = off;  // contiguous with the B images (zeroed together)
     off += p.uimg_bytes;

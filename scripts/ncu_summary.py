@@ -25,6 +25,8 @@ KEYS = [
     "smsp__inst_executed.sum", "thread_inst_executed",
     "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
     "lts__t_bytes.sum", "sm__cycles_elapsed.avg.per_second",
+    "lts__t_sector_hit_rate.pct", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+    "TPC.TriageCompute.sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
 ]
 UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
 

@@ -51,6 +51,24 @@ if what in ("parity", "all"):
         print("C4 prec", prec, "err", err(out.cpu().numpy(), ref), "argmax agree",
               float((am.cpu().numpy() == ref.argmax(1)).mean()), flush=True)
 
+if what == "time1":   # v2 single pass only (A/B of kernel variants)
+    for cfg, n in (("C4", 100_000), ("C5", 18944 * 16)):
+        g = config_graph(cfg)
+        xd = bench.device_uniform(n, g.n_features, 4002, 0, torch.device("cuda"))
+        P = spnb.Plan(spnb.Graph(g), tc_precision=1, layered_kernel=2)
+        out, am = P.infer(xd)
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(3):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            P.infer(xd, out=out, argmax=am)
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        print(cfg, "v2 prec 1 ms", round(min(ts), 3), "samples/s", f"{n / min(ts) * 1e3:.3e}",
+              "mean logp", float(out.float().mean()), flush=True)
+
 if what in ("time", "all"):
     for cfg, n in (("C4", 100_000), ("C5", 18944 * 16)):
         g = config_graph(cfg)

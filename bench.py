@@ -424,19 +424,30 @@ def run_ours(args):
                                   "n-ary log-sum-exp)",
                     "hbm_mufu": metric_roof, "hbm": hbm_part}
         else:
-            # layered path: the binding pipe is FP32 FMA (leaf layer + stage-2
-            # contractions); tensor fraction on algorithmic one-pass flops
-            roof = {"bound": "alu", "pipe": "FP32 FMA (leaf layer, 128 lanes/clk/SM)",
-                    "achieved": fma / 1e9, "peak": fma_peak / 1e9, "unit": "GFMA/s",
-                    "frac": fma / fma_peak, "traffic": traffic,
-                    "peak_source": "128 FMA/clk/SM " + peak_note,
-                    "hbm_mufu": metric_roof,
-                    "tensor": {"achieved": tc / 1e12, "peak": tc_peak / 1e12,
-                               "unit": "TFLOP/s", "frac": tc / tc_peak,
-                               "flops": "algorithmic, one pass (2 na nb S per sum region)",
-                               "passes_executed": info["tc_passes"],
-                               "peak_source": f"bf16_tflops ({src}); f16 dense rate = bf16"},
-                    "kernel": f"layered v{info['layered_kernel']}"}
+            # layered path: the binding unit is the one with the highest
+            # fraction -- FP32 FMA (FMA leaf layer + stage-2 contractions) or,
+            # with the leaf layer on the tensor cores (leaf_tc), the tensor
+            # pipe (algorithmic one-pass flops: leaf GEMMs + sum contractions)
+            ltc = bool(info.get("leaf_tc"))
+            fma_part = {"achieved": fma / 1e9, "peak": fma_peak / 1e9, "unit": "GFMA/s",
+                        "frac": fma / fma_peak, "peak_source": "128 FMA/clk/SM " + peak_note,
+                        "pipe": ("FP32 FMA (stage-2 contractions)" if ltc else
+                                 "FP32 FMA (leaf layer + stage-2 contractions, 128 lanes/clk/SM)")}
+            tc_part = {"achieved": tc / 1e12, "peak": tc_peak / 1e12, "unit": "TFLOP/s",
+                       "frac": tc / tc_peak,
+                       "flops": ("algorithmic, one pass: 2 I (2V+1) per leaf region (tensor-core "
+                                 "leaves) + 2 na nb S per sum region" if ltc else
+                                 "algorithmic, one pass (2 na nb S per sum region)"),
+                       "passes_executed": {"leaf": 3 if ltc else 0, "sum": info["tc_passes"]},
+                       "peak_source": f"bf16_tflops ({src}); f16 dense rate = bf16"}
+            if tc_part["frac"] > fma_part["frac"]:
+                roof = {"bound": "tensor", **tc_part, "traffic": traffic, "fma": fma_part,
+                        "hbm_mufu": metric_roof}
+            else:
+                roof = {"bound": "alu", **fma_part, "traffic": traffic, "tensor": tc_part,
+                        "hbm_mufu": metric_roof}
+            roof["kernel"] = (f"layered v{info['layered_kernel']}" +
+                              (", tensor-core leaves" if ltc else ""))
         # the oracle baseline is timed on rank 0 at N = 1 only (contract)
         cpu = cpu_baseline(g, x, args.marginal) if world == 1 else None
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
@@ -453,7 +464,7 @@ def run_ours(args):
                                                   "max_stack", "kernel_regs", "ctas_per_sm",
                                                   "mufu_exec_per_sample", "compile_ms",
                                                   "chunk_samples", "layered_kernel",
-                                                  "tc_passes")},
+                                                  "tc_passes", "leaf_tc", "certified")},
                     "prepare_s": prep_s,
                     "tc_precision": args.tc_precision},
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk,

@@ -113,7 +113,17 @@ typedef struct spn_prepare_options {
                                    in [2^-100, 2^100]: sums become FFMA chains
                                    and the only MUFU op is one lg2 per root.
                                    2 on an ineligible graph: E_UNSUPPORTED  */
-    int32_t reserved[5];        /* must be zero                                */
+    int32_t leaf_tc;            /* layered v2: leaf layer on the tensor cores
+                                   (one GEMM of per-sample features x~^2, x~
+                                   against the Gaussians' expanded constants,
+                                   f16 hi/lo split, fp32 accumulation in TMEM).
+                                   0 auto (= off: measured slower than the FMA
+                                   leaves on C4/C5), 1 off
+                                   (FP32 FMA leaves), 2 on (needs tc_precision
+                                   0: the certification recomputes inputs
+                                   outside the split's range; E_UNSUPPORTED if
+                                   not applicable)                           */
+    int32_t reserved[4];        /* must be zero                                */
 } spn_prepare_options;
 
 /* Statistics of a prepared plan (used by the benchmark's roofline). */
@@ -166,6 +176,8 @@ typedef struct spn_plan_stats {
                                    - cert_err) for all its roots (the other
                                    0.1e-4 of the tolerance covers the fp32
                                    arithmetic both precisions share)          */
+    int32_t leaf_tc;            /* layered v2: 1 when the leaf layer runs on
+                                   the tensor cores (spn_prepare_options)    */
 } spn_plan_stats;
 
 /* Fill *opt with defaults (all auto). */
@@ -291,6 +303,18 @@ int spn_build_layered(const spn_handle *graph, int32_t *is_layered, char *why, i
 int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
                        int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
                        void *wimg, int32_t *root_map, double *tc_err_1pass);
+/*
+ * spn_build_layered2_ex: spn_build_layered2 with leaf_tc = 1 building the
+ *   tensor-core leaf variant (spn_prepare_options.leaf_tc): per leaf step
+ *   fparams holds the centres M[lvp] and the weight-image bytes at w_off
+ *   hold the joint parameter image [hi, lo] (wbytes_a bytes each, K = kl_j)
+ *   then the marginal one (wbytes_b each, K = kl_m), both K-major f16 with
+ *   48 rows; dims[14] = dims[11] of spn_build_layered2 then {lvp, kl_j,
+ *   kl_m}.  leaf_tc = 0: exactly spn_build_layered2 (dims[11]).
+ */
+int spn_build_layered2_ex(const spn_handle *graph, int32_t leaf_tc, int32_t *ok, char *why,
+                          int64_t why_len, int64_t *sizes, int32_t *dims, void *steps, int32_t *vars,
+                          float *fparams, void *wimg, int32_t *root_map, double *tc_err_1pass);
 int spn_partition_graph(const spn_handle *graph, int64_t max_task_ops, int32_t *task_of_node,
                         int32_t *n_tasks, int64_t *cost, int64_t *cut_values);
 int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32_t x_in_smem,

@@ -55,7 +55,7 @@ class _Options(ctypes.Structure):
                 ("max_task_nodes", ctypes.c_int64), ("tc_precision", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("compiled_path", ctypes.c_int32),
                 ("layered_kernel", ctypes.c_int32), ("value_space", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 5)]
+                ("leaf_tc", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
 
 
 class _Stats(ctypes.Structure):
@@ -71,7 +71,7 @@ class _Stats(ctypes.Structure):
         ("compile_ms", ctypes.c_double), ("chunk_samples", ctypes.c_int64),
         ("layered_kernel", ctypes.c_int32), ("tc_passes", ctypes.c_int32),
         ("value_space", ctypes.c_int32), ("certified", ctypes.c_int32),
-        ("cert_err", ctypes.c_double)]
+        ("cert_err", ctypes.c_double), ("leaf_tc", ctypes.c_int32)]
 
 
 _lib = None
@@ -172,7 +172,8 @@ class Plan:
     def __init__(self, graph: Graph, device: int | None = None, block_threads: int = 0,
                  samples_per_thread: int = 0, max_task_nodes: int = 0,
                  layered_path: int = 0, tc_precision: int = 0, ctas_per_sm: int = 0,
-                 compiled_path: int = 0, layered_kernel: int = 0, value_space: int = 0):
+                 compiled_path: int = 0, layered_kernel: int = 0, value_space: int = 0,
+                 leaf_tc: int = 0):
         lib = load_library()
         opt = _Options()
         lib.spn_default_options(ctypes.byref(opt))
@@ -189,6 +190,7 @@ class Plan:
         opt.compiled_path = compiled_path
         opt.layered_kernel = layered_kernel
         opt.value_space = value_space
+        opt.leaf_tc = leaf_tc
         h = ctypes.c_void_p()
         _check(lib.spn_prepare(graph.handle, ctypes.byref(opt), ctypes.byref(h)))
         self._h = h
@@ -342,17 +344,19 @@ R2STEP_DTYPE = np.dtype([(n, "<i4") for n in ("type", "root", "n_out", "na", "nb
                                               "wbytes_a", "wbytes_b")])
 
 
-def build_layered2(graph: Graph):
-    """Host-only: the v2 layered kernel's plan (``spn_build_layered2``).
-    Returns (plan dict, "") or (None, reason)."""
+def build_layered2(graph: Graph, leaf_tc: bool = False):
+    """Host-only: the v2 layered kernel's plan (``spn_build_layered2_ex``;
+    leaf_tc: the tensor-core leaf variant).  Returns (plan dict, "") or
+    (None, reason)."""
     lib = load_library()
     ok = ctypes.c_int32()
     why = ctypes.create_string_buffer(256)
     sizes = np.zeros(6, dtype=np.int64)
-    dims = np.zeros(11, dtype=np.int32)
+    dims = np.zeros(14, dtype=np.int32)
     err = ctypes.c_double()
-    _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
-                                  _ptr(dims), None, None, None, None, None, ctypes.byref(err)))
+    lt = 1 if leaf_tc else 0
+    _check(lib.spn_build_layered2_ex(graph.handle, lt, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                     _ptr(dims), None, None, None, None, None, ctypes.byref(err)))
     if not ok.value:
         return None, why.value.decode()
     assert sizes[5] == R2STEP_DTYPE.itemsize, (sizes[5], R2STEP_DTYPE.itemsize)
@@ -361,13 +365,14 @@ def build_layered2(graph: Graph):
     fp = np.zeros(sizes[2], dtype=np.float32)
     w = np.zeros(sizes[3] // 2, dtype=np.float16)
     rm = np.zeros(sizes[4], dtype=np.int32)
-    _check(lib.spn_build_layered2(graph.handle, ctypes.byref(ok), why, 256, _ptr(sizes),
-                                  _ptr(dims), _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w),
-                                  _ptr(rm), None))
+    _check(lib.spn_build_layered2_ex(graph.handle, lt, ctypes.byref(ok), why, 256, _ptr(sizes),
+                                     _ptr(dims), _ptr(steps), _ptr(vars_), _ptr(fp), _ptr(w),
+                                     _ptr(rm), None))
     keys = ("F", "C", "I", "S", "D", "gcols", "kpad_bot", "kpad_up", "max_wgroup", "max_vars",
-            "max_blk")
+            "max_blk", "lvp", "kl_j", "kl_m")
     return {"steps": steps, "vars": vars_, "fparams": fp, "wimg": w, "root_map": rm,
-            "tc_err_1pass": float(err.value), **{k: int(v) for k, v in zip(keys, dims)}}, ""
+            "tc_err_1pass": float(err.value), "leaf_tc": bool(leaf_tc),
+            **{k: int(v) for k, v in zip(keys, dims)}}, ""
 
 
 def codegen(graph: Graph, task: int = 0, lang: str = "cpp", compile: bool = False,

@@ -42,7 +42,7 @@ cudaError_t transpose_launch(const float *x, int64_t n, int64_t ld, int F, float
                              int64_t rows_pad, cudaStream_t st);
 bool rat2_supported_shape(int I, int S);
 int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int kpad_up,
-                int max_wgroup, int prec, int n_in, int n_w);
+                int max_wgroup, int prec, int n_in, int n_w, int lvp, int kl_j, int kl_m);
 cudaError_t cert_gather_launch(const float *x, int64_t ld, int F, const int64_t *idx,
                                const int32_t *count, int64_t off, int64_t cap, float *xT,
                                int64_t ldT, cudaStream_t st);
@@ -130,6 +130,7 @@ struct DevicePlan {
     // certified single pass (tc_precision auto): samples whose a-priori
     // error bound does not fit the tolerance are recomputed by v1 in hi/lo
     bool cert = false;
+    bool leaf_tc = false;  // v2 with the leaf layer on the tensor cores
     float cert_err = 0.f;
     int32_t *d_flag_count = nullptr;
     int64_t *d_flag_idx = nullptr;  // grown (stream-ordered) to the largest n seen
@@ -223,7 +224,7 @@ void free_plan(DevicePlan *p) {
         if (p->r2) {
             unsigned long long h2[32];
             if (cudaMemcpy(h2, p->d_prof, sizeof(h2), cudaMemcpyDeviceToHost) == cudaSuccess) {
-                const char *roles[4] = {"leaf(8 warps)", "epilogue(4)", "mma", "producer"};
+                const char *roles[4] = {"leaf warps", "epilogue(8)", "mma", "producers"};
                 const char *ph[4][8] = {
                     {"wait_in", "compute", "shift", "wait_out", "exp+write", "-", "-", "-"},
                     {"wait_leaf", "up_phase1", "wait_mma", "sums", "tile_io", "step_end", "ld_issue", "ld_wait"},
@@ -572,7 +573,27 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     if (const char *r2env = getenv("SPNB_RAT2"); r2env && want_r2 == 0) want_r2 = atoi(r2env) == 0 ? 1 : 0;
     if (want_r2 != 1) {
         Rat2Plan r2;
-        build_rat2(lp, r2);
+        // tensor-core leaves (opt-in, leaf_tc 2): measured slower than the FMA
+        // leaves on C4 / C5, so auto keeps the FMA leaves;
+        // they need the certification (it recomputes the inputs outside the
+        // split operands' range)
+        const bool try_ltc = opt.leaf_tc == 2;
+        std::string ltc_why;
+        if (try_ltc) {
+            build_rat2(lp, r2, true);
+            if (r2.ok && !std::isfinite(r2.tc_err_1pass)) {
+                r2.ok = false;
+                r2.why = "no certification bound (a zero sum weight)";
+            }
+            if (!r2.ok) ltc_why = r2.why;
+        }
+        if (opt.leaf_tc == 2 && (!r2.ok || opt.tc_precision != 0)) {
+            free_plan(P);
+            return set_err(SPN_E_UNSUPPORTED, opt.tc_precision != 0
+                                                  ? std::string("leaf_tc 2 needs tc_precision 0 (certified)")
+                                                  : "leaf_tc not applicable: " + ltc_why);
+        }
+        if (!r2.ok) build_rat2(lp, r2);
         if (r2.ok && !rat2_supported_shape(r2.I, r2.S)) {
             r2.ok = false;
             r2.why = "no v2 kernel instance for I = " + std::to_string(r2.I) + ", S = " +
@@ -587,6 +608,9 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         // MMA warp holds a pair at once); the left/right leaf outputs have
         // R2_NAB = 3 slots (the leaf warps' run-ahead past the epilogue)
         static const int kRings[][2] = {{3, 3}, {3, 2}, {2, 3}, {2, 2}, {2, 2}};
+        // tensor-core leaves: two input slots (features + parameter image)
+        static const int kRingsT[][2] = {{2, 3}, {2, 2}, {2, 2}, {2, 2}, {2, 2}};
+        const bool ltc = r2.ok && r2.leaf_tc;
         // v2 runs the single f16 pass (hi/lo operands do not fit its shared
         // memory on C4/C5-sized regions): tc_precision 2 keeps v1
         if (r2.ok && opt.tc_precision == 2) {
@@ -595,7 +619,19 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
         }
         for (int a = 0; r2.ok && a < 5 && !fits; ++a)
             fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
-                               r2.max_wgroup, 1, kRings[a][0], kRings[a][1]) <= smem_optin;
+                               r2.max_wgroup, 1, ltc ? kRingsT[a][0] : kRings[a][0],
+                               ltc ? kRingsT[a][1] : kRings[a][1], ltc ? r2.lvp : 0, r2.kl_j,
+                               r2.kl_m) <= smem_optin;
+        if (ltc && !fits && opt.leaf_tc != 2) {  // FMA leaves fit in less shared memory
+            build_rat2(lp, r2);
+            for (int a = 0; r2.ok && a < 5 && !fits; ++a)
+                fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
+                                   r2.max_wgroup, 1, kRings[a][0], kRings[a][1], 0, 0, 0) <= smem_optin;
+        }
+        if (opt.leaf_tc == 2 && !(r2.ok && r2.leaf_tc && fits)) {
+            free_plan(P);
+            return set_err(SPN_E_UNSUPPORTED, "leaf_tc not applicable: shared memory");
+        }
         if (r2.ok && fits) {
             std::vector<int32_t> leaf_idx, sum_idx;
             for (int32_t t = 0; t < (int32_t)r2.steps.size(); ++t)
@@ -634,6 +670,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
             P->cert = opt.tc_precision == 0 && std::isfinite(r2.tc_err_1pass);
             P->cert_err = (float)r2.tc_err_1pass;
             P->n_r2leaf = (int32_t)leaf_idx.size();
+            P->leaf_tc = r2.leaf_tc;
             P->n_r2sum = (int32_t)sum_idx.size();
             // (P->smem stays the v1 kernel's: it serves the certification fallback)
             // persistent kernel over many tiles per launch: 8 tiles per CTA
@@ -683,6 +720,15 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     s.fma_per_sample = lp.fma_per_sample;
     s.mufu_per_sample = lp.mufu_per_sample;
     s.tc_flops_per_sample = lp.tc_flops_per_sample;  // algorithmic (one pass)
+    if (P->r2 && P->leaf_tc) {
+        // the leaf layer moved from the FMA pipe (2 per variable and
+        // distribution) to the tensor cores (one GEMM of K = 2V + 1 per region)
+        for (const LStep &st : lp.steps)
+            if (st.type == 0) {
+                s.fma_per_sample -= 2LL * st.n_out * st.n_vars;
+                s.tc_flops_per_sample += 2LL * st.n_out * (2LL * st.n_vars + 1);
+            }
+    }
     s.bytes_per_sample = 4 * (int64_t)g.F + 4 * (int64_t)lp.C + 4;
     s.path = 1;
     s.chunk_samples = chunk;
@@ -695,6 +741,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     s.tc_passes = P->r2 ? 1 : (P->prec == 3 ? 3 : 1);
     s.cert_err = P->r2 ? P->cert_err : 0.0;
     s.certified = P->cert ? 1 : 0;
+    s.leaf_tc = P->r2 && P->leaf_tc ? 1 : 0;
     s.prepare_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     spn_handle *h = new (std::nothrow) spn_handle();
@@ -941,8 +988,10 @@ int spn_prepare(const spn_handle *graph, const spn_prepare_options *opt_in,
     spn_prepare_options opt;
     spn_default_options(&opt);
     if (opt_in) opt = *opt_in;
-    for (int i = 0; i < 5; ++i)
+    for (int i = 0; i < 4; ++i)
         if (opt.reserved[i]) return set_err(SPN_E_ARG, "reserved option fields must be zero");
+    if (opt.leaf_tc < 0 || opt.leaf_tc > 2)
+        return set_err(SPN_E_ARG, "leaf_tc must be 0 (auto), 1 (off) or 2 (force)");
     if (opt.value_space < 0 || opt.value_space > 2)
         return set_err(SPN_E_ARG, "value_space must be 0 (auto), 1 (log2) or 2 (linear)");
     if (opt.value_space == 2 && (opt.compiled_path == 1 || opt.layered_path == 2))
@@ -1248,11 +1297,18 @@ int spn_build_program(const spn_handle *graph, int32_t samples_per_thread, int32
 int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t why_len,
                        int64_t *sizes, int32_t *dims, void *steps, int32_t *vars, float *fparams,
                        void *wimg, int32_t *root_map, double *tc_err_1pass) {
+    return spn_build_layered2_ex(graph, 0, ok, why, why_len, sizes, dims, steps, vars, fparams, wimg,
+                                 root_map, tc_err_1pass);
+}
+
+int spn_build_layered2_ex(const spn_handle *graph, int32_t leaf_tc, int32_t *ok, char *why,
+                          int64_t why_len, int64_t *sizes, int32_t *dims, void *steps, int32_t *vars,
+                          float *fparams, void *wimg, int32_t *root_map, double *tc_err_1pass) {
     if (!valid_graph_handle(graph) || !ok || !sizes || !dims) return set_err(SPN_E_ARG, "bad arguments");
     LayeredPlan lp;
     detect_layered(*graph->graph, lp);
     Rat2Plan p;
-    build_rat2(lp, p);
+    build_rat2(lp, p, leaf_tc != 0);
     *ok = p.ok ? 1 : 0;
     if (why && why_len > 0) {
         strncpy(why, p.why.c_str(), (size_t)why_len - 1);
@@ -1264,9 +1320,9 @@ int spn_build_layered2(const spn_handle *graph, int32_t *ok, char *why, int64_t 
     sizes[3] = (int64_t)p.wimg.size() * 2;
     sizes[4] = (int64_t)p.root_map.size();
     sizes[5] = (int64_t)sizeof(R2Step);
-    const int32_t d[11] = {p.F, p.C, p.I, p.S, p.D, p.gcols, p.kpad_bot, p.kpad_up,
-                           p.max_wgroup, p.max_vars, p.max_blk};
-    memcpy(dims, d, sizeof(d));
+    const int32_t d[14] = {p.F, p.C, p.I, p.S, p.D, p.gcols, p.kpad_bot, p.kpad_up,
+                           p.max_wgroup, p.max_vars, p.max_blk, p.lvp, p.kl_j, p.kl_m};
+    memcpy(dims, d, (leaf_tc ? 14 : 11) * sizeof(int32_t));
     if (tc_err_1pass) *tc_err_1pass = p.tc_err_1pass;
     if (steps) memcpy(steps, p.steps.data(), p.steps.size() * sizeof(R2Step));
     if (vars) memcpy(vars, p.vars.data(), p.vars.size() * 4);

@@ -478,7 +478,7 @@ void detect_layered(const GraphData &g, LayeredPlan &plan, int n_cap) {
 }
 
 // ---------------------------------------------------------------- v2 plan
-void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
+void build_rat2(const LayeredPlan &lp, Rat2Plan &p, bool leaf_tc) {
     p = Rat2Plan();
     auto fail = [&](const std::string &why) {
         p.ok = false;
@@ -535,10 +535,23 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
     // the D activation slots and the C root accumulators
     const int32_t fixed_cols = D * S + p.C;
     const int32_t na_max = std::max(I, S);
-    if (R2_COLS_A + R2_COLS_B + fixed_cols > 512)
+    const int32_t CA = leaf_tc ? R2T_COLS_A : R2_COLS_A, CB = leaf_tc ? R2T_COLS_B : R2_COLS_B;
+    const int32_t CL = leaf_tc ? R2T_COLS_L : 0;
+    if (CA + CB + CL + fixed_cols > 512)
         return fail("TMEM budget: " + std::to_string(fixed_cols) + " activation/root columns");
-    if (na_max > R2_COLS_B) return fail("region wider than an accumulator buffer");
-    p.gcols = R2_COLS_A + R2_COLS_B;
+    if (na_max > CB) return fail("region wider than an accumulator buffer");
+    p.gcols = CA + CB + CL;
+    p.cols_a = CA;
+    p.cols_b = CB;
+    p.leaf_tc = leaf_tc;
+    if (leaf_tc) {
+        int32_t vmax = 0;
+        for (const LStep &st : lp.steps)
+            if (st.type == 0) vmax = std::max(vmax, st.n_vars);
+        p.lvp = (vmax + 3) / 4 * 4;
+        p.kl_j = (2 * p.lvp + 1 + 15) / 16 * 16;
+        p.kl_m = (3 * p.lvp + 15) / 16 * 16;
+    }
     p.ea_max = (na_max + 7) / 8 * 8;
     p.kpad_bot = (I + 15) / 16 * 16;
     p.kpad_up = S > 0 ? (S + 15) / 16 * 16 : 16;
@@ -553,6 +566,74 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
         r.n_out = st.n_out;
         r.slot_out = st.type == 1 ? slot[t] : 0;
         r.root = st.type == 2 ? 1 : 0;
+        if (st.type == 0 && leaf_tc) {
+            // tensor-core leaf layer: centres M_v, the joint and marginal
+            // parameter images (B operand, K-major, N = R2T_COLS_L rows)
+            const int32_t V = st.n_vars, NL = R2T_COLS_L, lvp = p.lvp;
+            r.n_vars = V;
+            r.vars_off = (int64_t)p.vars.size();
+            p.vars.insert(p.vars.end(), lp.vars.begin() + st.vars_off,
+                          lp.vars.begin() + st.vars_off + V);
+            const std::vector<double> &raw = lp.raw[t];
+            while (p.fparams.size() % 4) p.fparams.push_back(0.f);
+            r.blk_off = (int64_t)p.fparams.size();
+            std::vector<float> M(lvp, 0.f);
+            for (int32_t v = 0; v < V; ++v) {  // midpoint of the region's means on variable v
+                double lo = INFINITY, hi = -INFINITY;
+                for (int32_t i = 0; i < I; ++i) {
+                    const double mu = raw[(size_t)V * I + (size_t)v * I + i] / raw[(size_t)v * I + i];
+                    lo = std::min(lo, mu);
+                    hi = std::max(hi, mu);
+                }
+                M[v] = (float)(0.5 * (lo + hi));
+                if (!std::isfinite(M[v])) return fail("leaf tensor cores: non-finite centre");
+            }
+            p.fparams.insert(p.fparams.end(), M.begin(), M.end());
+            r.blk_floats = lvp;
+            // P[k][i]: k = 2v -a^2, 2v+1 2 a b~, then the constant column
+            // sum_v (c_v - b~^2) (joint) or per-variable c_v - b~^2 (marginal)
+            const double K0 = 0.5 * std::log2(M_LN2 / M_PI);  // c_v = log2(a) + K0
+            std::vector<double> Pj((size_t)p.kl_j * NL, 0.0), Pm((size_t)p.kl_m * NL, 0.0);
+            for (int32_t i = 0; i < I; ++i) {
+                double cj = 0.0;
+                for (int32_t v = 0; v < V; ++v) {
+                    const double a = raw[(size_t)v * I + i], b = raw[(size_t)V * I + (size_t)v * I + i];
+                    const double bt = b - a * (double)M[v];
+                    const double pq = -a * a, px = 2.0 * a * bt, pz = std::log2(a) + K0 - bt * bt;
+                    Pj[(size_t)(2 * v) * NL + i] = Pm[(size_t)(2 * v) * NL + i] = pq;
+                    Pj[(size_t)(2 * v + 1) * NL + i] = Pm[(size_t)(2 * v + 1) * NL + i] = px;
+                    Pm[(size_t)(2 * lvp + v) * NL + i] = pz;
+                    cj += pz;
+                }
+                Pj[(size_t)(2 * lvp) * NL + i] = cj;
+            }
+            while (p.wimg.size() % 64) p.wimg.push_back(0);  // 128-byte aligned images
+            r.w_off = (int64_t)p.wimg.size() * 2;
+            r.wbytes_a = (int64_t)NL * p.kl_j * 2;
+            r.wbytes_b = (int64_t)NL * p.kl_m * 2;
+            for (int pass = 0; pass < 2; ++pass) {
+                const std::vector<double> &P = pass ? Pm : Pj;
+                const int32_t K = pass ? p.kl_m : p.kl_j;
+                std::vector<uint16_t> hi((size_t)NL * K, 0), lo((size_t)NL * K, 0);
+                for (int32_t k = 0; k < K; ++k)
+                    for (int32_t n = 0; n < NL; ++n) {
+                        const double v = P[(size_t)k * NL + n];
+                        if (!(std::fabs(v) < 60000.0)) return fail("leaf tensor cores: constant outside f16");
+                        const uint16_t h = f32_to_f16((float)v);
+                        const size_t idx = (size_t)(k / 8) * ((size_t)NL / 8) * 64 + (size_t)(n / 8) * 64 +
+                                           (size_t)(n % 8) * 8 + (size_t)(k % 8);
+                        hi[idx] = h;
+                        lo[idx] = f32_to_f16((float)(v - (double)f16_to_f32(h)));
+                    }
+                p.wimg.insert(p.wimg.end(), hi.begin(), hi.end());
+                p.wimg.insert(p.wimg.end(), lo.begin(), lo.end());
+            }
+            p.max_vars = std::max(p.max_vars, V);
+            p.max_blk = std::max<int32_t>(p.max_blk, (int32_t)r.blk_floats);
+            p.n_leaf++;
+            p.steps.push_back(r);
+            continue;
+        }
         if (st.type == 0) {
             const int32_t V = st.n_vars;
             r.n_vars = V;
@@ -591,7 +672,7 @@ void build_rat2(const LayeredPlan &lp, Rat2Plan &p) {
             while (c > 1 && (c * na + 15) / 16 * 16 > cols) --c;
             return std::max(1, c);
         };
-        const int32_t cap_a = cap(R2_COLS_A), cap_b = cap(R2_COLS_B);
+        const int32_t cap_a = cap(CA), cap_b = cap(CB);
         int32_t spg_a = cap_a, spg_b = cap_b;
         if (n_out <= cap_a + cap_b) {  // one pair: split in proportion to the buffers
             spg_a = std::min(cap_a, (n_out * cap_a + cap_a + cap_b - 1) / (cap_a + cap_b));

@@ -88,12 +88,17 @@ struct R2Step {
     int32_t n_vars;      // LEAF: variables of the region
     int32_t pad_;
     int64_t vars_off;    // LEAF: int32 offset into vars
-    int64_t blk_off;     // LEAF: float offset of the block (a,b)[v][I], C[I]; SUM: kscale[n_out]
+    int64_t blk_off;     // LEAF: float offset of the block (a,b)[v][I], C[I] (tensor-core
+                         // leaves: the per-variable centres M[lvp]); SUM: kscale[n_out]
     int64_t blk_floats;  // LEAF: block size in floats (multiple of 4)
     int64_t w_off;       // SUM: byte offset of the images: per group pair [A hi, A lo, B hi, B lo]
-    int64_t wbytes_a, wbytes_b;  // bytes of one part image of an A / B group
+                         // LEAF (tensor-core leaves): joint image [hi, lo], then marginal [hi, lo]
+    int64_t wbytes_a, wbytes_b;  // bytes of one part image of an A / B group (LEAF: joint / marginal)
 };
 constexpr int R2_COLS_A = 240, R2_COLS_B = 160;  // TMEM accumulator buffers (columns)
+// tensor-core leaf layer: narrower sum accumulators make room for the leaf
+// accumulator (N = 48 >= I) in TMEM
+constexpr int R2T_COLS_A = 160, R2T_COLS_B = 160, R2T_COLS_L = 48;
 
 struct Rat2Plan {
     bool ok = false;
@@ -102,8 +107,18 @@ struct Rat2Plan {
     int32_t max_vars = 0, max_blk = 0;          // largest leaf region / parameter block (floats)
     int32_t kpad_bot = 0, kpad_up = 0;          // K of the BOT / UP contractions (x16)
     int32_t max_wgroup = 0;                     // bytes of the largest (group, part) image
-    int32_t gcols = 0;                          // TMEM columns of both accumulators (A + B)
+    int32_t gcols = 0;                          // TMEM columns before the activation slots
+    int32_t cols_a = 0, cols_b = 0;             // accumulator widths (R2_COLS_* / R2T_COLS_*)
     int32_t ea_max = 0;                         // max(I, S) rounded up to 8
+    // tensor-core leaf layer (leaf_tc): a leaf region's log-densities are one
+    // GEMM L[m, i] = sum_k F[m, k] P[k, i] over the per-sample features
+    // F = (x~^2, x~) per variable (x~ = x - M_v, hi/lo f16 split) plus a
+    // constant column (joint) or per-variable observed indicators
+    // (marginal); P holds -a^2, 2 a b~ and c - b~^2 (PAPER.md L128-167
+    // Gaussian, expanded around the centre M_v: b~ = b - a M_v)
+    bool leaf_tc = false;
+    int32_t lvp = 0;                            // variables per region rounded up to 4
+    int32_t kl_j = 0, kl_m = 0;                 // K of the joint / marginal leaf GEMM (x16)
     std::vector<R2Step> steps;
     std::vector<int32_t> vars;
     std::vector<float> fparams;                 // leaf blocks, then per-sum scale exponents
@@ -122,7 +137,9 @@ struct Rat2Plan {
 
 // Builds the v2 plan from a detected layered plan; fails (ok = false, why)
 // when the structure is outside the v2 kernel's constraints.
-void build_rat2(const LayeredPlan &lp, Rat2Plan &p);
+// leaf_tc: tensor-core leaf layer (fails when a leaf constant or centre is
+// outside the f16 range of the split operands).
+void build_rat2(const LayeredPlan &lp, Rat2Plan &p, bool leaf_tc = false);
 
 // Kernel parameters of rat2_kernel.
 struct R2Params {
@@ -140,6 +157,10 @@ struct R2Params {
     int32_t *argmax;
     int32_t prec;         // 1: one f16 pass; 3: hi/lo split (3 MMAs)
     int32_t max_vars, max_blk, kpad_bot, kpad_up, max_wgroup, gcols, D;
+    // tensor-core leaf layer: K of the leaf GEMM (joint / marginal), vars
+    // rounded up to 4, feature image (hi part, lo part follows) and the
+    // offset of the parameter image inside an input slot
+    int32_t lvp, kl_j, kl_m, off_f, f_bytes, pimg_off;
     int32_t n_in, n_w;    // ring depths: leaf inputs, weight groups
     // shared-memory carve-up (byte offsets, computed on the host)
     int32_t off_in, in_bytes, off_ea, ea_bytes, off_bimg, bimg_bytes, off_uimg, uimg_bytes,

@@ -76,8 +76,19 @@ static_assert(4 * NLG * REG_LEAF + 8 * REG_EPI + 4 * REG_PROD <= (4 * NLG + 12) 
 constexpr int W_EPI0 = 4 * NLG;   // epilogue warps: two per TMEM lane quarter
 constexpr int W_PROD = W_EPI0 + 8, W_MMA = W_PROD + 1, W_WPROD = W_PROD + 2;
 constexpr float EB_SHIFT = 15.f;  // eb' = 2^(b - hb + 15): f16-normal down to eb = 2^-29
-// TMEM accumulators: A = columns [0, R2_COLS_A), B = [R2_COLS_A, +R2_COLS_B);
-// the groups of a step alternate A, B (layered.h R2Step)
+// TMEM accumulators: A = columns [0, CA), B = [CA, CA + CB); the groups of a
+// step alternate A, B (layered.h R2Step).  FMA leaves: 240 + 160; tensor-core
+// leaves (LTC): 160 + 160, then the leaf accumulator (48 columns); the
+// activation slots and root columns follow.  LTC keeps two left/right
+// leaf-output slots (its feature image takes the third one's shared memory).
+template <bool LTC>
+struct Cols {
+    static constexpr int A = LTC ? R2T_COLS_A : R2_COLS_A;
+    static constexpr int B = LTC ? R2T_COLS_B : R2_COLS_B;
+    static constexpr int L = A + B;
+    static constexpr int SLOTS = A + B + (LTC ? R2T_COLS_L : 0);
+    static constexpr int NAB = LTC ? 2 : R2_NAB;
+};
 
 __device__ __forceinline__ float ex2(float x) {
     float y;
@@ -282,7 +293,9 @@ enum {
     B_W_EMPTY = 34,   // [8]
     B_T_FULL = 42,    // [2]
     B_T_EMPTY = 44,   // [2]
-    B_COUNT = 46
+    B_F_FULL = 46,    // tensor-core leaves: feature image written (leaf warps -> leaf MMA)
+    B_LT_FULL = 47,   // tensor-core leaves: leaf accumulator ready (leaf MMA commit -> leaf warps)
+    B_COUNT = 48
 };
 
 struct Smem {
@@ -309,6 +322,12 @@ struct Smem {
     __device__ uint8_t *bimg(int s) const { return base + p.off_bimg + s * p.bimg_bytes; }
     __device__ uint8_t *uimg() const { return base + p.off_uimg; }
     __device__ uint8_t *wbuf(int s) const { return base + p.off_w + s * p.w_bytes; }
+    // tensor-core leaves: feature image (hi part, lo part after it) and the
+    // parameter image inside input slot s
+    __device__ uint8_t *fimg() const { return base + p.off_f; }
+    __device__ uint8_t *in_pimg(int s) const {
+        return reinterpret_cast<uint8_t *>(in_x(s)) + p.pimg_off;
+    }
 };
 
 // ============================================================== LEAF groups
@@ -404,7 +423,11 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
             bar_wait(sm.bar(B_IN_FULL + s), (li / (uint32_t)p.n_in) & 1u);
             pf.mark(0);
             float acc[DPB][SPT];
+#ifdef R2_KO_LEAF  // knockout (critical-path experiments; wrong results): no leaf FMAs
+            leaf_compute<DPB, SPT, MARG>(sm.in_x(s), sm.in_prm(s), 0, I, m0, d0, acc);
+#else
             leaf_compute<DPB, SPT, MARG>(sm.in_x(s), sm.in_prm(s), st.n_vars, I, m0, d0, acc);
+#endif
             // the slot's next fill is an async-proxy (TMA) write: order this
             // warp's generic-proxy reads before the release of the slot
             fence_async_smem();
@@ -487,6 +510,7 @@ __device__ void leaf_role(const R2Params &p, const Smem &sm, const int32_t *leaf
 // Two warps so leaf inputs never queue behind weight groups (the weight
 // ring drains at the pace of the epilogue): warp W_PROD streams each leaf
 // region's feature rows + parameter block, warp W_WPROD every weight group.
+template <bool LTC, bool MARG>
 __device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
                                    int n_leaf, int lane) {
     const int64_t n_tiles = (p.n + RT - 1) / RT;
@@ -504,8 +528,17 @@ __device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int3
             const uint32_t pbytes = (uint32_t)st.blk_floats * 4;
             const uint32_t dst = smem_u32(sm.in_x(s));
             if (lane == 0) {
-                bar_expect_tx(full, (uint32_t)st.n_vars * RT * 4 + pbytes);
-                bulk_g2s(smem_u32(sm.in_prm(s)), p.fparams + st.blk_off, pbytes, full);
+                if constexpr (LTC) {
+                    // centres + the query's parameter image (hi, lo)
+                    const uint32_t ib = 2u * (uint32_t)(MARG ? st.wbytes_b : st.wbytes_a);
+                    bar_expect_tx(full, (uint32_t)st.n_vars * RT * 4 + pbytes + ib);
+                    bulk_g2s(smem_u32(sm.in_prm(s)), p.fparams + st.blk_off, pbytes, full);
+                    bulk_g2s(smem_u32(sm.in_pimg(s)), p.wimg + st.w_off + (MARG ? 2 * st.wbytes_a : 0), ib,
+                             full);
+                } else {
+                    bar_expect_tx(full, (uint32_t)st.n_vars * RT * 4 + pbytes);
+                    bulk_g2s(smem_u32(sm.in_prm(s)), p.fparams + st.blk_off, pbytes, full);
+                }
             }
             __syncwarp();
             for (int v = lane; v < st.n_vars; v += 32) {
@@ -585,11 +618,15 @@ __device__ void weight_producer_role(const R2Params &p, const Smem &sm, const in
                 const uint32_t full = sm.bar(B_W_FULL) + 8u * w_idx;
                 if (lane == 0) {
                     const uint32_t gb = (uint32_t)gr.bytes;
+#ifdef R2_KO_W  // knockout (wrong results): weight slots handed over without copies
+                    bar_arrive(full);
+#else
                     bar_expect_tx(full, gb * parts);
                     const uint8_t *src = p.wimg + st.w_off + gr.off;
                     for (int pt = 0; pt < parts; ++pt)
                         bulk_g2s(smem_u32(sm.wbuf((int)w_idx)) + pt * (uint32_t)p.max_wgroup,
                                  src + (size_t)pt * gb, gb, full);
+#endif
                 }
                 __syncwarp();
                 if (++w_idx == n_w) {
@@ -613,6 +650,7 @@ __device__ __forceinline__ uint64_t desc_hi(uint32_t lbo, uint32_t sbo) {
     return ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
            ((uint64_t)1 << 46);
 }
+template <bool LTC>
 __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps, int n_sum,
                          uint32_t tmem, int lane) {
     const int64_t n_tiles = (p.n + RT - 1) / RT;
@@ -636,8 +674,8 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
             const int G = st.n_groups, ksteps = st.kpad / 16;
             uint32_t a_addr;
             if (bot) {
-                const int ab = (int)(kb % NAB);
-                bar_wait(sm.bar(B_B_FULL + ab), (kb / NAB) & 1u);
+                const int ab = (int)(kb % Cols<LTC>::NAB);
+                bar_wait(sm.bar(B_B_FULL + ab), (kb / Cols<LTC>::NAB) & 1u);
                 a_addr = smem_u32(sm.bimg(ab));
             } else {
                 bar_wait(sm.bar(B_U_FULL), ku & 1u);
@@ -673,7 +711,7 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                         desc_hi(lbo_b, 128) | (uint64_t)(((wbase + wsl * wstride) >> 4) & 0x3FFFu);
                     const uint32_t kw_d = (2 * lbo_b) >> 4;
                     const uint32_t idesc = (1u << 4) | ((uint32_t)(gr.ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
-                    const uint32_t d = tmem + (b ? (uint32_t)R2_COLS_A : 0u);
+                    const uint32_t d = tmem + (b ? (uint32_t)Cols<LTC>::A : 0u);
                     if (gr.ns > 0)
                         for (int kk = 0; kk < ksteps; ++kk) {
                             const uint64_t ad = a_desc + kk * ka_d, wd = w_desc + kk * kw_d;
@@ -721,10 +759,13 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                         idesc[b] = (1u << 4) | ((uint32_t)(gr[b].ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
                     }
                     for (int kk = 0; kk < ksteps; ++kk) {
+#ifdef R2_KO_MMA  // knockout (wrong results): commits only, no tensor-core work
+                        break;
+#endif
 #pragma unroll
                         for (int b = 0; b < 2; ++b) {
                             if (gr[b].ns > 0) {
-                                const uint32_t d = tmem + (b ? (uint32_t)R2_COLS_A : 0u);
+                                const uint32_t d = tmem + (b ? (uint32_t)Cols<LTC>::A : 0u);
                                 const uint64_t ad = a_desc + kk * ka_d, wd = w_desc[b] + kk * kw_d[b];
                                 umma_f16(d, ad, wd, idesc[b], kk > 0);
                                 if (split) {
@@ -743,7 +784,7 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                 __syncwarp();
             }
 #endif
-            if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb % NAB) : B_U_EMPTY));
+            if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb % Cols<LTC>::NAB) : B_U_EMPTY));
             __syncwarp();
             if (bot) ++kb;
             else ++ku;
@@ -799,7 +840,7 @@ __device__ __forceinline__ float dot4(const float (&ea)[NA], const float *t) {
     return ((q[0].x + q[0].y) + (q[1].x + q[1].y)) + ((q[2].x + q[2].y) + (q[3].x + q[3].y));
 }
 
-template <int NA, bool ROOT>
+template <int NA, bool ROOT, bool LTC>
 __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const SumStep &st,
                                            const float (&ear)[NA], float shift, uint32_t lane_base,
                                            uint32_t out_col, uint32_t col_root, uint32_t &tp,
@@ -830,7 +871,7 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         bar_wait(sm.bar(B_T_FULL + b), (tp & 1u));
         pf.mark(2);
         tc_fence_after();
-        const uint32_t acc = lane_base + (b ? (uint32_t)R2_COLS_A : 0u);
+        const uint32_t acc = lane_base + (b ? (uint32_t)Cols<LTC>::A : 0u);
         const int ns = gr.ns;
         const int mine = ns > h ? (ns - h + 1) / 2 : 0;  // this warp's sums: h, h + 2, ...
         for (int k0 = 0; k0 < mine; k0 += QB) {
@@ -868,7 +909,7 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         bar_wait(sm.bar(B_T_FULL + b), (tp & 1u));
         pf.mark(2);
         tc_fence_after();
-        const uint32_t acc = lane_base + (b ? (uint32_t)R2_COLS_A : 0u);
+        const uint32_t acc = lane_base + (b ? (uint32_t)Cols<LTC>::A : 0u);
         const int ns = gr.ns;
         // batches of PB sums (one tcgen05.ld of PB * NA <= 80 columns, one
         // wait): the sums' dot products are independent chains the scheduler
@@ -886,8 +927,13 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
                 bar_arrive(sm.bar(B_T_EMPTY + b));  // all of this group's columns are in registers
             }
             float val[PB];
+#ifdef R2_KO_EPI  // knockout (wrong results): no stage-2 dot products
+#pragma unroll
+            for (int k = 0; k < PB; ++k) val[k] = t[k * NA] + ear[k];
+#else
 #pragma unroll
             for (int k = 0; k < PB; ++k) val[k] = dot4(ear, t + k * NA);
+#endif
 #pragma unroll
             for (int k = 0; k < PB; ++k)
                 if (sl + k < ns) fin(gr.s0 + sl + k, val[k], kv[k]);
@@ -900,14 +946,194 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
     }
 }
 
-template <int I, int S, bool MARG>
+// ============================================================== LEAF on tensor cores (LTC)
+// Gaussian leaf region (log2 units): L[m, i] = sum_v
+// c_vi - (a_vi x_mv - b_vi)^2.  Expanded around a per-variable centre M_v
+// (x~ = x - M_v, b~ = b - a M_v) it is one GEMM over the features
+//   F[m] = (x~_0^2, x~_0, x~_1^2, x~_1, ..., 1)            joint
+//   F[m] = (x~_0^2, x~_0, ..., z_0, z_1, ...)               marginal (z_v = x_v observed;
+//                                                            a missing x_v has x~ = 0)
+// against P = (-a^2, 2 a b~, ..., c - b~^2) (layered.cpp build_rat2).  The
+// operands are split hi/lo in f16 (F = F_h + F_l, P = P_h + P_l) and
+// L = F_h P_h + F_h P_l + F_l P_h accumulates in fp32 in TMEM: about 2^-21
+// relative per term, fp32-class like the FMA leaves it replaces.  A
+// sample whose |x~| exceeds 240 (f16 range of x~^2) or is infinite gets a NaN
+// shift, hence NaN outputs, which the certification recomputes in v1.
+//
+// Leaf warps (thread = sample m = TMEM lane): per region l, read back
+// L(l-1), build F(l) (the single feature image is free once L(l-1) is
+// complete), hand it to the leaf MMA warp, then the shift / exps of l-1
+// while the tensor core computes L(l).
+template <int I, bool MARG>
+__device__ void leaf_tc_role(const R2Params &p, const Smem &sm, const int32_t *leaf_steps,
+                             int n_leaf, uint32_t tmem, int warp, int lane) {
+    static_assert(I % 8 == 0, "leaf width");
+    constexpr int NAB2 = Cols<true>::NAB;
+    const int m = warp * 32 + lane;
+    const uint32_t lacc = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)Cols<true>::L;
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    uint8_t *fh = sm.fimg();
+    uint8_t *fl = fh + p.f_bytes;
+    const int nq = p.lvp >> 2;
+    const int zcol = 2 * p.lvp;
+    const uint32_t n_in = (uint32_t)p.n_in;
+    uint32_t li = 0, s = 0, sph = 0;
+    bool bad_prev = false;
+    float L[I];
+    Prof pf(sm.prof(0), p.prof != nullptr);  // 0 wait input, 1 build F, 2 wait L, 3 wait output slot, 4 exps + write
+    // shift / exps of region lj (values in L) into its left / right slot
+    auto exps = [&](uint32_t lj, bool bad) {
+        const bool side_b = (lj & 1u) != 0;
+        const uint32_t j = lj >> 1;
+        float h = L[0];
+#pragma unroll
+        for (int i = 1; i < I; ++i) h = maxnan(h, L[i]);
+        if (bad) h = CUDART_NAN_F;
+        const int ab = (int)(j % NAB2);
+        const uint32_t ph = (j / NAB2) & 1u;
+        bar_wait(sm.bar(B_A_EMPTY + ab), ph ^ 1u);
+        if (side_b) bar_wait(sm.bar(B_B_EMPTY + ab), ph ^ 1u);
+        pf.mark(3);
+        if (!side_b) {
+            float *ea = sm.ea(ab);
+            const float hc = fmaxf(h, -1e30f);
+#pragma unroll
+            for (int i = 0; i < I; ++i) ea[i * RT + m] = ex2(L[i] - hc);
+            sm.ha(ab)[m] = h;
+            bar_arrive(sm.bar(B_A_FULL + ab));
+        } else {
+            uint8_t *img = sm.bimg(ab);
+            const float hc = fmaxf(h, -1e30f) - EB_SHIFT;
+#pragma unroll
+            for (int i = 0; i < I; i += 8)
+                *reinterpret_cast<uint4 *>(img + img_off(m, i)) =
+                    make_uint4(pack_h2(ex2(L[i] - hc), ex2(L[i + 1] - hc)),
+                               pack_h2(ex2(L[i + 2] - hc), ex2(L[i + 3] - hc)),
+                               pack_h2(ex2(L[i + 4] - hc), ex2(L[i + 5] - hc)),
+                               pack_h2(ex2(L[i + 6] - hc), ex2(L[i + 7] - hc)));
+            sm.hb(ab)[m] = h - EB_SHIFT;
+            fence_async_smem();
+            bar_arrive(sm.bar(B_B_FULL + ab));
+        }
+        pf.mark(4);
+    };
+    auto read_l = [&](uint32_t lj) {
+        bar_wait(sm.bar(B_LT_FULL), lj & 1u);
+        tc_fence_after();
+        ld_cols<I>(lacc, L);
+        tmem_wait_ld();
+        pf.mark(2);
+    };
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int l = 0; l < n_leaf; ++l, ++li) {
+            const int V = __ldg(&p.steps[__ldg(leaf_steps + l)].n_vars);
+            bar_wait(sm.bar(B_IN_FULL + (int)s), sph);
+            pf.mark(0);
+            if (li > 0) read_l(li - 1);  // also: the feature image is free again
+            const float *xs = sm.in_x((int)s);
+            const float *Mv = sm.in_prm((int)s);
+            float amax = 0.f;
+            for (int c = 0; c < nq; ++c) {
+                const float4 M4 = *reinterpret_cast<const float4 *>(Mv + 4 * c);
+                const float mm[4] = {M4.x, M4.y, M4.z, M4.w};
+                uint32_t hw[4], lw[4];
+                float zf[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int v = 4 * c + k;
+                    float xt = (v < V ? xs[v * RT + m] : mm[k]) - mm[k];
+                    float z = v < V ? 1.f : 0.f;
+                    if constexpr (MARG) {
+                        const bool nan = xt != xt;
+                        xt = nan ? 0.f : xt;
+                        z = nan ? 0.f : z;
+                    }
+                    amax = fmaxf(amax, fabsf(xt));
+                    const float q = xt * xt;
+                    hw[k] = pack_h2(q, xt);
+                    const float2 hf = __half22float2(*reinterpret_cast<const __half2 *>(&hw[k]));
+                    lw[k] = pack_h2(q - hf.x, xt - hf.y);
+                    zf[k] = z;
+                }
+                const uint32_t o = img_off(m, 8 * c);
+                *reinterpret_cast<uint4 *>(fh + o) = make_uint4(hw[0], hw[1], hw[2], hw[3]);
+                *reinterpret_cast<uint4 *>(fl + o) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+                if constexpr (MARG)
+                    *reinterpret_cast<uint2 *>(fh + img_off(m, zcol + 4 * c)) =
+                        make_uint2(pack_h2(zf[0], zf[1]), pack_h2(zf[2], zf[3]));
+            }
+            const bool bad = !(amax <= 240.f);
+            fence_async_smem();  // the feature image is read by the tensor core (async proxy)
+            tc_fence_before();   // ... and the tcgen05.ld of L(l-1) is complete
+            bar_arrive(sm.bar(B_F_FULL));
+            pf.mark(1);
+            if (li > 0) exps(li - 1, bad_prev);
+            bad_prev = bad;
+            if (++s == n_in) {
+                s = 0;
+                sph ^= 1u;
+            }
+        }
+    }
+    if (li > 0) {
+        read_l(li - 1);
+        exps(li - 1, bad_prev);
+    }
+}
+
+// Leaf MMA warp (LTC): L = F_h P_h + F_h P_l + F_l P_h (M = 128, N = 48,
+// K = kl) into the leaf accumulator; the commit releases the input slot
+// (the parameter image) and signals the leaf warps.  A second issuing warp
+// keeps the leaf GEMMs off the sum-layer MMA warp's chain.
+template <bool MARG>
+__device__ void leaf_mma_role(const R2Params &p, const Smem &sm, int n_leaf, uint32_t tmem,
+                              int lane) {
+    constexpr uint32_t NL = R2T_COLS_L;
+    const int64_t n_tiles = (p.n + RT - 1) / RT;
+    const uint32_t d = tmem + (uint32_t)Cols<true>::L;
+    const uint32_t idesc = (1u << 4) | ((NL >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
+    const uint64_t a_hi = desc_hi(RT * 16, 128), b_hi = desc_hi(NL * 16, 128);
+    const int kl = MARG ? p.kl_m : p.kl_j;
+    const int ks = kl >> 4, ks_lo = (2 * p.lvp + 15) >> 4;
+    const uint32_t ka_d = (2 * RT * 16) >> 4, kb_d = (2 * NL * 16) >> 4;
+    const uint32_t fa = smem_u32(sm.fimg()), fl = fa + (uint32_t)p.f_bytes;
+    const uint32_t pbytes = NL * (uint32_t)kl * 2;
+    const uint32_t n_in = (uint32_t)p.n_in;
+    uint32_t li = 0, s = 0, sph = 0;
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        for (int l = 0; l < n_leaf; ++l, ++li) {
+            bar_wait(sm.bar(B_F_FULL), li & 1u);
+            bar_wait(sm.bar(B_IN_FULL + (int)s), sph);  // the parameter image has landed
+            tc_fence_after();
+            if (lane == 0) {
+                const uint32_t pa = smem_u32(sm.in_pimg((int)s)), pl = pa + pbytes;
+                const uint64_t A = a_hi | (uint64_t)((fa >> 4) & 0x3FFFu);
+                const uint64_t Al = a_hi | (uint64_t)((fl >> 4) & 0x3FFFu);
+                const uint64_t B = b_hi | (uint64_t)((pa >> 4) & 0x3FFFu);
+                const uint64_t Bl = b_hi | (uint64_t)((pl >> 4) & 0x3FFFu);
+                for (int kk = 0; kk < ks; ++kk) umma_f16(d, A + kk * ka_d, B + kk * kb_d, idesc, kk > 0);
+                for (int kk = 0; kk < ks; ++kk) umma_f16(d, A + kk * ka_d, Bl + kk * kb_d, idesc, 1);
+                for (int kk = 0; kk < ks_lo; ++kk) umma_f16(d, Al + kk * ka_d, B + kk * kb_d, idesc, 1);
+                umma_commit(sm.bar(B_LT_FULL));
+                umma_commit(sm.bar(B_IN_EMPTY + (int)s));
+            }
+            __syncwarp();
+            if (++s == n_in) {
+                s = 0;
+                sph ^= 1u;
+            }
+        }
+    }
+}
+
+template <int I, int S, bool MARG, bool LTC>
 __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *sum_steps,
                               int n_sum, uint32_t tmem, int warp, int lane) {
     const int qd = warp & 3;
     const int h = (warp - W_EPI0) >> 2;  // 0: groups in accumulator A, 1: in accumulator B
     const int m = qd * 32 + lane;
     const uint32_t lane_base = tmem + ((uint32_t)(qd * 32) << 16);
-    const uint32_t col_slots = (uint32_t)(R2_COLS_A + R2_COLS_B);
+    const uint32_t col_slots = (uint32_t)Cols<LTC>::SLOTS;
     // the two warps of a lane quarter exchange activation slots / root
     // columns through TMEM: wait for own stores, then a 64-thread barrier
     auto pair_sync = [&]() {
@@ -934,8 +1160,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
             const uint32_t out_col = col_slots + (uint32_t)((es.slot_out - 1) * S);
             if (es.type == 1) {
                 // BOT: ea from leaf group 0, hb from leaf group 1
-                const int ab = (int)(kb % NAB);
-                const uint32_t ph = (kb / NAB) & 1u;
+                const int ab = (int)(kb % Cols<LTC>::NAB);
+                const uint32_t ph = (kb / Cols<LTC>::NAB) & 1u;
                 bar_wait(sm.bar(B_A_FULL + ab), ph);
                 bar_wait(sm.bar(B_B_FULL + ab), ph);
                 pf.mark(0);
@@ -946,8 +1172,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 const float shift = sm.ha(ab)[m] + sm.hb(ab)[m];
                 bar_arrive(sm.bar(B_A_EMPTY + ab));
                 ++kb;
-                if (es.root) sum_groups<I, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
-                else sum_groups<I, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                if (es.root) sum_groups<I, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                else sum_groups<I, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
             } else {
                 // UP: children in activation slots; B side -> f16 image, A side -> registers
                 float vb[SU], ear[SU];
@@ -987,8 +1213,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 for (int i = 0; i < SU; ++i) ear[i] = ex2(ear[i] - hac);
                 const float shift = ha + hb - EB_SHIFT;
                 pf.mark(1);
-                if (es.root) sum_groups<SU, true>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
-                else sum_groups<SU, false>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                if (es.root) sum_groups<SU, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                else sum_groups<SU, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
             }
             tmem_wait_st();
         }
@@ -1015,6 +1241,9 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
             const float av = fabsf(v);
             if (av < CUDART_INF_F && !(p.cert_err <= p.cert_tol * fmaxf(1.f, av - p.cert_err)))
                 cert = false;
+            // tensor-core leaves: NaN marks an input outside the split operands'
+            // range (or a NaN input, recomputed alike)
+            if (LTC && v != v) cert = false;
         }
         if (row < p.n && p.argmax) p.argmax[row] = best;
         if (row < p.n && p.flag_count && !cert) p.flag_idx[atomicAdd(p.flag_count, 1)] = p.row0 + row;
@@ -1022,7 +1251,7 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
     }
 }
 
-template <int I, int S, bool MARG>
+template <int I, int S, bool MARG, bool LTC>
 __global__ void __launch_bounds__(NTHREADS, 1)
     rat2_kernel(const R2Params p, const int32_t *__restrict__ leaf_steps, int n_leaf,
                 const int32_t *__restrict__ sum_steps, int n_sum) {
@@ -1041,14 +1270,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     if (tid == 0) {
         for (int i = 0; i < 4; ++i) {
             bar_init(sm.bar(B_IN_FULL + i), 1);
-            bar_init(sm.bar(B_IN_EMPTY + i), WPG);  // the warps of one leaf group
+            // the warps of one leaf group (LTC: the leaf MMA's commit)
+            bar_init(sm.bar(B_IN_EMPTY + i), LTC ? 1 : WPG);
         }
         for (int i = 0; i < 8; ++i) {
             bar_init(sm.bar(B_W_FULL + i), 1);
             bar_init(sm.bar(B_W_EMPTY + i), 1);
         }
-        for (int i = 0; i < NAB; ++i) {
-            bar_init(sm.bar(B_A_FULL + i), WPG * 32);  // the threads of one leaf group
+        for (int i = 0; i < Cols<LTC>::NAB; ++i) {
+            bar_init(sm.bar(B_A_FULL + i), WPG * 32);  // the threads of one leaf group (LTC: 128)
             bar_init(sm.bar(B_A_EMPTY + i), 256);  // both epilogue warps of each quarter
             bar_init(sm.bar(B_B_FULL + i), WPG * 32);
             bar_init(sm.bar(B_B_EMPTY + i), 1);
@@ -1059,12 +1289,24 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         bar_init(sm.bar(B_U_FULL), 128);
         bar_init(sm.bar(B_U_EMPTY), 1);
+        bar_init(sm.bar(B_F_FULL), 128);
+        bar_init(sm.bar(B_LT_FULL), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         for (int k = 0; k < 32; ++k) sm.prof(0)[k] = 0;
     }
     // zero the operand images once (the K padding columns stay zero)
-    for (int i = tid * 16; i < NAB * p.bimg_bytes + p.uimg_bytes; i += NTHREADS * 16)
+    for (int i = tid * 16; i < Cols<LTC>::NAB * p.bimg_bytes + p.uimg_bytes; i += NTHREADS * 16)
         *reinterpret_cast<uint4 *>(base + p.off_bimg + i) = make_uint4(0, 0, 0, 0);
+    if constexpr (LTC) {
+        static_assert(NLG == 1, "tensor-core leaves: one leaf warpgroup (thread = sample)");
+        // feature image: zero (K padding, lo part of the constant columns),
+        // joint: the constant column 2 lvp = 1
+        for (int i = tid * 16; i < 2 * p.f_bytes; i += NTHREADS * 16)
+            *reinterpret_cast<uint4 *>(sm.fimg() + i) = make_uint4(0, 0, 0, 0);
+        __syncthreads();
+        if (!MARG && tid < RT)
+            *reinterpret_cast<uint16_t *>(sm.fimg() + img_off(tid, 2 * p.lvp)) = 0x3C00u;  // f16 1.0
+    }
     fence_async_smem();
     tc_fence_before();
     __syncthreads();
@@ -1078,15 +1320,18 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     else if (REG_LEAF > LAUNCH_REGS)
         asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(REG_LEAF));
     if (warp < W_EPI0) {
-        leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
+        if constexpr (LTC) leaf_tc_role<I, MARG>(p, sm, leaf_steps, n_leaf, tmem, warp, lane);
+        else leaf_role<I / 4, MARG>(p, sm, leaf_steps, n_leaf, warp, lane);
     } else if (warp < W_PROD) {
-        epilogue_role<I, S, MARG>(p, sm, sum_steps, n_sum, tmem, warp, lane);
+        epilogue_role<I, S, MARG, LTC>(p, sm, sum_steps, n_sum, tmem, warp, lane);
     } else if (warp == W_PROD) {
-        leaf_producer_role(p, sm, leaf_steps, n_leaf, lane);
+        leaf_producer_role<LTC, MARG>(p, sm, leaf_steps, n_leaf, lane);
     } else if (warp == W_MMA) {
-        mma_role(p, sm, sum_steps, n_sum, tmem, lane);
+        mma_role<LTC>(p, sm, sum_steps, n_sum, tmem, lane);
     } else if (warp == W_WPROD) {
         weight_producer_role(p, sm, sum_steps, n_sum, lane);
+    } else if (LTC && warp == W_WPROD + 1) {
+        leaf_mma_role<MARG>(p, sm, n_leaf, tmem, lane);
     }
     tc_fence_before();
     __syncthreads();
@@ -1109,8 +1354,10 @@ bool rat2_supported_shape(int I, int S) {
 
 // host: shared-memory carve-up for ring depths (n_in, n_w); returns bytes
 int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int kpad_up,
-                int max_wgroup, int prec, int n_in, int n_w) {
+                int max_wgroup, int prec, int n_in, int n_w, int lvp, int kl_j, int kl_m) {
     const int parts = prec == 3 ? 2 : 1;
+    const bool ltc = lvp > 0;  // tensor-core leaves
+    const int nab = ltc ? r2::Cols<true>::NAB : r2::Cols<false>::NAB;
     auto up = [](int x, int a) { return (x + a - 1) / a * a; };
     int off = 0;
     p.off_bar = off;
@@ -1118,15 +1365,20 @@ int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int
     off = up(off, 128);
     p.n_in = n_in;
     p.in_bytes = up(max_vars * r2::RT * 4 + max_blk * 4, 128);
+    p.lvp = lvp;
+    p.kl_j = kl_j;
+    p.kl_m = kl_m;
+    p.pimg_off = p.in_bytes;
+    if (ltc) p.in_bytes += 2 * R2T_COLS_L * std::max(kl_j, kl_m) * 2;  // parameter image hi + lo
     p.off_in = off;
     off += n_in * p.in_bytes;
     p.ea_bytes = up((I + 2) * r2::RT * 4, 128);
     p.off_ea = off;
-    off += r2::NAB * p.ea_bytes;
+    off += nab * p.ea_bytes;
     off = up(off, 1024);
     p.bimg_bytes = r2::RT * kpad_bot * 2 * parts;
     p.off_bimg = off;
-    off += r2::NAB * p.bimg_bytes;
+    off += nab * p.bimg_bytes;
     p.uimg_bytes = r2::RT * kpad_up * 2 * parts;
     p.off_uimg = off;  // contiguous with the B images (zeroed together)
     off += p.uimg_bytes;
@@ -1135,6 +1387,9 @@ int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int
     p.w_bytes = up(max_wgroup * parts, 1024);
     p.off_w = off;
     off += n_w * p.w_bytes;
+    p.f_bytes = ltc ? r2::RT * std::max(kl_j, kl_m) * 2 : 0;  // feature image: hi, lo
+    p.off_f = off;
+    off += 2 * p.f_bytes;
     p.smem_bytes = off + 1024;  // alignment slack of the dynamic base
     return p.smem_bytes;
 }
@@ -1142,9 +1397,11 @@ int rat2_layout(R2Params &p, int I, int max_vars, int max_blk, int kpad_bot, int
 cudaError_t rat2_launch(const R2Params &p, const int32_t *leaf_steps, int n_leaf,
                         const int32_t *sum_steps, int n_sum, bool marg, int grid, cudaStream_t st) {
     void (*fn)(const R2Params, const int32_t *, int, const int32_t *, int) = nullptr;
+    const bool ltc = p.lvp > 0;
 #define R2_CASE(I_, S_)                                                                          \
     if (p.I == I_ && (p.S == S_ || (p.S == 0 && 2 * S_ == I_)))                                  \
-        fn = marg ? r2::rat2_kernel<I_, S_, true> : r2::rat2_kernel<I_, S_, false>;
+        fn = ltc ? (marg ? r2::rat2_kernel<I_, S_, true, true> : r2::rat2_kernel<I_, S_, false, true>) \
+                 : (marg ? r2::rat2_kernel<I_, S_, true, false> : r2::rat2_kernel<I_, S_, false, false>);
     R2_CASE(8, 4) R2_CASE(16, 8) R2_CASE(40, 20) R2_CASE(32, 16) R2_CASE(16, 16) R2_CASE(48, 24)
 #undef R2_CASE
     if (!fn) return cudaErrorInvalidConfiguration;

@@ -1,6 +1,6 @@
 """GPU check of the v2 layered kernel (rat2.cu): parity against the fp64
 oracle on small RAT-SPNs and a C4 sample, then timings of v1 / v2 on C4 / C5.
-usage: python scripts/r2_check.py [parity|time|all]"""
+usage: python scripts/r2_check.py [parity|time|time1|ltc|ltctime|all]"""
 import os
 import sys
 import time
@@ -94,3 +94,56 @@ if what in ("time", "all"):
             if kern == 1:
                 print("   v1 vs v2(prec1) max abs diff", float((out - o1).abs().max()), flush=True)
             P.close()
+
+if what == "ltc":   # tensor-core leaves (leaf_tc): parity small shapes + C4 sample, joint / marginal
+    shapes = [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (24, 1, 1, 4, 8, 2), (96, 4, 2, 20, 40, 10)]
+    for shape in shapes:
+        F, D, R, S, I, C = shape
+        g = rat_spn(7, F=F, D=D, R=R, S=S, I=I, C=C)
+        x, _ = ancestral_sample(g, 1000, 3)
+        xm = nan_mask(x, 0.2, 4)
+        ref, _ = oracle_eval(g, x)
+        refm, _ = oracle_eval(g, xm, marginal=True)
+        for ltc in (2, 1):
+            P = spnb.Plan(spnb.Graph(g), layered_path=2, layered_kernel=2, leaf_tc=ltc)
+            out, am = P.infer(torch.from_numpy(x).cuda())
+            outm, _ = P.infer(torch.from_numpy(xm).cuda(), marginal=True)
+            torch.cuda.synchronize()
+            print("shape", shape, "leaf_tc", P.info()["leaf_tc"], "err", err(out.cpu().numpy(), ref),
+                  "marg err", err(outm.cpu().numpy(), refm), flush=True)
+    g = config_graph("C4")
+    x, _ = ancestral_sample(g, 300, 4002)
+    ref, _ = oracle_eval(g, x)
+    for ltc in (2, 1):
+        P = spnb.Plan(spnb.Graph(g), leaf_tc=ltc)
+        out, am = P.infer(torch.from_numpy(x).cuda())
+        torch.cuda.synchronize()
+        o = out.cpu().numpy()
+        print("C4 leaf_tc", P.info()["leaf_tc"], "err", err(o, ref), "max abs", float(np.abs(o - ref).max()),
+              "argmax agree", float((am.cpu().numpy() == ref.argmax(1)).mean()), flush=True)
+
+if what == "ltctime":   # certified v2, tensor-core leaves vs FMA leaves
+    for cfg, n in (("C4", 100_000), ("C5", 18944 * 16)):
+        g = config_graph(cfg)
+        G = spnb.Graph(g)
+        xd = bench.device_uniform(n, g.n_features, 4002, 0, torch.device("cuda"))
+        outs = {}
+        for ltc in (2, 1):
+            P = spnb.Plan(G, leaf_tc=ltc)
+            out, am = P.infer(xd)
+            torch.cuda.synchronize()
+            ts = []
+            for _ in range(3):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                P.infer(xd, out=out, argmax=am)
+                e1.record()
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            outs[ltc] = out.clone()
+            print(cfg, "leaf_tc", P.info()["leaf_tc"], "ms", round(min(ts), 3), "samples/s",
+                  f"{n / min(ts) * 1e3:.3e}", "smem", P.info()["smem_bytes"], flush=True)
+            P.close()
+        d = (outs[2] - outs[1]).abs()
+        print(cfg, "tc vs fma leaves: max abs diff", float(d.max()), "rel",
+              float((d / outs[1].abs().clamp(min=1)).max()), flush=True)

@@ -54,6 +54,42 @@ def _decode_weights(plan, st, prec):
     return W
 
 
+def _leaf_tc(plan, st, xd, marginal):
+    """Tensor-core leaf variant: L[i, m] = sum_k F[m, k] P[k, i] with the
+    features F = (x~^2, x~ per variable; 1 or the observed indicators) and
+    the parameter image decoded from the plan, both split hi/lo in f16 and
+    multiplied as F_h P_h + F_h P_l + F_l P_h (the kernel's three passes)."""
+    I, lvp = plan["I"], plan["lvp"]
+    V = int(st["n_vars"])
+    N = xd.shape[0]
+    NL = 48
+    K = plan["kl_m"] if marginal else plan["kl_j"]
+    fp = plan["fparams"].astype(np.float64)
+    M = fp[int(st["blk_off"]):int(st["blk_off"]) + lvp]
+    off = int(st["w_off"]) // 2 + (2 * int(st["wbytes_a"]) // 2 if marginal else 0)
+    part = NL * K
+    idx = np.array([[_img_index(n, k, NL) for n in range(NL)] for k in range(K)])
+    Ph = plan["wimg"][off:off + part].astype(np.float64)[idx]
+    Pl = plan["wimg"][off + part:off + 2 * part].astype(np.float64)[idx]
+    F = np.zeros((N, K))
+    for v in range(V):
+        xv = xd[:, int(plan["vars"][int(st["vars_off"]) + v])]
+        xt = (xv.astype(np.float32) - np.float32(M[v])).astype(np.float64)
+        if marginal:
+            obs = ~np.isnan(xt)
+            xt = np.where(obs, xt, 0.0)
+            F[:, 2 * lvp + v] = obs
+        F[:, 2 * v] = xt * xt
+        F[:, 2 * v + 1] = xt
+    if not marginal:
+        F[:, 2 * lvp] = 1.0
+    Fh = F.astype(np.float16).astype(np.float64)
+    Fl = (F - Fh).astype(np.float16).astype(np.float64)
+    Fl[:, 2 * lvp:] = 0.0   # constant / indicator columns are exact
+    L = Fh @ Ph + Fh @ Pl + Fl @ Ph
+    return L[:, :I].T
+
+
 def emulate_layered2(plan: dict, x: np.ndarray, marginal: bool = False, prec: int = 3):
     steps, vars_, fp = plan["steps"], plan["vars"], plan["fparams"].astype(np.float64)
     C, I = plan["C"], plan["I"]
@@ -66,6 +102,9 @@ def emulate_layered2(plan: dict, x: np.ndarray, marginal: bool = False, prec: in
     with np.errstate(invalid="ignore", divide="ignore", over="ignore"):
         for st in steps:
             t = int(st["type"])
+            if t == 0 and plan.get("leaf_tc"):
+                pending.append(_leaf_tc(plan, st, xd, marginal))
+                continue
             if t == 0:
                 V = int(st["n_vars"])
                 blk = fp[int(st["blk_off"]):int(st["blk_off"]) + int(st["blk_floats"])]

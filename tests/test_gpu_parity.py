@@ -252,11 +252,34 @@ def test_layered_rat_small_matches_oracle(shape, kernel):
     F, D, R, S, I, C = shape
     g = rat_spn(11, F=F, D=D, R=R, S=S, I=I, C=C)
     x, _ = ancestral_sample(g, 1000, 12)
-    for prec in ((0, 1) if kernel == 2 else (2,)):
-        err, P = _parity(g, x, layered_path=2, tc_precision=prec, layered_kernel=kernel)
-        assert P.info()["path"] == 1 and P.info()["layered_kernel"] == kernel
+    # v2: certified with tensor-core leaves (leaf_tc 2), certified with FMA
+    # leaves (auto), raw single pass (FMA leaves); v1: hi/lo
+    for prec, ltc in (((0, 2), (0, 0), (1, 0)) if kernel == 2 else ((2, 0),)):
+        err, P = _parity(g, x, layered_path=2, tc_precision=prec, layered_kernel=kernel, leaf_tc=ltc)
+        info = P.info()
+        assert info["path"] == 1 and info["layered_kernel"] == kernel
+        assert info["leaf_tc"] == (1 if ltc == 2 else 0)
         _parity(g, nan_mask(x, 0.2, 13), marginal=True, layered_path=2, tc_precision=prec,
-                layered_kernel=kernel)
+                layered_kernel=kernel, leaf_tc=ltc)
+
+
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (128, 3, 2, 20, 40, 10)])
+def test_layered_leaf_tc_out_of_range_inputs(shape):
+    """Tensor-core leaves: inputs outside the f16 split's range (|x - M| > 240,
+    +-inf) and NaN in a joint query are recomputed by the certification
+    (v1, FMA leaves); every row matches the oracle (NaN / -inf included)."""
+    F, D, R, S, I, C = shape
+    g = rat_spn(15, F=F, D=D, R=R, S=S, I=I, C=C)
+    x, _ = ancestral_sample(g, 3000, 16)
+    rng = np.random.default_rng(17)
+    rows = rng.choice(len(x), 60, replace=False)
+    cols = rng.integers(0, F, size=60)
+    vals = np.array([1e3, -5e2, 300.0, np.inf, -np.inf, np.nan] * 10, dtype=np.float32)
+    x[rows, cols] = vals
+    err, P = _parity(g, x, layered_path=2, layered_kernel=2, leaf_tc=2)
+    assert P.info()["leaf_tc"] == 1
+    xm = nan_mask(x, 0.2, 18)
+    _parity(g, xm, marginal=True, layered_path=2, layered_kernel=2, leaf_tc=2)
 
 
 def test_layered_matches_generic_path():

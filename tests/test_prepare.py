@@ -293,6 +293,32 @@ def test_layered2_plan_matches_oracle(shape):
         assert (np.abs(em1 - ref) / np.maximum(1.0, np.abs(ref))).max() < 5e-3
 
 
+@pytest.mark.parametrize("shape", [(32, 2, 2, 4, 8, 3), (64, 3, 3, 8, 16, 5), (24, 1, 1, 4, 8, 2),
+                                   (96, 4, 2, 20, 40, 10)])
+def test_layered2_leaf_tc_plan_matches_oracle(shape):
+    """Tensor-core leaf variant of the v2 plan (centres, joint / marginal
+    parameter images; narrower sum accumulators) emulated with the kernel's
+    hi/lo f16 operand split equals the oracle: the expanded Gaussian
+    (x~^2, x~, constant) restates the leaf density exactly and the split
+    keeps it fp32-class."""
+    from spn_inputs import rat_spn
+    from tests.layered2_emulator import emulate_layered2
+    F, D, R, S, I, C = shape
+    g = rat_spn(7, F=F, D=D, R=R, S=S, I=I, C=C)
+    plan, why = spnb.build_layered2(spnb.Graph(g), leaf_tc=True)
+    assert plan is not None, why
+    assert plan["lvp"] % 4 == 0 and plan["lvp"] >= plan["max_vars"]
+    assert plan["kl_j"] % 16 == 0 and plan["kl_j"] >= 2 * plan["lvp"] + 1
+    assert plan["kl_m"] % 16 == 0 and plan["kl_m"] >= 3 * plan["lvp"]
+    assert plan["gcols"] == 160 + 160 + 48
+    x, _ = ancestral_sample(g, 120, 3)
+    for marg, xx in ((False, x), (True, nan_mask(x, 0.2, 4))):
+        ref, _ = oracle_eval(g, xx, marginal=marg)
+        em = emulate_layered2(plan, xx, marginal=marg, prec=3)
+        err = np.abs(em - ref) / np.maximum(1.0, np.abs(ref))
+        assert err.max() < 2e-6, err.max()
+
+
 def test_layered2_rejects_outside_constraints():
     from spn_inputs import rat_spn
     p, why = spnb.build_layered2(spnb.Graph(rat_spn(7, F=32, D=2, R=2, S=4, I=12, C=3)))

@@ -617,6 +617,13 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
             r2.ok = false;
             r2.why = "tc_precision 2 (hi/lo) runs on the v1 kernel";
         }
+        // SPNB_R2_RINGS=n_in,n_w (development): try these ring depths first
+        if (const char *ev = getenv("SPNB_R2_RINGS"); ev && r2.ok && !ltc) {
+            int ni = 0, nw = 0;
+            if (sscanf(ev, "%d,%d", &ni, &nw) == 2 && ni >= 2 && ni <= 4 && nw >= 2 && nw <= 8)
+                fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
+                                   r2.max_wgroup, 1, ni, nw, 0, 0, 0) <= smem_optin;
+        }
         for (int a = 0; r2.ok && a < 5 && !fits; ++a)
             fits = rat2_layout(rp, r2.I, r2.max_vars, r2.max_blk, r2.kpad_bot, r2.kpad_up,
                                r2.max_wgroup, 1, ltc ? kRingsT[a][0] : kRings[a][0],

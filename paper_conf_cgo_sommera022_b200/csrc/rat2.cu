@@ -32,6 +32,8 @@
 #include <math_constants.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 #include "layered.h"
 
 namespace spnb {
@@ -62,6 +64,20 @@ constexpr int REG_LEAF = 152, REG_EPI = 152, REG_PROD = 56;
 constexpr int NAB = R2_NAB;
 #ifndef EPI_SHARE
 #define EPI_SHARE 0  // 1: both epilogue warps of a lane quarter drain every group (measured slower)
+#endif
+#ifndef R2_XROWS_CPASYNC
+#define R2_XROWS_CPASYNC 0  // 1: leaf feature rows by cp.async (LSU) instead of per-row bulk copies (TMA)
+#endif
+#ifndef R2_MMA_PERGROUP
+// 1: the MMA warp issues each group as soon as its own accumulator is
+// drained (C5 +5% over waiting for both accumulators of a pair)
+#define R2_MMA_PERGROUP 1
+#endif
+#ifndef R2_MMA_INTERLEAVE
+#define R2_MMA_INTERLEAVE 0  // 1: K-steps of the two accumulators interleaved (round-1 order; measured slower)
+#endif
+#ifndef R2_UPIMG_H
+#define R2_UPIMG_H 0  // epilogue warp (0: accumulator A side, 1: B side) that writes the UP operand image
 #endif
 #ifndef LEAF_SPT
 #define LEAF_SPT 4  // samples per leaf thread (4: one region per 4 warps; 8: per 2 warps, measured no faster)
@@ -118,10 +134,10 @@ __device__ __forceinline__ uint32_t smem_u32(const void *p) {
 __device__ __forceinline__ void bar_init(uint32_t b, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(b), "r"(count));
 }
-// try_wait with a suspend-time hint: a waiting warp is parked by the
-// hardware until the phase completes (or the hint expires) instead of
-// spinning -- spinning producer / MMA warps (the highest warp ids, which the
-// scheduler favours) would otherwise take issue slots from the epilogue
+// plain try_wait (the instruction itself suspends the warp for a
+// hardware-defined time).  Measured alternatives (C5, scripts/gpu/r02_*.sh):
+// a 10 ms suspend-time hint (R2_WAIT_HINT; compiles to a NANOSLEEP.SYNCS
+// loop) -1%, test_wait + nanosleep 32 / 128 ns (R2_WAIT_SLEEP) -4% / -1%.
 // R2_WATCHDOG builds (development): a wait that has not completed after
 // 2^34 cycles (~9 s; a 128-sample tile takes ~6 ms on C5) is a protocol
 // deadlock -- trap so the launch fails instead of hanging the device.  Off
@@ -132,12 +148,33 @@ __device__ __forceinline__ void bar_wait(uint32_t b, uint32_t parity) {
     long long t0 = 0;
 #endif
     while (true) {
+#if defined(R2_WAIT_SLEEP)
+        // poll without parking on the barrier unit: test, then sleep
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}\n"
+            : "=r"(done)
+            : "r"(b), "r"(parity)
+            : "memory");
+        if (done) break;
+        __nanosleep(R2_WAIT_SLEEP);
+        continue;
+#endif
+#ifndef R2_WAIT_HINT
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}\n"
+            : "=r"(done)
+            : "r"(b), "r"(parity)
+            : "memory");
+#else
         asm volatile(
             "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
             "selp.u32 %0, 1, 0, p;\n\t}\n"
             : "=r"(done)
             : "r"(b), "r"(parity), "r"(0x989680u)
             : "memory");
+#endif
         if (done) break;
 #ifdef R2_WATCHDOG
         long long t;
@@ -266,14 +303,33 @@ __device__ __forceinline__ long long clk64() {
     asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
     return t;
 }
+#ifdef R2_TRACE
+// development timeline (R2_TRACE builds with SPNB_PROFILE=1): CTA 0's phase
+// marks as (clock, warp << 8 | phase) pairs in per-warp regions (plain
+// stores, no atomics on the timed path), read back by spnb_r2_trace
+constexpr unsigned TRACE_W = 8192;  // events per warp
+constexpr unsigned TRACE_N = 16 * TRACE_W;
+__device__ unsigned long long g_trace[2 * TRACE_N];
+#endif
 struct Prof {
     unsigned long long *acc;  // shared-memory counters of this role (nullptr: off)
     long long t;
+#ifdef R2_TRACE
+    unsigned cnt = 0;
+#endif
     __device__ Prof(unsigned long long *a, bool on) : acc(on ? a : nullptr), t(clk64()) {}
     __device__ __forceinline__ void mark(int k) {
         if (acc) {
             const long long now = clk64();
+#ifdef R2_TRACE
+            if ((threadIdx.x & 31) == 0 && blockIdx.x == 0 && cnt < TRACE_W) {
+                const unsigned i = (threadIdx.x >> 5) * TRACE_W + cnt++;
+                g_trace[2 * i] = (unsigned long long)now;
+                g_trace[2 * i + 1] = ((threadIdx.x >> 5) << 8) | (unsigned)k;
+            }
+#else
             if ((threadIdx.x & 31) == 0) atomicAdd(acc + k, (unsigned long long)(now - t));
+#endif
             t = now;
         }
     }
@@ -527,6 +583,36 @@ __device__ void leaf_producer_role(const R2Params &p, const Smem &sm, const int3
             const uint32_t full = sm.bar(B_IN_FULL + s);
             const uint32_t pbytes = (uint32_t)st.blk_floats * 4;
             const uint32_t dst = smem_u32(sm.in_x(s));
+#if R2_XROWS_CPASYNC
+            // feature rows through the LSU path (cp.async, 16 B per lane per
+            // row): hundreds of 512-byte bulk copies per tile would queue
+            // ahead of the weight groups in the TMA unit.  Each lane's
+            // cp.async.mbarrier.arrive adds a pending arrival now and
+            // completes it when its copies land, so the slot's phase waits
+            // for them; issued before lane 0's expect_tx arrive.
+            if (!LTC) {
+                for (int v0 = 0; v0 < st.n_vars; v0 += 32) {
+                    const int vl = v0 + lane < st.n_vars ? __ldg(p.vars + st.vars_off + v0 + lane) : 0;
+                    const int nv = min(32, st.n_vars - v0);
+                    for (int v = 0; v < nv; ++v) {
+                        const int f = __shfl_sync(0xffffffffu, vl, v);
+                        const float *src = p.xT + (int64_t)f * p.ldT + base + lane * 4;
+                        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(
+                                         dst + (uint32_t)((v0 + v) * RT * 4 + lane * 16)),
+                                     "l"(src)
+                                     : "memory");
+                    }
+                }
+                asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(full) : "memory");
+                __syncwarp();
+                if (lane == 0) {
+                    bar_expect_tx(full, pbytes);
+                    bulk_g2s(smem_u32(sm.in_prm(s)), p.fparams + st.blk_off, pbytes, full);
+                }
+                __syncwarp();
+                continue;
+            }
+#endif
             if (lane == 0) {
                 if constexpr (LTC) {
                     // centres + the query's parameter image (hi, lo)
@@ -685,7 +771,7 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
             const uint64_t a_desc = a_hi_bits | (uint64_t)((a_addr >> 4) & 0x3FFFu);
             const uint32_t a_lo_d = ((uint32_t)(bot ? p.bimg_bytes : p.uimg_bytes) / 2) >> 4;
             const uint32_t ka_d = (2 * lbo_a) >> 4;
-#if EPI_SHARE
+#if EPI_SHARE || R2_MMA_PERGROUP
             // per group: wait only for this group's accumulator, so group g+1's
             // chain starts while the epilogue still drains the other buffer
             for (int gi = 0; gi < G; ++gi) {
@@ -758,12 +844,21 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                         kw_d[b] = (2 * lbo_b) >> 4;
                         idesc[b] = (1u << 4) | ((uint32_t)(gr[b].ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
                     }
+#ifndef R2_KO_MMA  // knockout (wrong results): commits only, no tensor-core work
+#if R2_MMA_INTERLEAVE
                     for (int kk = 0; kk < ksteps; ++kk) {
-#ifdef R2_KO_MMA  // knockout (wrong results): commits only, no tensor-core work
-                        break;
-#endif
 #pragma unroll
                         for (int b = 0; b < 2; ++b) {
+#else
+                    // each accumulator's K-steps back to back: chained MMAs into
+                    // one accumulator pipeline, while an MMA whose accumulator
+                    // was last written by an earlier, non-adjacent MMA waits for
+                    // it (scripts/micro/umma_issue.cu: 160 vs 294 cycles per MMA
+                    // for two accumulators, K-steps consecutive vs interleaved)
+#pragma unroll
+                    for (int b = 0; b < 2; ++b) {
+                        for (int kk = 0; kk < ksteps; ++kk) {
+#endif
                             if (gr[b].ns > 0) {
                                 const uint32_t d = tmem + (b ? (uint32_t)Cols<LTC>::A : 0u);
                                 const uint64_t ad = a_desc + kk * ka_d, wd = w_desc[b] + kk * kw_d[b];
@@ -775,6 +870,7 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                             }
                         }
                     }
+#endif
                     umma_commit(bar_tfull);
                     umma_commit(bar_tfull + 8u);
 #pragma unroll
@@ -917,11 +1013,19 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         // subtract, store -- measured ~190 cycles; scripts/micro/epi_sum.cu)
         for (int sl = 0; sl < ns; sl += PB) {
             float t[PB * NA], kv[PB];
+#ifdef R2_KO_TLD  // knockout (wrong results): no accumulator reads
+#pragma unroll
+            for (int k = 0; k < PB * NA; ++k) t[k] = __int_as_float(acc + k);
+#else
             ld_cols<PB * NA>(acc + (uint32_t)(sl * NA), t);
+#endif
 #pragma unroll
             for (int k = 0; k < PB; ++k)  // the sums' scale exponents, in flight with the TMEM batch
                 kv[k] = sl + k < ns ? __ldg(ks + gr.s0 + sl + k) : 0.f;
             tmem_wait_ld();
+#ifdef R2_TRACE
+            pf.mark(6);
+#endif
             if (sl + PB >= ns) {
                 tc_fence_before();
                 bar_arrive(sm.bar(B_T_EMPTY + b));  // all of this group's columns are in registers
@@ -937,6 +1041,9 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
 #pragma unroll
             for (int k = 0; k < PB; ++k)
                 if (sl + k < ns) fin(gr.s0 + sl + k, val[k], kv[k]);
+#ifdef R2_TRACE
+            pf.mark(7);
+#endif
         }
         if (ns == 0) {
             tc_fence_before();
@@ -1187,7 +1294,7 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                     hb = maxnan(hb, vb[i]);
                     ha = maxnan(ha, ear[i]);
                 }
-                if (h == 0) {  // one warp of the pair writes the B-side operand image
+                if (h == R2_UPIMG_H) {  // one warp of the pair writes the B-side operand image
                     bar_wait(sm.bar(B_U_EMPTY), (ku & 1u) ^ 1u);
                     uint8_t *img = sm.uimg();
                     const float hc = fmaxf(hb, -1e30f) - EB_SHIFT;
@@ -1343,6 +1450,18 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 }
 
 }  // namespace r2
+
+#ifdef R2_TRACE
+extern "C" int spnb_r2_trace(unsigned long long *out, int max_pairs) {
+    // all per-warp regions (unused entries are zero); clears them
+    const int n = std::min(max_pairs, (int)r2::TRACE_N);
+    cudaMemcpyFromSymbol(out, r2::g_trace, 2 * sizeof(unsigned long long) * n);
+    static unsigned long long zero[2 * 4096];
+    for (unsigned o = 0; o < 2 * r2::TRACE_N; o += 2 * 4096)
+        cudaMemcpyToSymbol(r2::g_trace, zero, sizeof(zero), o * sizeof(unsigned long long));
+    return n;
+}
+#endif
 
 // (I, S) pairs with a compiled kernel instance (S = 0: no sum regions)
 bool rat2_supported_shape(int I, int S) {

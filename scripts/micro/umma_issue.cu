@@ -17,7 +17,7 @@ __device__ __forceinline__ uint64_t desc(uint32_t addr, uint32_t lbo, uint32_t s
     d |= (uint64_t)1 << 46;
     return d;
 }
-__global__ void k(int N, int nacc, int commits, int readers, unsigned long long *cyc) {
+__global__ void k(int N, int nacc, int commits, int readers, unsigned long long *cyc, int seq) {
     extern __shared__ __align__(1024) uint8_t sm[];
     __shared__ uint32_t slot;
     __shared__ __align__(8) uint64_t bar[16];
@@ -46,14 +46,18 @@ __global__ void k(int N, int nacc, int commits, int readers, unsigned long long 
         const uint32_t idesc = (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
         const unsigned long long t0 = clock64();
         for (int it = 0; it < BATCHES; ++it) {
-            for (int kk = 0; kk < kpad / 16; ++kk)
-                for (int q = 0; q < nacc; ++q) {
+            for (int kq = 0; kq < (kpad / 16) * nacc; ++kq) {
+                // seq = 0: K-steps interleaved across the nacc accumulators;
+                // seq = 1: each accumulator's K-steps back to back (groups in turn)
+                const int kk = seq ? kq % (kpad / 16) : kq / nacc, q = seq ? kq / (kpad / 16) : kq % nacc;
+                {
                     const uint32_t b = a + RT * kpad * 2 + q * 256 * kpad * 2;
                     const uint64_t da = desc(a + kk * 2 * lbo_a, lbo_a, 128), db = desc(b + kk * 2 * lbo_b, lbo_b, 128);
                     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                                  "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem + q * N),
                                  "l"(da), "l"(db), "r"(idesc), "r"((uint32_t)(kk > 0)));
                 }
+            }
             for (int c = 0; c < commits; ++c)
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                     (uint32_t)__cvta_generic_to_shared(&bar[c])));
@@ -92,18 +96,19 @@ int main() {
     cudaMalloc(&c, 8 * 1024);
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     const size_t smem = (128 + 4 * 256) * 48 * 2;
+    for (int seq : {0, 1})
     for (int readers : {0, 1})
-        for (int N : {80, 160, 256})
-            for (int nacc : {1, 2, 4})
-                for (int commits : {1, 8}) {
-                    if (nacc * N > 400 || (commits == 8 && nacc == 1)) continue;
-                    k<<<sms, 160, smem>>>(N, nacc, commits, readers, c);
+        for (int N : {80, 96, 128, 160, 240, 256})
+            for (int nacc : {1, 2, 3, 4})
+                for (int commits : {1}) {
+                    if (nacc * N > 512 || (seq && nacc == 1)) continue;
+                    k<<<sms, 160, smem>>>(N, nacc, commits, readers, c, seq);
                     cudaError_t e = cudaDeviceSynchronize();
                     unsigned long long h;
                     cudaMemcpy(&h, c, 8, cudaMemcpyDeviceToHost);
                     const double mmas = (double)BATCHES * nacc * 3;
                     const double flop = mmas * 2.0 * 128 * N * 16;
-                    printf("readers=%d N=%3d acc=%d commits/batch=%d: %6.1f clk/MMA %6.0f flop/clk/SM %s\n", readers, N,
+                    printf("seq=%d readers=%d N=%3d acc=%d commits/batch=%d: %6.1f clk/MMA %6.0f flop/clk/SM %s\n", seq, readers, N,
                            nacc, commits, h / mmas, flop / h, cudaGetErrorString(e));
                 }
     return 0;

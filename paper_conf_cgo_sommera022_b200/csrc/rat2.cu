@@ -73,6 +73,15 @@ constexpr int NAB = R2_NAB;
 // drained (C5 +5% over waiting for both accumulators of a pair)
 #define R2_MMA_PERGROUP 1
 #endif
+#ifndef R2_EPI_RELEASE
+// 1: the epilogue, having observed a group's T_FULL, releases its weight slot
+// (and after the step's last group the step's operand image) with a plain
+// mbarrier arrive, so the MMA warp issues one tcgen05.commit per group
+// instead of two (+ one per step); needs R2_MMA_PERGROUP.  Measured 2%
+// slower on C5 (the release moves onto the epilogue's critical path)
+#define R2_EPI_RELEASE 0
+#endif
+static_assert(!(EPI_SHARE && R2_EPI_RELEASE), "R2_EPI_RELEASE needs one drainer per group");
 #ifndef R2_MMA_INTERLEAVE
 #define R2_MMA_INTERLEAVE 0  // 1: K-steps of the two accumulators interleaved (round-1 order; measured slower)
 #endif
@@ -798,6 +807,7 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                     const uint32_t kw_d = (2 * lbo_b) >> 4;
                     const uint32_t idesc = (1u << 4) | ((uint32_t)(gr.ncol >> 3) << 17) | ((uint32_t)(RT >> 4) << 24);
                     const uint32_t d = tmem + (b ? (uint32_t)Cols<LTC>::A : 0u);
+#ifndef R2_KO_MMA
                     if (gr.ns > 0)
                         for (int kk = 0; kk < ksteps; ++kk) {
                             const uint64_t ad = a_desc + kk * ka_d, wd = w_desc + kk * kw_d;
@@ -807,8 +817,20 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                                 umma_f16(d, ad, wd + wlo_d, idesc, 1);
                             }
                         }
+#endif
+#ifdef R2_TRACE
+                    pf.mark(4);
+#endif
                     umma_commit(bar_tfull + 8u * b);
+#ifdef R2_TRACE
+                    pf.mark(5);
+#endif
+#if !R2_EPI_RELEASE
                     if (gr.ns > 0) umma_commit(bar_wempty + 8u * wsl);
+#endif
+#ifdef R2_TRACE
+                    pf.mark(6);
+#endif
                 }
                 __syncwarp();
                 if (b) ++tp;
@@ -880,8 +902,10 @@ __device__ void mma_role(const R2Params &p, const Smem &sm, const int32_t *sum_s
                 __syncwarp();
             }
 #endif
+#if !R2_EPI_RELEASE
             if (lane == 0) umma_commit(sm.bar(bot ? B_B_EMPTY + (int)(kb % Cols<LTC>::NAB) : B_U_EMPTY));
             __syncwarp();
+#endif
             if (bot) ++kb;
             else ++ku;
             pf.mark(3);
@@ -936,11 +960,17 @@ __device__ __forceinline__ float dot4(const float (&ea)[NA], const float *t) {
     return ((q[0].x + q[0].y) + (q[1].x + q[1].y)) + ((q[2].x + q[2].y) + (q[3].x + q[3].y));
 }
 
+// R2_EPI_RELEASE: lane 0 of the lane-quarter-0 warp draining a group
+// releases that group's weight slot once it has seen the group's T_FULL
+// (the MMAs that read the slot are complete), and the warp draining the
+// step's last group releases the step's operand image (rel_bar); wslot is
+// the weight-ring position of the step's first non-empty group
 template <int NA, bool ROOT, bool LTC>
 __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, const SumStep &st,
                                            const float (&ear)[NA], float shift, uint32_t lane_base,
                                            uint32_t out_col, uint32_t col_root, uint32_t &tp,
-                                           Prof &pf, int h) {
+                                           Prof &pf, int h, uint32_t &wslot, uint32_t rel_bar,
+                                           bool releaser) {
     static_assert(NA % 4 == 0, "region width");
     constexpr int PB = NA >= EPI_COLS ? 1 : EPI_COLS / NA;  // sums per TMEM batch
     const float *ks = p.fparams + st.blk_off;
@@ -998,13 +1028,31 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
     }
     return;
 #endif
-    for (int gi = h; gi < G; gi += 2) {  // this warp's accumulator: groups of parity h
-        const int b = gi & 1;
+#if R2_EPI_RELEASE
+    uint32_t wpos = wslot;  // ring position of group gi's weights (non-empty groups only)
+    const uint32_t n_w = (uint32_t)p.n_w;
+#endif
+    for (int gi = 0; gi < G; ++gi) {
+#if R2_EPI_RELEASE
         const GroupInfo gr = group_info(st, gi);
+        const uint32_t my_w = wpos;
+        if (gr.ns > 0 && ++wpos == n_w) wpos = 0;
+        if ((gi & 1) != h) continue;  // this warp's accumulator: groups of parity h
+#else
+        if ((gi & 1) != h) continue;
+        const GroupInfo gr = group_info(st, gi);
+#endif
+        const int b = gi & 1;
         pf.mark(3);
         bar_wait(sm.bar(B_T_FULL + b), (tp & 1u));
         pf.mark(2);
         tc_fence_after();
+#if R2_EPI_RELEASE
+        if (releaser) {
+            if (gr.ns > 0) bar_arrive(sm.bar(B_W_EMPTY) + 8u * my_w);
+            if (gi == G - 1) bar_arrive(rel_bar);
+        }
+#endif
         const uint32_t acc = lane_base + (b ? (uint32_t)Cols<LTC>::A : 0u);
         const int ns = gr.ns;
         // batches of PB sums (one tcgen05.ld of PB * NA <= 80 columns, one
@@ -1051,6 +1099,9 @@ __device__ __forceinline__ void sum_groups(const R2Params &p, const Smem &sm, co
         }
         ++tp;
     }
+#if R2_EPI_RELEASE
+    wslot = wpos;
+#endif
 }
 
 // ============================================================== LEAF on tensor cores (LTC)
@@ -1252,6 +1303,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
     const uint32_t col_root = col_slots + (uint32_t)(p.D * S);
     const int64_t n_tiles = (p.n + RT - 1) / RT;
     uint32_t kb = 0, ku = 0, tp = 0;
+    uint32_t wslot = 0;                          // weight-ring position (R2_EPI_RELEASE)
+    const bool releaser = qd == 0 && lane == 0;  // releases slots for this warp's groups
     const int part_u = p.uimg_bytes / 2;
     constexpr int SU = S > 0 ? S : 4;
     Prof pf(sm.prof(1), p.prof != nullptr);  // 0 wait leaf outputs, 1 UP phase 1, 2 wait TMEM full, 3 sums, 4 tile I/O, 5 step setup
@@ -1278,9 +1331,10 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 for (int i = 0; i < I; ++i) ear[i] = ea[i * RT + m];
                 const float shift = sm.ha(ab)[m] + sm.hb(ab)[m];
                 bar_arrive(sm.bar(B_A_EMPTY + ab));
+                const uint32_t rel_b = sm.bar(B_B_EMPTY + ab);  // the B image, after the step's MMAs
                 ++kb;
-                if (es.root) sum_groups<I, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
-                else sum_groups<I, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                if (es.root) sum_groups<I, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h, wslot, rel_b, releaser);
+                else sum_groups<I, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h, wslot, rel_b, releaser);
             } else {
                 // UP: children in activation slots; B side -> f16 image, A side -> registers
                 float vb[SU], ear[SU];
@@ -1320,8 +1374,8 @@ __device__ void epilogue_role(const R2Params &p, const Smem &sm, const int32_t *
                 for (int i = 0; i < SU; ++i) ear[i] = ex2(ear[i] - hac);
                 const float shift = ha + hb - EB_SHIFT;
                 pf.mark(1);
-                if (es.root) sum_groups<SU, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
-                else sum_groups<SU, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h);
+                if (es.root) sum_groups<SU, true, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h, wslot, sm.bar(B_U_EMPTY), releaser);
+                else sum_groups<SU, false, LTC>(p, sm, es, ear, shift, lane_base, out_col, col_root, tp, pf, h, wslot, sm.bar(B_U_EMPTY), releaser);
             }
             tmem_wait_st();
         }

@@ -15,7 +15,7 @@ o = np.argsort(t, kind="stable")
 t, w, k = t[o] - t[o][0], w[o], k[o]
 NAMES = {"leaf": {0: "in-wait", 1: "compute", 2: "shift", 3: "out-wait", 4: "exp+write"},
          "epi": {5: "step-setup", 0: "leaf-wait", 1: "up-phase1", 3: "sums", 2: "T_FULL-wait", 4: "tile-io", 6: "tmem-ld", 7: "dots+fin"},
-         12: {7: "issue", 0: "in-slot-wait"}, 13: {0: "A-wait", 3: "issue", 1: "W-wait", 2: "T_EMPTY-wait"},
+         12: {7: "issue", 0: "in-slot-wait"}, 13: {0: "A-wait", 3: "issue", 1: "W-wait", 2: "T_EMPTY-wait", 4: "mma-issue", 5: "commit-T", 6: "commit-W"},
          14: {7: "issue", 2: "W-slot-wait"}}
 
 

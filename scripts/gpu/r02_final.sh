@@ -1,0 +1,18 @@
+#!/bin/bash
+# r02 final evidence on HEAD: GPU tests, smoke, bench lines (default C5 + configs + reference arm),
+# C5 launch list, ncu --set full of the v2 kernel on C5, compute-sanitizer on the v2 kernel
+cd "${GRAFT_REPO_ROOT:-/root/repo}"
+O=gpurun_out/r02_final; mkdir -p $O; : > $O/status.txt
+python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1; echo "build=$?" >> $O/status.txt
+timeout 2400 python -m pytest tests -m gpu -q --timeout 1200 > $O/pytest_gpu.log 2>&1; echo "pytest=$?" >> $O/status.txt
+timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke=$?" >> $O/status.txt
+timeout 1200 python bench.py > $O/bench_C5.log 2>&1; echo "bench_C5=$?" >> $O/status.txt
+for a in "C4" "C4 --marginal" "C2" "C2 --marginal" "C3 --marginal" "C1 --samples 100000000" "C1 --marginal --samples 100000000"; do
+  n=$(echo $a | tr -d ' -' | sed 's/samples100000000/_1e8/'); timeout 900 python bench.py --config $a > $O/bench_$n.log 2>&1; echo "bench_$n=$?" >> $O/status.txt
+done
+timeout 900 python bench.py --impl reference > $O/bench_reference.log 2>&1; echo "bench_reference=$?" >> $O/status.txt
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv --log-file $O/launches_C5.csv python bench.py --steps 1 --warmup 3 > $O/ncu_l_C5.log 2>&1; echo "ncul_C5=$?" >> $O/status.txt
+SPNB_PROFILE=0 timeout 900 bash scripts/gpu/ncu_cap.sh $O/C5v2 rat2 0 1 python scripts/profile_layered.py C5 0; echo "ncu_C5=$?" >> $O/status.txt
+timeout 600 compute-sanitizer --tool memcheck --error-exitcode 9 python scripts/sanitize_cases.py v2 > $O/v2_memcheck.log 2>&1; echo "v2_memcheck=$?" >> $O/status.txt
+timeout 600 compute-sanitizer --tool synccheck --error-exitcode 9 python scripts/sanitize_cases.py v2 > $O/v2_synccheck.log 2>&1; echo "v2_synccheck=$?" >> $O/status.txt
+echo done >> $O/status.txt

@@ -118,7 +118,7 @@ typedef struct spn_prepare_options {
                                    against the Gaussians' expanded constants,
                                    f16 hi/lo split, fp32 accumulation in TMEM).
                                    0 auto (= off: measured slower than the FMA
-                                   leaves on C4/C5, DESIGN.md §5.3.6), 1 off
+                                   leaves on C4/C5, DESIGN.md §5.3.5), 1 off
                                    (FP32 FMA leaves), 2 on (needs tc_precision
                                    0: the certification recomputes inputs
                                    outside the split's range; E_UNSUPPORTED if

@@ -574,7 +574,7 @@ int prepare_layered(const GraphData &g, const LayeredPlan &lp, const spn_prepare
     if (want_r2 != 1) {
         Rat2Plan r2;
         // tensor-core leaves (opt-in, leaf_tc 2): measured slower than the FMA
-        // leaves on C4 / C5 (DESIGN.md §5.3.6), so auto keeps the FMA leaves;
+        // leaves on C4 / C5 (DESIGN.md §5.3.5), so auto keeps the FMA leaves;
         // they need the certification (it recomputes the inputs outside the
         // split operands' range)
         const bool try_ltc = opt.leaf_tc == 2;

@@ -788,6 +788,8 @@ int prepare_compiled(const GraphData &g, const spn_prepare_options &opt, int dev
     // 1.42e9 vs 3.6e9 samples/s on C2)
     if ((int64_t)g.kind.size() <= 64) jo.samples_per_thread = 4;
     if (const char *e = getenv("SPNB_JIT_K")) jo.samples_per_thread = std::min(4, std::max(1, atoi(e)));
+    // SPNB_JIT_TASKCAP (development): pack connected components up to this many nodes per kernel
+    if (const char *e = getenv("SPNB_JIT_TASKCAP")) jo.task_cap_nodes = std::max<int64_t>(1, atoll(e));
     if (const char *e = getenv("SPNB_JIT_BAR")) jo.bar_every = std::max(0, atoi(e));
     JitProgram jp;
     std::string msg;

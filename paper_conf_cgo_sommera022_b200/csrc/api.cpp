@@ -103,6 +103,13 @@ struct DevicePlan {
     float *hout[2] = {nullptr, nullptr};
     int32_t *ham[2] = {nullptr, nullptr};
     int64_t host_chunk = 0;
+    // certified layered plans: whole groups of host rows resident on the
+    // device (one certification round per group instead of one per chunk)
+    float *gx = nullptr, *gout = nullptr;
+    int32_t *gam = nullptr;
+    int64_t group_cap = 0;
+    std::vector<cudaEvent_t> gev;  // per transposed chunk: its rows have landed
+    cudaEvent_t gdone = nullptr;   // the group's kernels no longer read gx
     // layered (RAT-SPN) path
     int path = 0;
     LStep *d_steps = nullptr;
@@ -246,6 +253,13 @@ void free_plan(DevicePlan *p) {
     for (int i = 0; i < 2; ++i) {
         if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
         cudaFree(p->hx[i]);
+        if (i == 0) {
+            cudaFree(p->gx);
+            cudaFree(p->gout);
+            cudaFree(p->gam);
+            for (cudaEvent_t ev : p->gev) cudaEventDestroy(ev);
+            if (p->gdone) cudaEventDestroy(p->gdone);
+        }
         cudaFree(p->hout[i]);
         cudaFree(p->ham[i]);
     }
@@ -280,7 +294,8 @@ int upload(T **dst, const std::vector<T> &v) {
 }
 
 int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
-                      int32_t *argmax, void *stream, bool marg);
+                      int32_t *argmax, void *stream, bool marg,
+                      const cudaEvent_t *ready = nullptr);
 
 int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                  int32_t *argmax, void *stream, bool marg) {
@@ -331,7 +346,8 @@ RParams v1_params(const DevicePlan &P) {
 }
 
 int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
-                      int32_t *argmax, void *stream, bool marg) {
+                      int32_t *argmax, void *stream, bool marg,
+                      const cudaEvent_t *ready) {
     if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
     DevicePlan &P = *h->plan;
     if (n < 0) return set_err(SPN_E_ARG, "n < 0");
@@ -385,8 +401,11 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
             rp.row0 = c0;
             const int64_t m = std::min(P.chunk, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
-            cudaError_t e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
-                                             (cudaStream_t)stream);
+            // host pipeline: this chunk's rows are still being copied in
+            if (ready && (e = cudaStreamWaitEvent((cudaStream_t)stream, ready[c0 / P.chunk], 0)) != cudaSuccess)
+                return cuda_err(e, "cudaStreamWaitEvent");
+            e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
+                                 (cudaStream_t)stream);
             if (e != cudaSuccess) return cuda_err(e, "transpose launch");
             rp.n = m;
             rp.out = out + c0 * P.R;
@@ -471,6 +490,83 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
     return launch_kernel(kp, P.K, marg, P.xs, grid, P.block, P.smem, (cudaStream_t)stream);
 }
 
+// Host pipeline of a certified layered v2 plan.  Its certification
+// recomputes flagged samples with the v1 kernel, whose latency is about one
+// 128-sample tile (~20 ms on C5) however few samples are flagged, so one
+// round per transposed chunk (~46 ms of work) would cost ~40%.  Instead a
+// whole group of host rows (up to ~4 GB of features) is kept on the device:
+// the copy stream lands it chunk by chunk (an event per chunk), the compute
+// stream starts each chunk as soon as its rows are in, and the group ends
+// with one certification round and one copy of the outputs back.
+int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, int64_t ld,
+                       float *out, int32_t *argmax, bool marg) {
+    cudaError_t e;
+    if (!P.gx) {
+        const int64_t per_chunk = P.chunk * P.F * 4;
+        int64_t chunks = std::max<int64_t>(1, ((int64_t)4 << 30) / per_chunk);
+        // SPNB_HOST_GROUP_CHUNKS (tests): smaller groups, to cover several groups per call
+        if (const char *ev = getenv("SPNB_HOST_GROUP_CHUNKS")) chunks = std::max(1, atoi(ev));
+        P.group_cap = chunks * P.chunk;
+        if ((e = cudaMalloc(&P.gx, (size_t)P.group_cap * P.F * 4)) != cudaSuccess ||
+            (e = cudaMalloc(&P.gout, (size_t)P.group_cap * P.R * 4)) != cudaSuccess ||
+            (e = cudaMalloc(&P.gam, (size_t)P.group_cap * 4)) != cudaSuccess)
+            return set_err(SPN_E_OOM, "host pipeline group buffers");
+        P.gev.resize((size_t)chunks);
+        for (auto &ev : P.gev)
+            if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess)
+                return cuda_err(e, "cudaEventCreate");
+        if ((e = cudaEventCreateWithFlags(&P.gdone, cudaEventDisableTiming)) != cudaSuccess)
+            return cuda_err(e, "cudaEventCreate");
+    }
+    cudaStream_t cp = P.hs[0], cs = P.hs[1];
+    bool first = true;
+    for (int64_t g0 = 0; g0 < n; g0 += P.group_cap) {
+        const int64_t m = std::min(P.group_cap, n - g0);
+        // the previous group's kernels and output copies are done with gx / gout
+        if (!first && (e = cudaStreamWaitEvent(cp, P.gdone, 0)) != cudaSuccess)
+            return cuda_err(e, "cudaStreamWaitEvent");
+        first = false;
+        for (int64_t c0 = 0; c0 < m; c0 += P.chunk) {
+            const int64_t mc = std::min(P.chunk, m - c0);
+            const float *src = x + (g0 + c0) * ld;
+            if (ld == P.F)
+                e = cudaMemcpyAsync(P.gx + c0 * P.F, src, (size_t)mc * P.F * 4, cudaMemcpyHostToDevice, cp);
+            else
+                e = cudaMemcpy2DAsync(P.gx + c0 * P.F, (size_t)P.F * 4, src, (size_t)ld * 4,
+                                      (size_t)P.F * 4, (size_t)mc, cudaMemcpyHostToDevice, cp);
+            if (e != cudaSuccess) return cuda_err(e, "H2D");
+            if ((e = cudaEventRecord(P.gev[(size_t)(c0 / P.chunk)], cp)) != cudaSuccess)
+                return cuda_err(e, "cudaEventRecord");
+        }
+        int rc;
+        {
+            // same scratch ordering as infer_device (another stream's call may still use it)
+            std::lock_guard<std::mutex> lk(P.scratch_mu);
+            if (P.scratch_ev && P.scratch_stream != (void *)cs &&
+                (e = cudaStreamWaitEvent(cs, P.scratch_ev, 0)) != cudaSuccess)
+                return cuda_err(e, "cudaStreamWaitEvent");
+            rc = infer_device_impl(h, P.gx, m, P.F, P.gout, argmax ? P.gam : nullptr, cs, marg,
+                                   P.gev.data());
+            if (rc != SPN_OK) return rc;
+            if (!P.scratch_ev &&
+                (e = cudaEventCreateWithFlags(&P.scratch_ev, cudaEventDisableTiming)) != cudaSuccess)
+                return cuda_err(e, "cudaEventCreate");
+            if ((e = cudaEventRecord(P.scratch_ev, cs)) != cudaSuccess) return cuda_err(e, "cudaEventRecord");
+            P.scratch_stream = cs;
+        }
+        if ((e = cudaMemcpyAsync(out + g0 * P.R, P.gout, (size_t)m * P.R * 4, cudaMemcpyDeviceToHost, cs)) !=
+            cudaSuccess)
+            return cuda_err(e, "D2H");
+        if (argmax && (e = cudaMemcpyAsync(argmax + g0, P.gam, (size_t)m * 4, cudaMemcpyDeviceToHost, cs)) !=
+                          cudaSuccess)
+            return cuda_err(e, "D2H argmax");
+        if ((e = cudaEventRecord(P.gdone, cs)) != cudaSuccess) return cuda_err(e, "cudaEventRecord");
+    }
+    for (int i = 0; i < 2; ++i)
+        if ((e = cudaStreamSynchronize(P.hs[i])) != cudaSuccess) return cuda_err(e, "sync");
+    return SPN_OK;
+}
+
 int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out, int32_t *argmax,
                bool marg) {
     if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
@@ -482,6 +578,7 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
     std::lock_guard<std::mutex> lk(P.host_mu);
     DeviceGuard dg(P.device);
     cudaError_t e;
+    const bool grouped = P.path == 1 && P.r2 && P.cert;
     if (!P.hs[0]) {
         // chunk sized to ~32 MB of features: big enough to amortise launches,
         // small enough to overlap H2D / kernel / D2H across the two streams
@@ -492,12 +589,14 @@ int infer_host(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
         for (int i = 0; i < 2; ++i) {
             if ((e = cudaStreamCreateWithFlags(&P.hs[i], cudaStreamNonBlocking)) != cudaSuccess)
                 return cuda_err(e, "cudaStreamCreate");
+            if (grouped) continue;  // infer_host_grouped allocates its own buffers
             if ((e = cudaMalloc(&P.hx[i], (size_t)P.host_chunk * P.F * 4)) != cudaSuccess ||
                 (e = cudaMalloc(&P.hout[i], (size_t)P.host_chunk * P.R * 4)) != cudaSuccess ||
                 (e = cudaMalloc(&P.ham[i], (size_t)P.host_chunk * 4)) != cudaSuccess)
                 return set_err(SPN_E_OOM, "host pipeline buffers");
         }
     }
+    if (grouped) return infer_host_grouped(P, h, x, n, ld, out, argmax, marg);
     const int64_t C = P.host_chunk;
     int rc = SPN_OK;
     for (int64_t c0 = 0, i = 0; c0 < n; c0 += C, ++i) {

@@ -513,3 +513,34 @@ def test_host_api_matches_oracle(which):
     ref, am_ref = oracle_eval(g, x[idx])
     _cmp(out[idx], ref)
     _cmp_argmax(am[idx], ref, am_ref)
+
+
+def test_host_api_layered_certified_groups(monkeypatch):
+    """Certified layered plans pipeline host rows group-wise (one
+    certification round per group, api.cpp infer_host_grouped): several
+    groups of one transposed chunk each plus a ragged tail, joint and
+    marginal, bitwise equal to the device-buffer call and within tolerance
+    of the oracle on rows of every group."""
+    from spn_inputs import config_graph, uniform_chunked
+    monkeypatch.setenv("SPNB_HOST_GROUP_CHUNKS", "1")
+    g = config_graph("C4")
+    G = spnb.Graph(g)
+    P = spnb.Plan(G)
+    info = P.info()
+    assert info["path"] == 1 and info["layered_kernel"] == 2 and info["certified"] == 1
+    c = info["chunk_samples"]
+    n = 2 * c + 7_777
+    x = uniform_chunked(n, g.n_features, 4242)   # the bench's inputs: mostly certified
+    x[::997] = ancestral_sample(g, len(x[::997]), 4243)[0]  # some rows the v1 recompute serves
+    x[::97, 5] = np.nan
+    xh = torch.from_numpy(x).pin_memory()
+    for marginal in (False, True):
+        dev, amd = P.infer(torch.from_numpy(x).cuda(), marginal=marginal)
+        out, am = P.infer_host(xh, marginal=marginal)
+        assert np.array_equal(out, dev.cpu().numpy(), equal_nan=True)
+        assert np.array_equal(am, amd.cpu().numpy())
+        idx = np.concatenate([np.arange(0, 8), np.arange(c - 4, c + 4), np.arange(2 * c - 4, 2 * c + 4),
+                              np.arange(n - 8, n)])
+        ref, am_ref = oracle_eval(g, x[idx], marginal=marginal)
+        _cmp(out[idx], ref)
+        _cmp_argmax(am[idx], ref, am_ref)

@@ -249,6 +249,12 @@ int spn_infer_marginal(spn_handle *plan, const float *x, int64_t n, int64_t ld,
  * device->host copies on its own streams (the paper's host<->device data
  * movement, >60% of GPU time, L448-454).  Synchronous: returns when out_host
  * is filled.  Pinned (page-locked) host memory gives full overlap.
+ * Certified layered plans (spn_plan_stats.certified) keep whole groups of up
+ * to ~4 GB of rows on the device (allocated on first use, freed with the
+ * plan): rows land in pieces of one tile per SM, each piece's kernel starts
+ * when its rows are in, and the group ends with one certification round and
+ * one copy of its outputs, so the result equals spn_infer_* on the same rows
+ * bit for bit.
  */
 int spn_infer_joint_host(spn_handle *plan, const float *x_host, int64_t n, int64_t ld,
                          float *out_host, int32_t *argmax_host);

@@ -107,8 +107,8 @@ struct DevicePlan {
     // device (one certification round per group instead of one per chunk)
     float *gx = nullptr, *gout = nullptr;
     int32_t *gam = nullptr;
-    int64_t group_cap = 0;
-    std::vector<cudaEvent_t> gev;  // per transposed chunk: its rows have landed
+    int64_t group_cap = 0, group_piece = 0;
+    std::vector<cudaEvent_t> gev;  // per piece (group_piece rows): its rows have landed
     cudaEvent_t gdone = nullptr;   // the group's kernels no longer read gx
     // layered (RAT-SPN) path
     int path = 0;
@@ -295,7 +295,7 @@ int upload(T **dst, const std::vector<T> &v) {
 
 int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                       int32_t *argmax, void *stream, bool marg,
-                      const cudaEvent_t *ready = nullptr);
+                      const cudaEvent_t *ready = nullptr, int64_t lchunk = 0);
 
 int infer_device(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                  int32_t *argmax, void *stream, bool marg) {
@@ -347,7 +347,7 @@ RParams v1_params(const DevicePlan &P) {
 
 int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, float *out,
                       int32_t *argmax, void *stream, bool marg,
-                      const cudaEvent_t *ready) {
+                      const cudaEvent_t *ready, int64_t lchunk) {
     if (!h || h->magic != H_PLAN) return set_err(SPN_E_ARG, "not a plan handle");
     DevicePlan &P = *h->plan;
     if (n < 0) return set_err(SPN_E_ARG, "n < 0");
@@ -397,12 +397,14 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
             // arithmetic both precisions share (measured 2.2e-7 relative on C4, hi/lo vs oracle)
             rp.cert_tol = 0.9e-4f;
         }
-        for (int64_t c0 = 0; c0 < n; c0 += P.chunk) {
+        // launch chunk: the transposed-scratch capacity, or (host pipeline)
+        // smaller pieces that start as soon as their rows have landed
+        const int64_t LC = lchunk > 0 ? std::min(lchunk, P.chunk) : P.chunk;
+        for (int64_t c0 = 0; c0 < n; c0 += LC) {
             rp.row0 = c0;
-            const int64_t m = std::min(P.chunk, n - c0);
+            const int64_t m = std::min(LC, n - c0);
             const int64_t rows_pad = (m + 127) / 128 * 128;
-            // host pipeline: this chunk's rows are still being copied in
-            if (ready && (e = cudaStreamWaitEvent((cudaStream_t)stream, ready[c0 / P.chunk], 0)) != cudaSuccess)
+            if (ready && (e = cudaStreamWaitEvent((cudaStream_t)stream, ready[c0 / LC], 0)) != cudaSuccess)
                 return cuda_err(e, "cudaStreamWaitEvent");
             e = transpose_launch(x + c0 * ld, m, ld, P.F, P.d_xT, P.chunk, rows_pad,
                                  (cudaStream_t)stream);
@@ -507,6 +509,10 @@ int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, 
         // SPNB_HOST_GROUP_CHUNKS (tests): smaller groups, to cover several groups per call
         if (const char *ev = getenv("SPNB_HOST_GROUP_CHUNKS")) chunks = std::max(1, atoi(ev));
         P.group_cap = chunks * P.chunk;
+        // copies and launches in pieces of one 128-sample tile per CTA, so the
+        // first launch waits for ~1/8 of a transposed chunk, not all of it
+        P.group_piece = std::max<int64_t>(128, P.chunk / 8 / 128 * 128);
+        chunks = (P.group_cap + P.group_piece - 1) / P.group_piece;
         if ((e = cudaMalloc(&P.gx, (size_t)P.group_cap * P.F * 4)) != cudaSuccess ||
             (e = cudaMalloc(&P.gout, (size_t)P.group_cap * P.R * 4)) != cudaSuccess ||
             (e = cudaMalloc(&P.gam, (size_t)P.group_cap * 4)) != cudaSuccess)
@@ -526,8 +532,8 @@ int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, 
         if (!first && (e = cudaStreamWaitEvent(cp, P.gdone, 0)) != cudaSuccess)
             return cuda_err(e, "cudaStreamWaitEvent");
         first = false;
-        for (int64_t c0 = 0; c0 < m; c0 += P.chunk) {
-            const int64_t mc = std::min(P.chunk, m - c0);
+        for (int64_t c0 = 0; c0 < m; c0 += P.group_piece) {
+            const int64_t mc = std::min(P.group_piece, m - c0);
             const float *src = x + (g0 + c0) * ld;
             if (ld == P.F)
                 e = cudaMemcpyAsync(P.gx + c0 * P.F, src, (size_t)mc * P.F * 4, cudaMemcpyHostToDevice, cp);
@@ -535,7 +541,7 @@ int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, 
                 e = cudaMemcpy2DAsync(P.gx + c0 * P.F, (size_t)P.F * 4, src, (size_t)ld * 4,
                                       (size_t)P.F * 4, (size_t)mc, cudaMemcpyHostToDevice, cp);
             if (e != cudaSuccess) return cuda_err(e, "H2D");
-            if ((e = cudaEventRecord(P.gev[(size_t)(c0 / P.chunk)], cp)) != cudaSuccess)
+            if ((e = cudaEventRecord(P.gev[(size_t)(c0 / P.group_piece)], cp)) != cudaSuccess)
                 return cuda_err(e, "cudaEventRecord");
         }
         int rc;
@@ -546,7 +552,7 @@ int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, 
                 (e = cudaStreamWaitEvent(cs, P.scratch_ev, 0)) != cudaSuccess)
                 return cuda_err(e, "cudaStreamWaitEvent");
             rc = infer_device_impl(h, P.gx, m, P.F, P.gout, argmax ? P.gam : nullptr, cs, marg,
-                                   P.gev.data());
+                                   P.gev.data(), P.group_piece);
             if (rc != SPN_OK) return rc;
             if (!P.scratch_ev &&
                 (e = cudaEventCreateWithFlags(&P.scratch_ev, cudaEventDisableTiming)) != cudaSuccess)

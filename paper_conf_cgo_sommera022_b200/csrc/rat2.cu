@@ -89,7 +89,10 @@ static_assert(!(EPI_SHARE && R2_EPI_RELEASE), "R2_EPI_RELEASE needs one drainer 
 #define R2_UPIMG_H 0  // epilogue warp (0: accumulator A side, 1: B side) that writes the UP operand image
 #endif
 #ifndef LEAF_SPT
-#define LEAF_SPT 4  // samples per leaf thread (4: one region per 4 warps; 8: per 2 warps, measured no faster)
+// samples per leaf thread: 8 = one region per 2 warps, the two leaf pairs on
+// alternate (left / right) regions (C5 +4%, C4 +5% over 4 = one region per
+// 4 warps once the MMA issues per group; scripts/gpu/r02/r02_leaf.sh)
+#define LEAF_SPT 8
 #endif
 constexpr int NTHREADS = (4 * NLG + 12) * 32;
 // registers per thread of the launch (65536 / NTHREADS rounded down to 8):
@@ -1439,9 +1442,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             bar_init(sm.bar(B_W_EMPTY + i), 1);
         }
         for (int i = 0; i < Cols<LTC>::NAB; ++i) {
-            bar_init(sm.bar(B_A_FULL + i), WPG * 32);  // the threads of one leaf group (LTC: 128)
+            // the threads of one leaf group (LTC: the 128 leaf threads, one per sample)
+            bar_init(sm.bar(B_A_FULL + i), LTC ? 128 : WPG * 32);
             bar_init(sm.bar(B_A_EMPTY + i), 256);  // both epilogue warps of each quarter
-            bar_init(sm.bar(B_B_FULL + i), WPG * 32);
+            bar_init(sm.bar(B_B_FULL + i), LTC ? 128 : WPG * 32);
             bar_init(sm.bar(B_B_EMPTY + i), 1);
         }
         for (int i = 0; i < 2; ++i) {

@@ -457,6 +457,27 @@ def test_c5_layered_full_graph_sampled():
     _cmp_argmax(am[idx], ref, am_ref)
 
 
+def test_c5_layered_marginal_sampled():
+    """Config 5 graph on the layered path (default plan: certified single
+    f16 pass) with 20% missing features: marginal query on ancestral samples
+    and on the bench's U[0,1] inputs, oracle on rows of both."""
+    from spn_inputs import config_graph, uniform_chunked
+    g = config_graph("C5")
+    P = spnb.Plan(spnb.Graph(g))
+    assert P.info()["path"] == 1 and P.info()["layered_kernel"] == 2
+    xa, _ = ancestral_sample(g, 4000, 5005)
+    xu = uniform_chunked(20_000, g.n_features, 5006)
+    for x, seed in ((xa, 5007), (xu, 5008)):
+        x = nan_mask(x, 0.2, seed)
+        out, am = P.infer(torch.from_numpy(x).cuda(), marginal=True)
+        torch.cuda.synchronize()
+        out, am = out.cpu().numpy(), am.cpu().numpy()
+        idx = np.random.default_rng(seed).choice(len(x), 24, replace=False)
+        ref, am_ref = oracle_eval(g, x[idx], marginal=True)
+        _cmp(out[idx], ref)
+        _cmp_argmax(am[idx], ref, am_ref)
+
+
 def test_c5_partitioned_generic_vs_layered_vs_oracle():
     """BASELINE configs[4] "partitioned into tasks": the C5 graph through the
     generic interpreter with the paper's <= 10k-operation tasks (PAPER.md

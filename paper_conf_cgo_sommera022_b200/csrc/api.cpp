@@ -503,25 +503,50 @@ int infer_device_impl(spn_handle *h, const float *x, int64_t n, int64_t ld, floa
 int infer_host_grouped(DevicePlan &P, spn_handle *h, const float *x, int64_t n, int64_t ld,
                        float *out, int32_t *argmax, bool marg) {
     cudaError_t e;
-    if (!P.gx) {
-        const int64_t per_chunk = P.chunk * P.F * 4;
-        int64_t chunks = std::max<int64_t>(1, ((int64_t)4 << 30) / per_chunk);
-        // SPNB_HOST_GROUP_CHUNKS (tests): smaller groups, to cover several groups per call
-        if (const char *ev = getenv("SPNB_HOST_GROUP_CHUNKS")) chunks = std::max(1, atoi(ev));
-        P.group_cap = chunks * P.chunk;
+    const int64_t per_chunk = P.chunk * P.F * 4;
+    int64_t max_chunks = std::max<int64_t>(1, ((int64_t)4 << 30) / per_chunk);
+    // SPNB_HOST_GROUP_CHUNKS (tests): smaller groups, to cover several groups per call
+    if (const char *ev = getenv("SPNB_HOST_GROUP_CHUNKS")) max_chunks = std::max(1, atoi(ev));
+    // groups as large as this call needs (up to ~4 GB of rows): (re)allocated
+    // when a call needs more than the current buffers hold, halved while the
+    // device is short of memory (down to one transposed chunk)
+    const int64_t want = std::min<int64_t>(max_chunks, std::max<int64_t>(1, (n + P.chunk - 1) / P.chunk));
+    if (!P.gx || want * P.chunk > P.group_cap) {
+        if (P.gx) {
+            for (int i = 0; i < 2; ++i) cudaStreamSynchronize(P.hs[i]);  // (an earlier call may have failed midway)
+            cudaFree(P.gx);
+            cudaFree(P.gout);
+            cudaFree(P.gam);
+            P.gx = nullptr;
+            P.gout = nullptr;
+            P.gam = nullptr;
+            for (cudaEvent_t ev : P.gev) cudaEventDestroy(ev);
+            P.gev.clear();
+        }
+        for (int64_t chunks = want;; chunks = (chunks + 1) / 2) {
+            P.group_cap = chunks * P.chunk;
+            if (cudaMalloc(&P.gx, (size_t)P.group_cap * P.F * 4) == cudaSuccess &&
+                cudaMalloc(&P.gout, (size_t)P.group_cap * P.R * 4) == cudaSuccess &&
+                cudaMalloc(&P.gam, (size_t)P.group_cap * 4) == cudaSuccess)
+                break;
+            cudaFree(P.gx);
+            cudaFree(P.gout);
+            cudaFree(P.gam);
+            P.gx = nullptr;
+            P.gout = nullptr;
+            P.gam = nullptr;
+            P.group_cap = 0;
+            cudaGetLastError();  // clear the allocation error
+            if (chunks == 1) return set_err(SPN_E_OOM, "host pipeline group buffers");
+        }
         // copies and launches in pieces of one 128-sample tile per CTA, so the
         // first launch waits for ~1/8 of a transposed chunk, not all of it
         P.group_piece = std::max<int64_t>(128, P.chunk / 8 / 128 * 128);
-        chunks = (P.group_cap + P.group_piece - 1) / P.group_piece;
-        if ((e = cudaMalloc(&P.gx, (size_t)P.group_cap * P.F * 4)) != cudaSuccess ||
-            (e = cudaMalloc(&P.gout, (size_t)P.group_cap * P.R * 4)) != cudaSuccess ||
-            (e = cudaMalloc(&P.gam, (size_t)P.group_cap * 4)) != cudaSuccess)
-            return set_err(SPN_E_OOM, "host pipeline group buffers");
-        P.gev.resize((size_t)chunks);
+        P.gev.resize((size_t)((P.group_cap + P.group_piece - 1) / P.group_piece), nullptr);
         for (auto &ev : P.gev)
             if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess)
                 return cuda_err(e, "cudaEventCreate");
-        if ((e = cudaEventCreateWithFlags(&P.gdone, cudaEventDisableTiming)) != cudaSuccess)
+        if (!P.gdone && (e = cudaEventCreateWithFlags(&P.gdone, cudaEventDisableTiming)) != cudaSuccess)
             return cuda_err(e, "cudaEventCreate");
     }
     cudaStream_t cp = P.hs[0], cs = P.hs[1];

@@ -555,9 +555,13 @@ def test_host_api_layered_certified_groups(monkeypatch):
     x[::997] = ancestral_sample(g, len(x[::997]), 4243)[0]  # some rows the v1 recompute serves
     x[::97, 5] = np.nan
     xh = torch.from_numpy(x).pin_memory()
+    # a small call first (buffers sized for it), then the full call regrows them
+    small, _ = P.infer_host(torch.from_numpy(x[:1000]).pin_memory())
     for marginal in (False, True):
         dev, amd = P.infer(torch.from_numpy(x).cuda(), marginal=marginal)
         out, am = P.infer_host(xh, marginal=marginal)
+        if not marginal:
+            assert np.array_equal(small, out[:1000], equal_nan=True)
         assert np.array_equal(out, dev.cpu().numpy(), equal_nan=True)
         assert np.array_equal(am, amd.cpu().numpy())
         idx = np.concatenate([np.arange(0, 8), np.arange(c - 4, c + 4), np.arange(2 * c - 4, 2 * c + 4),
